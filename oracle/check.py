@@ -1,0 +1,111 @@
+"""Invariants every valid scheduled-permutation plan satisfies. ORACLE — test infrastructure only.
+
+A plan is (kappa, {(sigma_phi, t_phi)}_{phi=1,2,3}) on an r x c view. The
+checker rebuilds Phi1..Phi3 from kappa and p itself (it never trusts a
+plan's own phase arrays) and verifies, vectorised so it scales to any n:
+
+ (i)   kappa restricted to each row is a bijection onto [0, c)        (L537 (1))
+ (ii)  within each colour class the destination rows are distinct      (L537 (2))
+ (iii) every Phi restricted to every line is a bijection               (L517)
+ (iv)  routing x through Phi1, Phi2, Phi3 lands at P(x)                (L539)
+ (v)   t = Phi(s) slot by slot, with s = w*sigma + lane                (L519)
+ (vi)  every warp-round reads w distinct banks and writes w distinct
+       banks                                                           (L531-L533, L213)
+ (vii) the s of each line cover [0, L) exactly once                   (L521-L525)
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+def phases_from_kappa(p: np.ndarray, kappa: np.ndarray, rows: int, cols: int):
+    """Phi1 (r,c), Phi2 (c,r), Phi3 (r,c) from kappa and P (L537-L539), vectorised."""
+    p = np.asarray(p, dtype=np.int64)
+    kappa = np.asarray(kappa, dtype=np.int64)
+    n = rows * cols
+    x = np.arange(n, dtype=np.int64)
+    src_row = x // cols
+    dest_row, dest_col = p // cols, p % cols
+    phi1 = kappa.reshape(rows, cols).copy()
+    phi2 = np.full((cols, rows), -1, dtype=np.int64)
+    phi3 = np.full((rows, cols), -1, dtype=np.int64)
+    phi2[kappa, src_row] = dest_row
+    phi3[dest_row, kappa] = dest_col
+    return phi1, phi2, phi3
+
+
+def _rows_are_perms(m: np.ndarray) -> bool:
+    L = m.shape[1]
+    if m.min() < 0 or m.max() >= L:
+        return False
+    s = np.sort(m, axis=1)
+    return bool(np.all(s == np.arange(L, dtype=s.dtype)[None, :]))
+
+
+def _rounds_distinct(v: np.ndarray, w: int) -> bool:
+    """v shape (lines, L): every group of w consecutive slots has distinct v mod w."""
+    lines, L = v.shape
+    b = np.sort((v % w).reshape(lines, L // w, w), axis=2)
+    return bool(np.all(b == np.arange(w)[None, None, :]))
+
+
+def check_plan(p, kappa, sched, rows: int, cols: int, w: int) -> dict:
+    """Return {invariant: bool}. ``sched`` = [(sigma1, t1), (sigma2, t2), (sigma3, t3)]
+    with shapes (r, c), (c, r), (r, c) in logical [line][slot] order."""
+    p = np.asarray(p, dtype=np.int64)
+    kappa = np.asarray(kappa, dtype=np.int64)
+    n = rows * cols
+    res = {}
+    res["shape"] = (p.size == n and kappa.size == n)
+    if not res["shape"]:
+        return res
+    # (i)
+    res["i_row_colours_bijective"] = _rows_are_perms(kappa.reshape(rows, cols))
+    # (ii)
+    key = kappa * rows + p // cols
+    res["ii_colour_dest_rows_distinct"] = bool(
+        kappa.min() >= 0 and kappa.max() < cols and np.unique(key).size == n)
+    if not (res["i_row_colours_bijective"] and res["ii_colour_dest_rows_distinct"]):
+        return res
+    phis = phases_from_kappa(p, kappa, rows, cols)
+    # (iii)
+    res["iii_phases_bijective"] = all(_rows_are_perms(ph) for ph in phis)
+    # (iv)
+    x = np.arange(n, dtype=np.int64)
+    i, j = x // cols, x % cols
+    k = phis[0][i, j]
+    row2 = phis[1][k, i]
+    col3 = phis[2][row2, k]
+    res["iv_composition_is_P"] = bool(np.all(row2 * cols + col3 == p))
+    ok_v = ok_vi = ok_vii = True
+    for phi, (sig, t) in zip(phis, sched):
+        sig = np.asarray(sig, dtype=np.int64)
+        t = np.asarray(t, dtype=np.int64)
+        lines, L = phi.shape
+        if sig.shape != (lines, L) or t.shape != (lines, L):
+            ok_v = ok_vi = ok_vii = False
+            continue
+        lane = np.arange(L, dtype=np.int64)[None, :] % w
+        s = w * sig + lane
+        if s.min() < 0 or s.max() >= L:
+            ok_v = ok_vi = ok_vii = False
+            continue
+        ok_vii &= _rows_are_perms(s)
+        ok_v &= bool(np.all(np.take_along_axis(phi, s, axis=1) == t))
+        ok_vi &= _rounds_distinct(s, w) and _rounds_distinct(t, w)
+    res["v_t_equals_phi_of_s"] = ok_v
+    res["vi_rounds_conflict_free"] = ok_vi
+    res["vii_sources_cover_line"] = ok_vii
+    return res
+
+
+def assert_plan(p, kappa, sched, rows, cols, w):
+    res = check_plan(p, kappa, sched, rows, cols, w)
+    bad = [k for k, v in res.items() if not v]
+    expected = {"shape", "i_row_colours_bijective", "ii_colour_dest_rows_distinct",
+                "iii_phases_bijective", "iv_composition_is_P", "v_t_equals_phi_of_s",
+                "vi_rounds_conflict_free", "vii_sources_cover_line"}
+    missing = expected - set(res)
+    if bad or missing:
+        raise AssertionError(f"plan invariants failed: {bad} missing: {sorted(missing)}")
+    return res
