@@ -1,0 +1,376 @@
+#!/usr/bin/env python
+"""Benchmark of the offline permutation hot path (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Metric: "4M-float32 permute time & effective HBM GB/s vs conventional
+b[p[i]] = a[i]". Workload (BASELINE configs[1]): n = 2^22 float32 (raw 32-bit
+words), the paper's five permutation families (identity, shuffle, random,
+bit-reversal, transpose). One STEP = one perm_apply of
+each of the five plans (all §8(a) rows: R1 -> R2 -> R3), with L2 flushed
+(256 MiB memset) before every apply, outside the event-timed region.
+
+value      = whole-job effective GB/s = sum over ranks of 5 * 2 * n * 4 B / step time
+             (device time from CUDA events on the launch stream, max over ranks)
+e2e        = the same metric through perm_apply_host (pinned host a -> device ->
+             apply -> host b, copies inside the timed region)
+roofline   = dominant kernel: algorithmic bytes per launch (read n*4 + write n*4 +
+             schedule n*E/8) / its mean event-timed duration, vs MEASURED_PEAKS hbm_gbs
+cpu_baseline = the oracle's plain C loop (oracle/c/apply_ref.c, all host cores)
+N > 1      = independent replicas, one per GPU (the 2^22 workload does not shard;
+             "scaling": "weak"); rank 0 prints the JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "4M-float32 permute time & effective HBM GB/s vs conventional b[p[i]]=a[i]"
+UNIT = "GB/s"
+FLUSH_BYTES = 256 << 20
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--log2n", type=int, default=22)
+    ap.add_argument("--families", default=",".join(W.FAMILIES))
+    ap.add_argument("--passes", type=int, default=0)
+    ap.add_argument("--h", default="0,0,0")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def measured_peaks() -> dict:
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            d = json.load(f)
+        d["_source"] = "measured"
+        return d
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "_source": "fallback"}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 100 ms during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(
+                    ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                     "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                if out.returncode == 0 and out.stdout.strip():
+                    self.rows.append([x.strip() for x in out.stdout.strip().split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.1)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self) -> dict:
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[3:7]):
+                if v.strip().lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(self.rows)}
+
+
+def cpu_oracle_baseline(plans_host, n, seconds: float) -> dict:
+    """The oracle's C loop (b[p[i]] = a[i], all host cores), bounded to ~`seconds`."""
+    from oracle import capply
+    fams = list(plans_host)
+    capply.apply_c(plans_host[fams[0]][0], plans_host[fams[0]][1])   # warm (build + page-in)
+    reps = 0
+    t0 = time.perf_counter()
+    moved = 0
+    while True:
+        for fam in fams:
+            p, a, out = plans_host[fam]
+            capply.apply_c(p, a, out)
+            moved += 2 * n * 4
+        reps += 1
+        if time.perf_counter() - t0 >= seconds:
+            break
+    dt = time.perf_counter() - t0
+    return {"value": moved / dt / 1e9, "unit": UNIT, "cores": capply.threads(), "kind": "oracle",
+            "sample": f"{reps} passes over the {len(fams)} families at n=2^{int(np.log2(n))} "
+                      f"({dt:.1f} s, oracle/c/apply_ref.c OpenMP loop)"}
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    n = 1 << args.log2n
+    fams = args.families.split(",")
+    host = {f: (W.make_perm(f, n), W.make_data(n), np.empty(n, dtype=np.uint32)) for f in fams}
+    from oracle import capply
+    for _ in range(max(args.warmup, 0)):
+        for f in fams:
+            capply.apply_c(*host[f])
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for f in fams:
+            capply.apply_c(*host[f])
+    dt = time.perf_counter() - t0
+    ms = dt / args.steps * 1e3
+    value = len(fams) * 2 * n * 4 / (dt / args.steps) / 1e9
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": f"n=2^{args.log2n} float32 words, families {fams}",
+                       "n": n, "families": fams},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": capply.threads(),
+                             "kind": "oracle",
+                             "sample": f"full workload, {args.steps} steps (no sampling needed)"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_icpp_kasagini13_b200 as pkg
+
+    n = 1 << args.log2n
+    fams = args.families.split(",")
+    h = tuple(int(x) for x in args.h.split(","))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+
+    plans, dA, dB, dP, host = {}, {}, {}, {}, {}
+    build_ms = {}
+    for f in fams:
+        p = W.make_perm(f, n)
+        a = W.make_data(n)
+        t0 = time.perf_counter()
+        plans[f] = pkg.Plan(p, passes=args.passes, h=h)
+        build_ms[f] = (time.perf_counter() - t0) * 1e3
+        dA[f] = torch.from_numpy(a.view(np.int32)).to(dev)
+        dB[f] = torch.empty_like(dA[f])
+        dP[f] = torch.from_numpy(p).to(dev)
+        host[f] = (p, a, np.empty(n, dtype=np.uint32))
+    info = plans[fams[0]].info()
+    flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+
+    def timed_apply(fn, ev0, ev1):
+        flush.zero_()
+        ev0.record(stream)
+        fn()
+        ev1.record(stream)
+
+    # ---- warm-up
+    for _ in range(max(args.warmup, 3)):
+        for f in fams:
+            plans[f].apply(dA[f], dB[f], stream)
+            pkg.scatter_baseline(dP[f], dA[f], dB[f], stream)
+    torch.cuda.synchronize()
+    # correctness of the last output (cheap: compare one family with the oracle)
+    from oracle import apply as OA
+    chk = fams[-1]
+    plans[chk].apply(dA[chk], dB[chk], stream)
+    torch.cuda.synchronize()
+    ok = bool(np.array_equal(dB[chk].cpu().numpy().view(np.uint32),
+                             OA.apply_ref(host[chk][0], host[chk][1])))
+
+    # ---- timed region: K steps, each = one apply per family
+    evs = {f: [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)] for f in fams}
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clocks:
+        t_wall = time.perf_counter()
+        for s in range(args.steps):
+            for f in fams:
+                timed_apply(lambda: plans[f].apply(dA[f], dB[f], stream), *evs[f][s])
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter() - t_wall
+    if world > 1:
+        dist.barrier()
+    per_fam_ms = {f: [e0.elapsed_time(e1) for e0, e1 in evs[f]] for f in fams}
+    step_ms = [sum(per_fam_ms[f][s] for f in fams) for s in range(args.steps)]
+    ms_per_step = statistics.mean(step_ms)
+    if world > 1:
+        t = torch.tensor([ms_per_step], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_per_step = float(t.item())
+    bytes_per_step = len(fams) * 2 * n * 4
+    value = world * bytes_per_step / (ms_per_step * 1e-3) / 1e9
+
+    # ---- conventional D-designated kernel (and S-designated) on the same inputs
+    conv = {}
+    gather = {}
+    dQ = {f: torch.from_numpy(OA.inverse(host[f][0])).to(dev) for f in fams}
+    for f in fams:
+        ts, tg = [], []
+        for _ in range(args.steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            timed_apply(lambda: pkg.scatter_baseline(dP[f], dA[f], dB[f], stream), e0, e1)
+            e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            timed_apply(lambda: pkg.gather_baseline(dQ[f], dA[f], dB[f], stream), e2, e3)
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+            tg.append(e2.elapsed_time(e3))
+        conv[f] = statistics.median(ts)
+        gather[f] = statistics.median(tg)
+
+    # ---- per-kernel durations (events between kernels; PDL overlap disabled here)
+    kern = {f: [] for f in fams}
+    for f in fams:
+        plans[f].set_profiling(True)
+        for _ in range(args.steps):
+            flush.zero_()
+            plans[f].apply(dA[f], dB[f], stream)
+            kern[f].append(plans[f].pass_times())
+        plans[f].set_profiling(False)
+    nk = len(kern[fams[0]][0])
+    mean_k = [statistics.mean(kern[f][s][i] for f in fams for s in range(args.steps))
+              for i in range(nk)]
+    dom = int(np.argmax(mean_k))
+    E = info["entry_bits"]
+    kinds = (["R1", "R2", "R3"] if info["passes"] == 3 else
+             ["R1", "T", "R2", "T", "R3"] if info["passes"] == 5 else ["fused R1+R2+R3"])
+    if info["passes"] == 3:
+        alg = [2 * n * 4 + n * E[i] / 8 for i in range(3)]
+    elif info["passes"] == 5:
+        alg = [2 * n * 4 + n * E[0] / 8, 2 * n * 4, 2 * n * 4 + n * E[1] / 8, 2 * n * 4,
+               2 * n * 4 + n * E[2] / 8]
+    else:
+        alg = [2 * n * 4 + n * sum(E) / 8]
+    peaks = measured_peaks()
+    achieved = alg[dom] / (mean_k[dom] * 1e-3) / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as fh:
+            tj = json.load(fh)
+        traffic = tj.get(f"n{args.log2n}", {}).get(kinds[dom])
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+                "kernel": kinds[dom], "kernel_ms": mean_k[dom],
+                "algorithmic_bytes_per_launch": alg[dom], "peak_source": peaks["_source"],
+                "per_kernel_ms": dict(zip([f"{k}#{i}" for i, k in enumerate(kinds)], mean_k))}
+
+    # ---- end to end through the C ABI with host buffers
+    e2e = None
+    if not args.no_e2e:
+        pinned = {f: (torch.from_numpy(host[f][1].view(np.int32)).pin_memory(),
+                      torch.empty(n, dtype=torch.int32).pin_memory()) for f in fams}
+        for f in fams:
+            plans[f].apply_host(pinned[f][0], pinned[f][1], stream)
+        ts = []
+        for _ in range(args.steps):
+            tot = 0.0
+            for f in fams:
+                flush.zero_()
+                torch.cuda.synchronize()
+                t0 = time.perf_counter()
+                plans[f].apply_host(pinned[f][0], pinned[f][1], stream)   # syncs the stream
+                tot += time.perf_counter() - t0
+            ts.append(tot)
+        e2e_s = statistics.mean(ts)
+        e2e = {"value": world * bytes_per_step / e2e_s / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": len(fams) * n * 4, "d2h_bytes_per_step": len(fams) * n * 4,
+               "ms_per_step": e2e_s * 1e3}
+
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        cpu = cpu_oracle_baseline(host, n, args.cpu_seconds)
+
+    if rank == 0:
+        per_fam_us = {f: 1e3 * statistics.median(per_fam_ms[f]) for f in fams}
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"n=2^{args.log2n} float32 (raw u32 words), 5 permutation "
+                                   "families, one perm_apply each per step",
+                       "n": n, "families": fams, "view": [info["rows"], info["cols"]],
+                       "passes": info["passes"], "h": info["h"],
+                       "l2": "flushed (256 MiB memset) before every timed apply",
+                       "parallelism": f"replicas x{world}"},
+            "apply_us": per_fam_us,
+            "conventional_us": {f: 1e3 * conv[f] for f in fams},
+            "s_designated_us": {f: 1e3 * gather[f] for f in fams},
+            "speedup_vs_conventional": {f: conv[f] * 1e3 / per_fam_us[f] for f in fams},
+            "effective_gbs": {f: 2 * n * 4 / (per_fam_us[f] * 1e-6) / 1e9 for f in fams},
+            "plan_build_ms": build_ms,
+            "sched_bytes": info["sched_bytes"],
+            "bitexact_check": ok,
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": args.steps * len(fams) * info["kernels_per_apply"],
+            "clocks": clocks.summary(),
+            "wall_s_timed_region": t_wall,
+        }
+        print(json.dumps(line), flush=True)
+    for pl in plans.values():
+        pl.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,168 @@
+/*
+ * perm.h — C ABI of libperm, the B200 (sm_100a) offline permutation library.
+ *
+ * Operation (§IV): given a permutation P of {0..n-1}, stored in
+ * an int32 array p with p[i] = P(i) and known in advance ("offline"), copy
+ * a[i] to b[P(i)] for every i. The result is unique; libperm produces it
+ * bit-exactly (raw 4-byte words are moved, never interpreted as floats).
+ *
+ * Method (§V-§VII, Thm 9): view a and b as r x c matrices and
+ * apply a row-wise permutation, a column-wise permutation (= transpose,
+ * row-wise, transpose; Lemma 8) and a row-wise permutation. The three
+ * per-line permutations come from a König edge-colouring of the row-level
+ * bipartite multigraph (L537-L539, L603-L605); every shared-memory permute
+ * hop is bank-conflict-free because of a second colouring of each line's
+ * bank-level graph (Thm 6). Both colourings are computed
+ * once per P on the host by perm_plan_create (the "offline" cost, timed and
+ * reported separately); perm_apply is the data-parallel hot path.
+ *
+ * Thread safety: distinct plans may be used from distinct threads. A plan
+ * is immutable after creation, but it owns scratch buffers, so at most ONE
+ * perm_apply may be in flight per plan at a time (use one plan per stream).
+ * Error status is thread-local (perm_last_error).
+ */
+#ifndef LIBPERM_PERM_H
+#define LIBPERM_PERM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* cudaStream_t is passed as an opaque pointer so this header does not need
+ * the CUDA headers; NULL means the legacy default stream. */
+typedef void* perm_stream_t;
+
+typedef struct perm_plan perm_plan;   /* opaque */
+
+enum perm_status {
+    PERM_OK           =  0,
+    PERM_EINVAL       = -1,  /* null pointer, n <= 0, a == b / overlapping buffers, bad option */
+    PERM_ENOTPERM     = -2,  /* p is not a permutation of 0..n-1 (value out of range or repeated) */
+    PERM_EUNSUPPORTED = -3,  /* n not a power of two in [2^10, 2^30], or elem_bytes != 4 */
+    PERM_ENOMEM       = -4,  /* host or device allocation failed */
+    PERM_ECUDA        = -5,  /* a CUDA runtime call failed (message has the CUDA error) */
+    PERM_ENCCL        = -6,  /* reserved for the row-sharded multi-GPU path */
+    PERM_ENODEVICE    = -7   /* the call needs a device but the plan is host-only / no GPU */
+};
+
+/* Pass structures a plan may use (perm_plan_info.passes). */
+enum perm_passes {
+    PERM_PASSES_AUTO  = 0,
+    PERM_PASSES_FUSED = 1,   /* n <= 2^15: all three phases inside one CTA's shared memory */
+    PERM_PASSES_3     = 3,   /* R1, R2, R3; both transposes absorbed into tiled layouts */
+    PERM_PASSES_5     = 5    /* R, T, R, T, R: the paper's five kernel calls (L699) */
+};
+
+typedef struct {
+    int32_t passes;      /* enum perm_passes; 0 = choose by n */
+    int32_t h1, h2, h3;  /* lines per CTA in the three row passes; 0 = choose */
+    int32_t reserved[8];
+} perm_plan_options;
+
+typedef struct {
+    int64_t n;
+    int64_t rows, cols;          /* the r x c view (L603) */
+    int64_t sched_bytes;         /* device bytes of the three packed bank schedules */
+    int64_t scratch_bytes;       /* device bytes of intermediate buffers */
+    int32_t elem_bytes;
+    int32_t passes;              /* 1, 3 or 5 */
+    int32_t kernels_per_apply;   /* kernel launches one perm_apply issues */
+    int32_t entry_bits[3];       /* bits per schedule entry, phase 1..3 (2*log2(L) - 5) */
+    int32_t h[3];                /* lines per CTA of the three row passes */
+    int32_t planner_threads;     /* OpenMP threads the planner used */
+    double  build_ms_colour;     /* row-level König colouring (Euler split) */
+    double  build_ms_bank;       /* per-line bank-level colourings + packing */
+    double  build_ms_upload;     /* device allocation + host->device copy */
+} perm_plan_info;
+
+/* ------------------------------------------------------------------ plans */
+
+/* Build a plan for P on the CURRENT CUDA device: validates p (O(n) bitmap),
+ * colours, packs and uploads the schedules and allocates scratch.
+ * p: host int32[n], borrowed for the duration of the call only.
+ * n: power of two, 2^10 <= n <= 2^30. elem_bytes: 4.
+ * Returns NULL on error (see perm_last_error). Synchronous. */
+perm_plan* perm_plan_create(const int32_t* p, int64_t n, int32_t elem_bytes);
+
+/* Same with explicit options (NULL = defaults). */
+perm_plan* perm_plan_create_ex(const int32_t* p, int64_t n, int32_t elem_bytes,
+                               const perm_plan_options* opt);
+
+/* Planner only: builds the host-side plan (colourings, packed schedules) and
+ * touches no CUDA API. Usable on a machine without a GPU for perm_plan_export
+ * and perm_plan_get_info; perm_apply on it returns PERM_ENODEVICE. */
+perm_plan* perm_plan_create_host(const int32_t* p, int64_t n, int32_t elem_bytes,
+                                 const perm_plan_options* opt);
+
+/* Frees host and device memory. NULL is a no-op. The caller must ensure no
+ * perm_apply on this plan is still running on the device. */
+void perm_plan_destroy(perm_plan* plan);
+
+int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out);
+
+/* Human/machine-readable JSON description of the plan's pass structure
+ * (views, per-pass lines per CTA, threads, elements per thread, shared-memory
+ * stride, simulated bank-conflict wavefronts, I/O layouts). Writes at most
+ * len bytes including the terminating NUL; returns the full length needed. */
+int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len);
+
+/* Export the plan in LOGICAL order for an independent checker:
+ *   kappa[x], x in [0,n): row-level colour of element x (uint16; c <= 2^15);
+ *   sched1[i*c + q], sched2[k*r + q], sched3[i*c + q]: for line i (rows for
+ *   phases 1 and 3, columns k for phase 2) and slot q = round*32 + lane,
+ *   the entry (sigma << 16) | t: the slot reads source s = 32*sigma + lane
+ *   and writes destination t.
+ * Any output pointer may be NULL to skip it. Host memory, caller-owned. */
+int perm_plan_export(const perm_plan* plan, uint16_t* kappa,
+                     uint32_t* sched1, uint32_t* sched2, uint32_t* sched3);
+
+/* ------------------------------------------------------------------ apply */
+
+/* b[P(i)] = a[i] for all i. a, b: DEVICE pointers to n*elem_bytes bytes on the
+ * plan's device, 16-byte aligned, not overlapping (the algorithm is
+ * out-of-place, L361). Asynchronous and stream-ordered: no host sync, no
+ * allocation. Launch errors are returned immediately (PERM_ECUDA); device
+ * faults surface at the caller's next synchronisation. */
+int perm_apply(const perm_plan* plan, const void* a, void* b, perm_stream_t stream);
+
+/* End-to-end variant with HOST buffers: copies a_host to the device, applies,
+ * copies the result to b_host, then synchronises the stream. The first call
+ * allocates 2*n*elem_bytes of device staging owned by the plan. Pinned host
+ * memory gives asynchronous copies; pageable memory works but is slower. */
+int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream);
+
+/* Per-kernel timing: when enabled, perm_apply records a CUDA event before its
+ * first kernel and after each kernel on the launch stream. perm_plan_pass_times
+ * waits for the last event and writes up to max_k kernel durations (ms) of the
+ * most recent apply; returns the number written or a negative status. */
+int perm_plan_set_profiling(perm_plan* plan, int enable);
+int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k);
+
+/* ------------------------------------------------------- comparators */
+
+/* D-designated (conventional) algorithm: b[p[i]] = a[i] in one
+ * kernel. p_dev: DEVICE int32[n] (a valid permutation; not checked). */
+int perm_scatter_baseline(const int32_t* p_dev, const void* a, void* b, int64_t n,
+                          int32_t elem_bytes, perm_stream_t stream);
+
+/* S-designated algorithm: b[i] = a[q[i]], q = P^{-1} (DEVICE). */
+int perm_gather_baseline(const int32_t* q_dev, const void* a, void* b, int64_t n,
+                         int32_t elem_bytes, perm_stream_t stream);
+
+/* Plain device-to-device copy of n*elem_bytes with the same vectorised
+ * kernel style (the identity lower bound used for roofline context). */
+int perm_copy_kernel(const void* a, void* b, int64_t n, int32_t elem_bytes,
+                     perm_stream_t stream);
+
+/* ------------------------------------------------------------- status */
+
+int         perm_last_error(void);          /* thread-local status of the last failed call */
+const char* perm_last_error_string(void);   /* thread-local message, never NULL */
+const char* perm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIBPERM_PERM_H */

@@ -1,0 +1,229 @@
+"""Thin ctypes binding of libperm (include/perm.h): argument marshalling only.
+
+Every step of the permutation runs in libperm's C++ planner and sm_100a
+kernels. PyTorch supplies device memory and streams (data_ptr / cuda_stream).
+There is no Python or CPU fallback: if libperm.so is missing this module
+raises on import.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libperm.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        f"{LIB_PATH} is not built; run `python -m paper_conf_icpp_kasagini13_b200.build` "
+        "or __graft_entry__.build() (there is no CPU fallback)")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+PERM_OK = 0
+STATUS = {0: "PERM_OK", -1: "PERM_EINVAL", -2: "PERM_ENOTPERM", -3: "PERM_EUNSUPPORTED",
+          -4: "PERM_ENOMEM", -5: "PERM_ECUDA", -6: "PERM_ENCCL", -7: "PERM_ENODEVICE"}
+
+
+class PermError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class PlanOptions(ctypes.Structure):
+    _fields_ = [("passes", ctypes.c_int32), ("h1", ctypes.c_int32), ("h2", ctypes.c_int32),
+                ("h3", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("rows", ctypes.c_int64), ("cols", ctypes.c_int64),
+                ("sched_bytes", ctypes.c_int64), ("scratch_bytes", ctypes.c_int64),
+                ("elem_bytes", ctypes.c_int32), ("passes", ctypes.c_int32),
+                ("kernels_per_apply", ctypes.c_int32), ("entry_bits", ctypes.c_int32 * 3),
+                ("h", ctypes.c_int32 * 3), ("planner_threads", ctypes.c_int32),
+                ("build_ms_colour", ctypes.c_double), ("build_ms_bank", ctypes.c_double),
+                ("build_ms_upload", ctypes.c_double)]
+
+    def as_dict(self) -> dict:
+        d = {}
+        for name, _ in self._fields_:
+            v = getattr(self, name)
+            d[name] = list(v) if isinstance(v, ctypes.Array) else v
+        return d
+
+
+_vp, _i64, _i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
+
+
+def _sig(name, res, *args):
+    f = getattr(_lib, name)
+    f.restype = res
+    f.argtypes = list(args)
+    return f
+
+
+_plan_create = _sig("perm_plan_create", _vp, _vp, _i64, _i32)
+_plan_create_ex = _sig("perm_plan_create_ex", _vp, _vp, _i64, _i32, ctypes.POINTER(PlanOptions))
+_plan_create_host = _sig("perm_plan_create_host", _vp, _vp, _i64, _i32, ctypes.POINTER(PlanOptions))
+_plan_destroy = _sig("perm_plan_destroy", None, _vp)
+_plan_get_info = _sig("perm_plan_get_info", ctypes.c_int, _vp, ctypes.POINTER(PlanInfo))
+_plan_describe = _sig("perm_plan_describe", _i64, _vp, ctypes.c_char_p, _i64)
+_plan_export = _sig("perm_plan_export", ctypes.c_int, _vp, _vp, _vp, _vp, _vp)
+_apply = _sig("perm_apply", ctypes.c_int, _vp, _vp, _vp, _vp)
+_apply_host = _sig("perm_apply_host", ctypes.c_int, _vp, _vp, _vp, _vp)
+_set_prof = _sig("perm_plan_set_profiling", ctypes.c_int, _vp, ctypes.c_int)
+_pass_times = _sig("perm_plan_pass_times", ctypes.c_int, _vp, ctypes.POINTER(ctypes.c_float), ctypes.c_int)
+_scatter = _sig("perm_scatter_baseline", ctypes.c_int, _vp, _vp, _vp, _i64, _i32, _vp)
+_gather = _sig("perm_gather_baseline", ctypes.c_int, _vp, _vp, _vp, _i64, _i32, _vp)
+_copy = _sig("perm_copy_kernel", ctypes.c_int, _vp, _vp, _i64, _i32, _vp)
+_last_error = _sig("perm_last_error", ctypes.c_int)
+_last_error_string = _sig("perm_last_error_string", ctypes.c_char_p)
+_version = _sig("perm_version", ctypes.c_char_p)
+
+
+def version() -> str:
+    return _version().decode()
+
+
+def _raise(status: int | None = None):
+    st = _last_error() if status is None else status
+    raise PermError(st, _last_error_string().decode())
+
+
+def _check(status: int):
+    if status != PERM_OK:
+        _raise(status)
+
+
+def _stream_handle(stream) -> int | None:
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def _ptr(x) -> int:
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    return int(x)
+
+
+def _as_int32_host(p) -> np.ndarray:
+    if hasattr(p, "detach"):       # torch tensor
+        p = p.detach().cpu().numpy()
+    return np.ascontiguousarray(p, dtype=np.int32)
+
+
+class Plan:
+    """perm_plan: the offline schedule of permutation p (int32, host)."""
+
+    def __init__(self, p, elem_bytes: int = 4, passes: int = 0, h=(0, 0, 0),
+                 device: bool = True):
+        p = _as_int32_host(p)
+        self.n = int(p.size)
+        self.elem_bytes = elem_bytes
+        opt = PlanOptions(passes, h[0], h[1], h[2])
+        if device:
+            handle = _plan_create_ex(p.ctypes.data, self.n, elem_bytes, ctypes.byref(opt))
+        else:
+            handle = _plan_create_host(p.ctypes.data, self.n, elem_bytes, ctypes.byref(opt))
+        if not handle:
+            _raise()
+        self._h = handle
+        self.on_device = device
+
+    # -- lifecycle
+    def close(self):
+        if getattr(self, "_h", None):
+            _plan_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # -- introspection
+    def info(self) -> dict:
+        inf = PlanInfo()
+        _check(_plan_get_info(self._h, ctypes.byref(inf)))
+        return inf.as_dict()
+
+    def describe(self) -> dict:
+        import json
+        need = _plan_describe(self._h, None, 0)
+        if need < 0:
+            _raise(int(need))
+        buf = ctypes.create_string_buffer(int(need))
+        _plan_describe(self._h, buf, need)
+        return json.loads(buf.value.decode())
+
+    def export(self):
+        """(kappa[n] uint16, [sched1 (r,c), sched2 (c,r), sched3 (r,c)] uint32 (sigma<<16)|t)."""
+        inf = self.info()
+        r, c = inf["rows"], inf["cols"]
+        kappa = np.empty(self.n, dtype=np.uint16)
+        s1 = np.empty((r, c), dtype=np.uint32)
+        s2 = np.empty((c, r), dtype=np.uint32)
+        s3 = np.empty((r, c), dtype=np.uint32)
+        _check(_plan_export(self._h, kappa.ctypes.data, s1.ctypes.data, s2.ctypes.data,
+                            s3.ctypes.data))
+        return kappa, [s1, s2, s3]
+
+    # -- hot path
+    def apply(self, a, b, stream=None):
+        """b[p[i]] = a[i]; a, b CUDA tensors of n elements (4-byte dtype), stream-ordered."""
+        _check(_apply(self._h, _ptr(a), _ptr(b), _stream_handle(stream)))
+        return b
+
+    def apply_host(self, a_host, b_host, stream=None):
+        """End-to-end: host a -> device -> apply -> host b (synchronises the stream)."""
+        _check(_apply_host(self._h, _ptr(a_host), _ptr(b_host), _stream_handle(stream)))
+        return b_host
+
+    def set_profiling(self, on: bool = True):
+        _check(_set_prof(self._h, 1 if on else 0))
+
+    def pass_times(self) -> list[float]:
+        buf = (ctypes.c_float * 8)()
+        k = _pass_times(self._h, buf, 8)
+        if k < 0:
+            _raise(k)
+        return [float(buf[i]) for i in range(k)]
+
+
+def scatter_baseline(p_dev, a, b, stream=None):
+    """D-designated b[p[i]] = a[i], one kernel. p_dev: int32 CUDA tensor."""
+    n = p_dev.numel()
+    _check(_scatter(_ptr(p_dev), _ptr(a), _ptr(b), n, 4, _stream_handle(stream)))
+    return b
+
+
+def gather_baseline(q_dev, a, b, stream=None):
+    """S-designated b[i] = a[q[i]], q = P^{-1} on the device."""
+    n = q_dev.numel()
+    _check(_gather(_ptr(q_dev), _ptr(a), _ptr(b), n, 4, _stream_handle(stream)))
+    return b
+
+
+def copy_kernel(a, b, stream=None):
+    _check(_copy(_ptr(a), _ptr(b), a.numel(), a.element_size(), _stream_handle(stream)))
+    return b
+
+
+def last_error() -> tuple[int, str]:
+    return int(_last_error()), _last_error_string().decode()

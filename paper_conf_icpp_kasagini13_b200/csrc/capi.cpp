@@ -1,0 +1,389 @@
+// capi.cpp — the C ABI of libperm (include/perm.h): plan lifecycle, error
+// model, device memory and the launch sequence of perm_apply.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "../../include/perm.h"
+#include "kernels.hpp"
+#include "plan.hpp"
+
+using perm::HostPlan;
+
+struct perm_plan {
+    HostPlan host;
+    bool on_device = false;
+    int device = -1;
+    uint32_t* d_sched = nullptr;          // the three phases back to back
+    uint32_t* d_phase[3] = {nullptr, nullptr, nullptr};
+    uint32_t* d_scratch[2] = {nullptr, nullptr};
+    int64_t sched_bytes = 0, scratch_bytes = 0;
+    double ms_upload = 0;
+    // staging for perm_apply_host
+    uint32_t* d_stage[2] = {nullptr, nullptr};
+    // profiling
+    bool profiling = false;
+    int n_events = 0;
+    cudaEvent_t ev[8] = {};
+    int last_kernels = 0;
+};
+
+namespace {
+
+thread_local int g_status = PERM_OK;
+thread_local std::string g_msg = "ok";
+
+int fail(int status, const std::string& msg) {
+    g_status = status;
+    g_msg = msg;
+    return status;
+}
+
+int cuda_fail(cudaError_t e, const char* what) {
+    return fail(PERM_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+void free_device(perm_plan* pl) {
+    if (!pl->on_device) return;
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (pl->device >= 0) cudaSetDevice(pl->device);
+    cudaFree(pl->d_sched);
+    cudaFree(pl->d_scratch[0]);
+    cudaFree(pl->d_scratch[1]);
+    cudaFree(pl->d_stage[0]);
+    cudaFree(pl->d_stage[1]);
+    for (int i = 0; i < pl->n_events; ++i) cudaEventDestroy(pl->ev[i]);
+    pl->n_events = 0;
+    if (cur >= 0) cudaSetDevice(cur);
+    pl->on_device = false;
+}
+
+int upload(perm_plan* pl) {
+    auto t0 = std::chrono::steady_clock::now();
+    HostPlan& P = pl->host;
+    cudaError_t e = cudaGetDevice(&pl->device);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    int64_t words = 0;
+    for (int f = 0; f < 3; ++f) words += P.ph[f].words + 32;   // +32: shuffle over-read guard
+    pl->sched_bytes = words * 4;
+    e = cudaMalloc(&pl->d_sched, (size_t)pl->sched_bytes);
+    if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc schedules: ") + cudaGetErrorString(e));
+    pl->on_device = true;
+    int64_t off = 0;
+    for (int f = 0; f < 3; ++f) {
+        pl->d_phase[f] = pl->d_sched + off;
+        e = cudaMemcpy(pl->d_phase[f], P.sched[f].data(), (size_t)P.ph[f].words * 4,
+                       cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy schedules");
+        e = cudaMemset(pl->d_phase[f] + P.ph[f].words, 0, 32 * 4);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemset");
+        off += P.ph[f].words + 32;
+    }
+    if (P.passes != 1) {
+        const size_t bytes = (size_t)P.n * P.eb;
+        for (int i = 0; i < 2; ++i) {
+            e = cudaMalloc(&pl->d_scratch[i], bytes);
+            if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc scratch: ") + cudaGetErrorString(e));
+        }
+        pl->scratch_bytes = 2 * (int64_t)bytes;
+    }
+    e = perm::prepare_kernels(P);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
+    for (int i = 0; i < 8; ++i) {
+        e = cudaEventCreate(&pl->ev[i]);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaEventCreate");
+        pl->n_events = i + 1;
+    }
+    e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceSynchronize");
+    pl->ms_upload =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return PERM_OK;
+}
+
+perm_plan* create(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
+                  bool device) {
+    perm_plan* pl = new (std::nothrow) perm_plan();
+    if (!pl) { fail(PERM_ENOMEM, "out of host memory"); return nullptr; }
+    std::string err;
+    int st;
+    try {
+        st = perm::build_host_plan(p, n, eb, opt, pl->host, err);
+    } catch (const std::bad_alloc&) {
+        st = PERM_ENOMEM;
+        err = "out of host memory while planning";
+    }
+    if (st != PERM_OK) {
+        fail(st, err);
+        delete pl;
+        return nullptr;
+    }
+    if (device) {
+        st = upload(pl);
+        if (st != PERM_OK) {
+            free_device(pl);
+            delete pl;
+            return nullptr;
+        }
+    }
+    g_status = PERM_OK;
+    g_msg = "ok";
+    return pl;
+}
+
+bool overlap(const void* a, const void* b, int64_t bytes) {
+    const char* x = static_cast<const char*>(a);
+    const char* y = static_cast<const char*>(b);
+    return x < y + bytes && y < x + bytes;
+}
+
+}  // namespace
+
+extern "C" {
+
+perm_plan* perm_plan_create(const int32_t* p, int64_t n, int32_t elem_bytes) {
+    return create(p, n, elem_bytes, nullptr, true);
+}
+
+perm_plan* perm_plan_create_ex(const int32_t* p, int64_t n, int32_t elem_bytes,
+                               const perm_plan_options* opt) {
+    return create(p, n, elem_bytes, opt, true);
+}
+
+perm_plan* perm_plan_create_host(const int32_t* p, int64_t n, int32_t elem_bytes,
+                                 const perm_plan_options* opt) {
+    return create(p, n, elem_bytes, opt, false);
+}
+
+void perm_plan_destroy(perm_plan* plan) {
+    if (!plan) return;
+    free_device(plan);
+    delete plan;
+}
+
+int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
+    if (!plan || !out) return fail(PERM_EINVAL, "null plan or info");
+    const HostPlan& P = plan->host;
+    std::memset(out, 0, sizeof(*out));
+    out->n = P.n;
+    out->rows = P.r;
+    out->cols = P.c;
+    int64_t words = 0;
+    for (int f = 0; f < 3; ++f) words += P.ph[f].words;
+    out->sched_bytes = plan->on_device ? plan->sched_bytes : words * 4;
+    out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes == 1 ? 0 : 2 * P.n * P.eb);
+    out->elem_bytes = P.eb;
+    out->passes = P.passes;
+    out->kernels_per_apply = P.passes;
+    for (int f = 0; f < 3; ++f) {
+        out->entry_bits[f] = P.ph[f].E;
+        out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
+    }
+    out->planner_threads = P.threads_used;
+    out->build_ms_colour = P.ms_colour;
+    out->build_ms_bank = P.ms_bank;
+    out->build_ms_upload = plan->ms_upload;
+    return PERM_OK;
+}
+
+int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
+    if (!plan) return fail(PERM_EINVAL, "null plan");
+    const HostPlan& P = plan->host;
+    std::string s = "{\"n\":" + std::to_string(P.n) + ",\"rows\":" + std::to_string(P.r) +
+                    ",\"cols\":" + std::to_string(P.c) + ",\"passes\":" + std::to_string(P.passes);
+    if (P.passes == 1) {
+        s += ",\"fused\":{\"threads\":" + std::to_string(P.fused_threads) + ",\"ept\":" +
+             std::to_string(P.fused_ept) + ",\"Ls\":" + std::to_string(P.fused_Ls) + "}";
+    } else {
+        s += ",\"row_passes\":[";
+        for (int f = 0; f < 3; ++f) {
+            const perm::RowPass& rp = P.rp[f];
+            auto io = [](const perm::IoMode& m) {
+                return std::string("{\"cross\":") + std::to_string(m.cross) + ",\"w\":" +
+                       std::to_string(m.w) + ",\"strideK\":" + std::to_string(m.strideK) +
+                       ",\"blockP\":" + std::to_string(m.blockP) + ",\"strideP\":" +
+                       std::to_string(m.strideP) + ",\"cta_stride\":" + std::to_string(m.cta_stride) + "}";
+            };
+            s += std::string(f ? "," : "") + "{\"phase\":" + std::to_string(rp.phase) +
+                 ",\"L\":" + std::to_string(P.ph[rp.phase].L) + ",\"E\":" +
+                 std::to_string(P.ph[rp.phase].E) + ",\"h\":" + std::to_string(rp.h) +
+                 ",\"ctas\":" + std::to_string(rp.ctas) + ",\"threads\":" +
+                 std::to_string(rp.threads) + ",\"ept\":" + std::to_string(rp.ept) +
+                 ",\"Ls\":" + std::to_string(rp.Ls) + ",\"smem_bytes\":" +
+                 std::to_string((int64_t)rp.h * rp.Ls * 4) + ",\"wavefronts_in\":" +
+                 std::to_string(rp.conflicts_in) + ",\"wavefronts_out\":" +
+                 std::to_string(rp.conflicts_out) + ",\"in\":" + io(rp.in) + ",\"out\":" +
+                 io(rp.out) + "}";
+        }
+        s += "]";
+    }
+    s += "}";
+    if (buf && len > 0) {
+        const int64_t m = std::min<int64_t>(len - 1, (int64_t)s.size());
+        std::memcpy(buf, s.data(), (size_t)m);
+        buf[m] = 0;
+    }
+    return (int64_t)s.size() + 1;
+}
+
+int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint32_t* s2,
+                     uint32_t* s3) {
+    if (!plan) return fail(PERM_EINVAL, "null plan");
+    const HostPlan& P = plan->host;
+    if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));
+    uint32_t* outs[3] = {s1, s2, s3};
+    for (int f = 0; f < 3; ++f) {
+        if (!outs[f]) continue;
+        const perm::PhaseGeom& g = P.ph[f];
+        const uint32_t tmask = (1u << g.logL) - 1u;
+#pragma omp parallel for schedule(static)
+        for (int64_t line = 0; line < g.lines; ++line) {
+            for (int64_t q = 0; q < g.L; ++q) {
+                const uint32_t e = perm::unpack_entry(P.sched[f], g, line, q);
+                outs[f][line * g.L + q] = ((e >> g.logL) << 16) | (e & tmask);
+            }
+        }
+    }
+    return PERM_OK;
+}
+
+int perm_plan_set_profiling(perm_plan* plan, int enable) {
+    if (!plan) return fail(PERM_EINVAL, "null plan");
+    plan->profiling = enable != 0;
+    return PERM_OK;
+}
+
+int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k) {
+    if (!plan || !ms) return fail(PERM_EINVAL, "null argument");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "host-only plan");
+    const int k = plan->last_kernels;
+    if (k <= 0) return 0;
+    cudaError_t e = cudaEventSynchronize(plan->ev[k]);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaEventSynchronize");
+    int w = 0;
+    for (int i = 0; i < k && w < max_k; ++i) {
+        float t = 0;
+        e = cudaEventElapsedTime(&t, plan->ev[i], plan->ev[i + 1]);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaEventElapsedTime");
+        ms[w++] = t;
+    }
+    return w;
+}
+
+int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t stream) {
+    perm_plan* plan = const_cast<perm_plan*>(plan_c);   // only profiling bookkeeping mutates
+    if (!plan || !a || !b) return fail(PERM_EINVAL, "null plan or buffer");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
+    const HostPlan& P = plan->host;
+    if (overlap(a, b, P.n * P.eb)) return fail(PERM_EINVAL, "a and b overlap (out-of-place only)");
+    if ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15)
+        return fail(PERM_EINVAL, "a and b must be 16-byte aligned");
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const uint32_t* in = static_cast<const uint32_t*>(a);
+    uint32_t* out = static_cast<uint32_t*>(b);
+    const bool prof = plan->profiling;
+    int ev = 0;
+    auto mark = [&]() {
+        if (prof) cudaEventRecord(plan->ev[ev++], s);
+    };
+    cudaError_t e = cudaSuccess;
+    int k = 0;   // index of the kernel being launched (for the error message)
+    mark();
+    if (P.passes == 1) {
+        const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
+        e = perm::launch_fused(P, sc, in, out, s);
+        mark();
+    } else if (P.passes == 3) {
+        uint32_t* x1 = plan->d_scratch[0];
+        uint32_t* x2 = plan->d_scratch[1];
+        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false);
+        mark();
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x1, x2, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof); mark(); }
+    } else {
+        uint32_t* x1 = plan->d_scratch[0];
+        uint32_t* x2 = plan->d_scratch[1];
+        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false);
+        mark();
+        if (e == cudaSuccess) { ++k; e = perm::launch_transpose(x1, x2, P.r, P.c, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x2, x1, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_transpose(x1, x2, P.c, P.r, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof); mark(); }
+    }
+    if (e != cudaSuccess) {
+        if (prof) plan->last_kernels = 0;
+        return cuda_fail(e, ("launch of kernel " + std::to_string(k) + " of " +
+                             std::to_string(P.passes)).c_str());
+    }
+    if (prof) plan->last_kernels = ev - 1;
+    e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+    return PERM_OK;
+}
+
+int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream) {
+    if (!plan || !a_host || !b_host) return fail(PERM_EINVAL, "null plan or buffer");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
+    const size_t bytes = (size_t)plan->host.n * plan->host.eb;
+    cudaError_t e;
+    if (!plan->d_stage[0]) {
+        for (int i = 0; i < 2; ++i) {
+            e = cudaMalloc(&plan->d_stage[i], bytes);
+            if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc staging: ") + cudaGetErrorString(e));
+        }
+    }
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    e = cudaMemcpyAsync(plan->d_stage[0], a_host, bytes, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync H2D");
+    int st = perm_apply(plan, plan->d_stage[0], plan->d_stage[1], stream);
+    if (st != PERM_OK) return st;
+    e = cudaMemcpyAsync(b_host, plan->d_stage[1], bytes, cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync D2H");
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+    return PERM_OK;
+}
+
+int perm_scatter_baseline(const int32_t* p_dev, const void* a, void* b, int64_t n,
+                          int32_t elem_bytes, perm_stream_t stream) {
+    if (!p_dev || !a || !b || n <= 0) return fail(PERM_EINVAL, "null argument or n <= 0");
+    if (elem_bytes != 4 || (n & 3)) return fail(PERM_EUNSUPPORTED, "elem_bytes 4, n % 4 == 0");
+    cudaError_t e = perm::launch_scatter(p_dev, static_cast<const uint32_t*>(a),
+                                         static_cast<uint32_t*>(b), n,
+                                         static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "scatter launch");
+    return PERM_OK;
+}
+
+int perm_gather_baseline(const int32_t* q_dev, const void* a, void* b, int64_t n,
+                         int32_t elem_bytes, perm_stream_t stream) {
+    if (!q_dev || !a || !b || n <= 0) return fail(PERM_EINVAL, "null argument or n <= 0");
+    if (elem_bytes != 4 || (n & 3)) return fail(PERM_EUNSUPPORTED, "elem_bytes 4, n % 4 == 0");
+    cudaError_t e = perm::launch_gather(q_dev, static_cast<const uint32_t*>(a),
+                                        static_cast<uint32_t*>(b), n,
+                                        static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "gather launch");
+    return PERM_OK;
+}
+
+int perm_copy_kernel(const void* a, void* b, int64_t n, int32_t elem_bytes, perm_stream_t stream) {
+    if (!a || !b || n <= 0) return fail(PERM_EINVAL, "null argument or n <= 0");
+    const int64_t words = n * elem_bytes / 4;
+    if (words & 3) return fail(PERM_EUNSUPPORTED, "n*elem_bytes must be a multiple of 16");
+    cudaError_t e = perm::launch_copy(static_cast<const uint32_t*>(a), static_cast<uint32_t*>(b),
+                                      words, static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "copy launch");
+    return PERM_OK;
+}
+
+int perm_last_error(void) { return g_status; }
+const char* perm_last_error_string(void) { return g_msg.c_str(); }
+const char* perm_version(void) { return "libperm 0.1 (sm_100a)"; }
+
+}  // extern "C"

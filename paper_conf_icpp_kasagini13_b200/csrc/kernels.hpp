@@ -1,0 +1,34 @@
+// kernels.hpp — launchers of the sm_100a kernels (libperm internals).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "plan.hpp"
+
+namespace perm {
+
+// Registers max dynamic shared memory for every kernel instantiation the plan uses.
+cudaError_t prepare_kernels(const HostPlan& P);
+
+// All three phases in one CTA (n <= 2^15): a -> smem -> R1, R2 (columns), R3 -> b.
+cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
+                         uint32_t* b, cudaStream_t s);
+
+// One row pass (pass index f in 0..2) of the 3- or 5-pass pipeline.
+cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, const uint32_t* in,
+                            uint32_t* out, cudaStream_t s, bool pdl);
+
+// out (cols x rows) = transpose of in (rows x cols), 32 x 32 tiles (§V).
+cudaError_t launch_transpose(const uint32_t* in, uint32_t* out, int64_t rows, int64_t cols,
+                             cudaStream_t s, bool pdl);
+
+// Comparators and a plain vector copy.
+cudaError_t launch_scatter(const int32_t* p, const uint32_t* a, uint32_t* b, int64_t n,
+                           cudaStream_t s);
+cudaError_t launch_gather(const int32_t* q, const uint32_t* a, uint32_t* b, int64_t n,
+                          cudaStream_t s);
+cudaError_t launch_copy(const uint32_t* a, uint32_t* b, int64_t n, cudaStream_t s);
+
+}  // namespace perm

@@ -1,0 +1,96 @@
+// plan.hpp — host-side plan of the scheduled offline permutation (libperm internals).
+//
+// PAPER.md §VI-§VII: P is split into three per-line permutations Phi1 (rows),
+// Phi2 (columns), Phi3 (rows) of an r x c view (L537-L539, L603-L605), and
+// every line's permutation into warp-rounds whose 32 reads and 32 writes hit
+// 32 distinct shared-memory banks (L531-L533). This header describes what the
+// planner (planner.cpp) produces and the kernels (kernels.cu) consume.
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/perm.h"
+
+namespace perm {
+
+constexpr int kW = 32;                 // HMM width w = warp size = banks (L199-L207)
+
+// One phase of row-wise permutations: `lines` independent lines of length L.
+// Packed schedule: for line g and warp-round k (k < L/32) there are E 32-bit
+// words; the entry of lane x occupies bits [E*x, E*x + E) of those words
+// (LSB first). entry = (sigma << logL) | t: the lane reads source position
+// s = 32*sigma + x (bank x) and writes destination position t (L519, L533).
+struct PhaseGeom {
+    int64_t lines = 0;
+    int32_t L = 0, logL = 0;
+    int32_t E = 0;        // entry bits = logL + (logL - 5)
+    int64_t words = 0;    // lines * (L/32) * E
+};
+
+// Layout of one row pass of the tiled 3-pass pipeline.
+// Element (line l, position pos) of CTA `cta` lives in global memory at
+//   RUNS : cta*cta_stride + (pos / w) * strideK + l * w + pos % w
+//   CROSS: cta*cta_stride + (pos / blockP) * strideP + (pos % blockP) * h + l
+struct IoMode {
+    int32_t cross = 0;
+    int32_t w = 0;            // RUNS run width (w = L means whole contiguous lines)
+    int64_t strideK = 0;      // RUNS
+    int32_t blockP = 0;       // CROSS
+    int64_t strideP = 0;      // CROSS
+    int64_t cta_stride = 0;
+};
+
+struct RowPass {
+    int32_t phase = 0;        // 0,1,2 -> Phi1, Phi2, Phi3
+    int32_t h = 0;            // lines per CTA
+    int32_t Ls = 0;           // shared-memory line stride (elements) = L + pad
+    int32_t ept = 0;          // elements per thread
+    int32_t threads = 0;
+    int64_t ctas = 0;
+    IoMode in, out;
+    int32_t conflicts_in = 1, conflicts_out = 1;   // simulated wavefronts per request
+};
+
+struct HostPlan {
+    int64_t n = 0;
+    int32_t eb = 4;
+    int32_t k = 0;             // log2 n
+    int64_t r = 0, c = 0;      // view
+    int32_t passes = 0;        // 1, 3, 5
+    PhaseGeom ph[3];
+    RowPass rp[3];
+    int32_t fused_ept = 0, fused_threads = 0, fused_Ls = 0;
+    std::vector<uint16_t> kappa;
+    std::vector<uint32_t> sched[3];
+    double ms_colour = 0, ms_bank = 0;
+    int32_t threads_used = 1;
+};
+
+// Builds everything host-side. Returns PERM_OK or a perm_status, with `err` set.
+int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
+                    HostPlan& out, std::string& err);
+
+// Colour a d-regular bipartite multigraph (d a power of two) with d colours by
+// recursive Euler splitting. U[e], V[e] < nodes, E = nodes * d edges.
+void euler_split_colour(int64_t nodes, int64_t d, int64_t E, const uint32_t* U,
+                        const uint32_t* V, uint32_t* colour, bool parallel);
+
+// Decode the entry of (line, slot q = round*32 + lane) from a packed phase.
+inline uint32_t unpack_entry(const std::vector<uint32_t>& words, const PhaseGeom& g,
+                             int64_t line, int64_t q) {
+    const int64_t round = q >> 5, lane = q & 31;
+    const uint64_t bit = (uint64_t)((line * (g.L >> 5) + round) * (int64_t)g.E) * 32u +
+                         (uint64_t)(g.E * lane);
+    const uint64_t w0 = bit >> 5, off = bit & 31;
+    uint64_t v = words[w0];
+    if (off + g.E > 32) v |= (uint64_t)words[w0 + 1] << 32;
+    return (uint32_t)((v >> off) & ((1ull << g.E) - 1));
+}
+
+// Simulated shared-memory wavefronts per warp request of a pass's load/store
+// loops (1 = conflict-free). Mirrors the index math in kernels.cu.
+int simulate_conflicts(const RowPass& rp, const PhaseGeom& g, bool input_side);
+
+}  // namespace perm

@@ -1,0 +1,418 @@
+// planner.cpp — offline plan builder of libperm (host, C++17 + OpenMP).
+//
+// PAPER.md §VII (L603-L605, L537-L539) and §VI (L515-L533):
+//  1. validate P (L361: p holds a permutation of 0..n-1);
+//  2. view the arrays as r x c (L603, "not restricted to a square matrix");
+//  3. colour the c-regular row-level bipartite multigraph (U = source rows,
+//     V = destination rows, one edge per element) with c colours (Thm 6);
+//  4. derive the three per-line permutations Phi1 (colour k -> column k),
+//     Phi2 (within column k, to the destination row), Phi3 (within the
+//     destination row, to the destination column);
+//  5. for every line of every phase colour its (L/32)-regular bank-level
+//     graph (edge (j mod 32, Phi(j) mod 32)) with L/32 colours: colour k is
+//     warp-round k, and lane x takes the colour-k edge leaving bank x
+//     (s = 32*sigma + x, t = Phi(s));
+//  6. pack (sigma, t) into 2*log2(L)-5 bit entries.
+//
+// The paper proves the colourings exist (König) but gives no algorithm; we
+// use Euler splitting, valid because every degree here is a power of two:
+// pair the edges at every node, the pairings form disjoint even alternating
+// cycles, colour each cycle 0,1,0,1,...: every node keeps exactly half its
+// edges on each side. Recurse log2(d) times. O(E log d).
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <numeric>
+
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#include "plan.hpp"
+
+namespace perm {
+
+namespace {
+
+using clk = std::chrono::steady_clock;
+double ms_since(clk::time_point t0) {
+    return std::chrono::duration<double, std::milli>(clk::now() - t0).count();
+}
+
+int ilog2(int64_t v) {
+    int k = 0;
+    while ((int64_t(1) << k) < v) ++k;
+    return k;
+}
+
+int64_t pow2_floor(int64_t v) {
+    if (v < 1) return 1;
+    int64_t p = 1;
+    while (p * 2 <= v) p *= 2;
+    return p;
+}
+
+constexpr uint32_t kNone = 0xFFFFFFFFu;
+
+// Reusable Euler-split colourer (scratch kept across calls).
+struct EulerColourer {
+    std::vector<uint32_t> ord, ord2, pu, pu2, pv, pv2, pL, pR;
+    std::vector<uint8_t> bit;
+
+    void split_group(int64_t base, int64_t S, int64_t nodes, std::vector<uint32_t>& pend) {
+        // pair consecutive incident edges at every left node, then every right node
+        std::fill(pend.begin(), pend.begin() + nodes, kNone);
+        for (int64_t i = base; i < base + S; ++i) {
+            uint32_t& q = pend[pu[i]];
+            if (q == kNone) q = (uint32_t)i;
+            else { pL[i] = q; pL[q] = (uint32_t)i; q = kNone; }
+        }
+        std::fill(pend.begin(), pend.begin() + nodes, kNone);
+        for (int64_t i = base; i < base + S; ++i) {
+            uint32_t& q = pend[pv[i]];
+            if (q == kNone) q = (uint32_t)i;
+            else { pR[i] = q; pR[q] = (uint32_t)i; q = kNone; }
+        }
+        // walk the alternating cycles, colouring 0,1,0,1,...
+        std::memset(bit.data() + base, 2, (size_t)S);
+        for (int64_t i = base; i < base + S; ++i) {
+            if (bit[i] != 2) continue;
+            uint32_t cur = (uint32_t)i;
+            do {
+                bit[cur] = 0;
+                uint32_t nx = pL[cur];
+                bit[nx] = 1;
+                cur = pR[nx];
+            } while (cur != (uint32_t)i);
+        }
+        // stable partition: bit 0 first half, bit 1 second half
+        int64_t z = base, o = base + S / 2;
+        for (int64_t i = base; i < base + S; ++i) {
+            int64_t dst = bit[i] ? o++ : z++;
+            ord2[dst] = ord[i];
+            pu2[dst] = pu[i];
+            pv2[dst] = pv[i];
+        }
+    }
+
+    void run(int64_t nodes, int64_t d, int64_t E, const uint32_t* U, const uint32_t* V,
+             uint32_t* colour, bool parallel) {
+        if (d <= 1) {
+            std::fill(colour, colour + E, 0u);
+            return;
+        }
+        if ((int64_t)ord.size() < E) {
+            ord.resize(E); ord2.resize(E); pu.resize(E); pu2.resize(E);
+            pv.resize(E); pv2.resize(E); pL.resize(E); pR.resize(E); bit.resize(E);
+        }
+        for (int64_t i = 0; i < E; ++i) { ord[i] = (uint32_t)i; pu[i] = U[i]; pv[i] = V[i]; }
+        const int levels = ilog2(d);
+        for (int lvl = 0; lvl < levels; ++lvl) {
+            const int64_t G = int64_t(1) << lvl, S = E / G;
+            if (parallel && G > 1) {
+#pragma omp parallel
+                {
+                    std::vector<uint32_t> pend(nodes);
+#pragma omp for schedule(dynamic, 1)
+                    for (int64_t g = 0; g < G; ++g) split_group(g * S, S, nodes, pend);
+                }
+            } else {
+                std::vector<uint32_t> pend(nodes);
+                for (int64_t g = 0; g < G; ++g) split_group(g * S, S, nodes, pend);
+            }
+            ord.swap(ord2); pu.swap(pu2); pv.swap(pv2);
+        }
+        const int64_t per = E / d;   // a perfect matching per colour
+        for (int64_t i = 0; i < E; ++i) colour[ord[i]] = (uint32_t)(i / per);
+    }
+};
+
+// ---------------------------------------------------------------- conflict model
+
+// Wavefronts of one 128-bit shared access by a warp: 4 phases of 8 lanes,
+// each phase needs one wavefront per distinct 16-byte chunk in one bank group.
+int wavefronts_v4(const int64_t* addr /*32 element addresses, 16B aligned*/) {
+    int total = 0;
+    for (int q = 0; q < 4; ++q) {
+        int worst = 0;
+        for (int bg = 0; bg < 8; ++bg) {
+            int64_t seen[8];
+            int cnt = 0;
+            for (int l = 0; l < 8; ++l) {
+                int64_t ch = addr[q * 8 + l] >> 2;
+                if ((ch & 7) != bg) continue;
+                bool dup = false;
+                for (int u = 0; u < cnt; ++u) dup |= seen[u] == ch;
+                if (!dup) seen[cnt++] = ch;
+            }
+            worst = std::max(worst, cnt);
+        }
+        total += std::max(worst, 1);
+    }
+    return (total + 3) / 4;
+}
+
+// Wavefronts of one 32-bit shared access by a warp.
+int wavefronts_s(const int64_t* addr) {
+    int worst = 0;
+    for (int b = 0; b < 32; ++b) {
+        int64_t seen[32];
+        int cnt = 0;
+        for (int l = 0; l < 32; ++l) {
+            if ((addr[l] & 31) != b) continue;
+            bool dup = false;
+            for (int u = 0; u < cnt; ++u) dup |= seen[u] == addr[l];
+            if (!dup) seen[cnt++] = addr[l];
+        }
+        worst = std::max(worst, cnt);
+    }
+    return std::max(worst, 1);
+}
+
+}  // namespace
+
+void euler_split_colour(int64_t nodes, int64_t d, int64_t E, const uint32_t* U,
+                        const uint32_t* V, uint32_t* colour, bool parallel) {
+    EulerColourer ec;
+    ec.run(nodes, d, E, U, V, colour, parallel);
+}
+
+// Mirrors the load/store loops of row_pass_kernel (kernels.cu): thread tid,
+// iteration it handles the 4-element vector f = 4*(tid + T*it).
+int simulate_conflicts(const RowPass& rp, const PhaseGeom& g, bool input_side) {
+    const IoMode& m = input_side ? rp.in : rp.out;
+    const int64_t L = g.L, h = rp.h, T = rp.threads, total = h * L;
+    const int64_t iters = total / (4 * T);
+    int worst = 1;
+    int64_t addr[32];
+    for (int64_t it = 0; it < iters; ++it) {
+        for (int64_t w0 = 0; w0 < T; w0 += 32) {
+            if (!m.cross) {
+                for (int l = 0; l < 32; ++l) {
+                    int64_t f = 4 * (w0 + l + T * it);
+                    int64_t K = f / (h * m.w), line = (f / m.w) % h, kk = f % m.w;
+                    addr[l] = line * rp.Ls + K * m.w + kk;
+                }
+                worst = std::max(worst, wavefronts_v4(addr));
+            } else {
+                for (int j = 0; j < 4; ++j) {
+                    for (int l = 0; l < 32; ++l) {
+                        int64_t f = 4 * (w0 + l + T * it);
+                        int64_t pos = f / h, line = f % h + j;
+                        addr[l] = line * rp.Ls + pos;
+                    }
+                    worst = std::max(worst, wavefronts_s(addr));
+                }
+            }
+        }
+    }
+    return worst;
+}
+
+namespace {
+
+void choose_threads(RowPass& rp, int64_t L) {
+    const int64_t total = rp.h * L;
+    int ept = 16;
+    while (total / ept > 512 && ept < 64) ept *= 2;
+    while (total / ept < 64 && ept > 4) ept /= 2;
+    rp.ept = ept;
+    rp.threads = (int32_t)(total / ept);
+}
+
+void choose_pad(RowPass& rp, const PhaseGeom& g) {
+    const bool needs_v4 = !rp.in.cross || !rp.out.cross;
+    int best_pad = 0, best = 1 << 30;
+    for (int pad = 0; pad < 32; ++pad) {
+        if (needs_v4 && (pad & 3)) continue;
+        rp.Ls = g.L + pad;
+        int ci = simulate_conflicts(rp, g, true);
+        int co = simulate_conflicts(rp, g, false);
+        if (ci + co < best) { best = ci + co; best_pad = pad; }
+        if (best == 2) break;
+    }
+    rp.Ls = g.L + best_pad;
+    rp.conflicts_in = simulate_conflicts(rp, g, true);
+    rp.conflicts_out = simulate_conflicts(rp, g, false);
+}
+
+IoMode runs(int64_t w, int64_t strideK, int64_t cta_stride) {
+    IoMode m;
+    m.cross = 0; m.w = (int32_t)w; m.strideK = strideK; m.cta_stride = cta_stride;
+    return m;
+}
+IoMode cross(int64_t blockP, int64_t strideP, int64_t cta_stride) {
+    IoMode m;
+    m.cross = 1; m.blockP = (int32_t)blockP; m.strideP = strideP; m.cta_stride = cta_stride;
+    return m;
+}
+
+}  // namespace
+
+int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
+                    HostPlan& P, std::string& err) {
+    if (!p || n <= 0) { err = "null p or n <= 0"; return PERM_EINVAL; }
+    if (eb != 4) { err = "elem_bytes must be 4"; return PERM_EUNSUPPORTED; }
+    const int k = ilog2(n);
+    if ((int64_t(1) << k) != n || k < 10 || k > 30) {
+        err = "n must be a power of two in [2^10, 2^30]";
+        return PERM_EUNSUPPORTED;
+    }
+    // 1. validate: bijection onto [0, n)
+    {
+        std::vector<uint8_t> seen((size_t)n, 0);
+        for (int64_t i = 0; i < n; ++i) {
+            const int32_t v = p[i];
+            if (v < 0 || v >= n || seen[v]) {
+                err = "p is not a permutation: entry " + std::to_string(i) + " = " +
+                      std::to_string(v);
+                return PERM_ENOTPERM;
+            }
+            seen[v] = 1;
+        }
+    }
+    P.n = n; P.eb = eb; P.k = k;
+    P.r = int64_t(1) << (k / 2);
+    P.c = int64_t(1) << (k - k / 2);
+    const int64_t r = P.r, c = P.c;
+    const int logc = k - k / 2, logr = k / 2;
+#ifdef _OPENMP
+    P.threads_used = omp_get_max_threads();
+#endif
+
+    // 2-3. row-level colouring
+    auto t0 = clk::now();
+    std::vector<uint32_t> colour((size_t)n);
+    {
+        std::vector<uint32_t> U((size_t)n), V((size_t)n);
+#pragma omp parallel for schedule(static)
+        for (int64_t x = 0; x < n; ++x) {
+            U[x] = (uint32_t)(x >> logc);
+            V[x] = (uint32_t)((uint32_t)p[x] >> logc);
+        }
+        EulerColourer ec;
+        ec.run(r, c, n, U.data(), V.data(), colour.data(), true);
+    }
+    P.kappa.resize((size_t)n);
+#pragma omp parallel for schedule(static)
+    for (int64_t x = 0; x < n; ++x) P.kappa[x] = (uint16_t)colour[x];
+    colour.clear();
+    colour.shrink_to_fit();
+    P.ms_colour = ms_since(t0);
+
+    // 4. phase permutations as per-line arrays (uint16: every L <= 2^15)
+    t0 = clk::now();
+    std::vector<uint16_t> phi[3];
+    for (auto& v : phi) v.resize((size_t)n);
+#pragma omp parallel for schedule(static)
+    for (int64_t x = 0; x < n; ++x) {
+        const int64_t i = x >> logc;
+        const uint32_t kk = P.kappa[x];
+        const uint32_t dest = (uint32_t)p[x];
+        const uint32_t drow = dest >> logc, dcol = dest & (uint32_t)(c - 1);
+        phi[0][x] = (uint16_t)kk;                               // Phi1_i(j) = kappa(x)
+        phi[1][(int64_t)kk * r + i] = (uint16_t)drow;           // Phi2_k(i) = P(x) div c
+        phi[2][(int64_t)drow * c + kk] = (uint16_t)dcol;        // Phi3_i'(k) = P(x) mod c
+    }
+    // 5-6. bank-level colouring of every line, packed
+    const int64_t lines[3] = {r, c, r};
+    const int64_t Ls[3] = {c, r, c};
+    const int logLs[3] = {logc, logr, logc};
+    for (int f = 0; f < 3; ++f) {
+        PhaseGeom& g = P.ph[f];
+        g.lines = lines[f];
+        g.L = (int32_t)Ls[f];
+        g.logL = logLs[f];
+        g.E = 2 * g.logL - 5;
+        g.words = g.lines * (g.L / kW) * g.E;
+        P.sched[f].assign((size_t)g.words, 0u);
+        const int64_t L = g.L;
+        const uint16_t* ph = phi[f].data();
+        uint32_t* W = P.sched[f].data();
+#pragma omp parallel
+        {
+            EulerColourer ec;
+            std::vector<uint32_t> U((size_t)L), V((size_t)L), col((size_t)L);
+#pragma omp for schedule(dynamic, 16)
+            for (int64_t line = 0; line < g.lines; ++line) {
+                const uint16_t* phl = ph + line * L;
+                for (int64_t j = 0; j < L; ++j) {
+                    U[j] = (uint32_t)(j & 31);
+                    V[j] = (uint32_t)(phl[j] & 31);
+                }
+                ec.run(kW, L / kW, L, U.data(), V.data(), col.data(), false);
+                uint32_t* Wl = W + line * (L / kW) * g.E;
+                for (int64_t j = 0; j < L; ++j) {
+                    const uint64_t sigma = (uint64_t)(j >> 5), lane = (uint64_t)(j & 31);
+                    const uint64_t entry = (sigma << g.logL) | phl[j];
+                    const uint64_t bit = (uint64_t)col[j] * g.E * 32u + (uint64_t)g.E * lane;
+                    const uint64_t w0 = bit >> 5, off = bit & 31;
+                    Wl[w0] |= (uint32_t)(entry << off);
+                    if (off + g.E > 32) Wl[w0 + 1] |= (uint32_t)(entry >> (32 - off));
+                }
+            }
+        }
+    }
+    P.ms_bank = ms_since(t0);
+
+    // pass structure
+    int passes = opt ? opt->passes : 0;
+    if (passes == 0) passes = (k <= 15) ? 1 : (k <= 26 ? 3 : 5);
+    if (passes == 1 && k > 15) { err = "fused single-CTA pass needs n <= 2^15"; return PERM_EUNSUPPORTED; }
+    if (passes != 1 && passes != 3 && passes != 5) { err = "passes must be 0, 1, 3 or 5"; return PERM_EINVAL; }
+    P.passes = passes;
+    if (passes == 1) {
+        P.fused_threads = (int32_t)std::min<int64_t>(512, n / 4);
+        P.fused_ept = (int32_t)(n / P.fused_threads);
+        P.fused_Ls = (int32_t)(c + 1);   // odd stride: rows AND columns conflict-free (Fig. 4 idea)
+        return PERM_OK;
+    }
+    const int64_t Q = std::min<int64_t>(16384, std::max<int64_t>(2048, pow2_floor(n / 296)));
+    auto pick = [&](int idx, int64_t dflt) -> int64_t {
+        int64_t v = opt ? (&opt->h1)[idx] : 0;
+        return v > 0 ? v : dflt;
+    };
+    if (passes == 3) {
+        int64_t h2 = pick(1, std::min<int64_t>(32, std::max<int64_t>(4, pow2_floor(Q / r))));
+        int64_t h1 = pick(0, std::max<int64_t>(1, pow2_floor(Q / c)));
+        int64_t h3 = pick(2, h1);
+        h2 = std::min(h2, c);
+        if (h2 < 4 || h2 > 32 || (h2 & (h2 - 1)) || h1 < 1 || h1 > r || (h1 & (h1 - 1)) ||
+            h3 < 1 || h3 > r || (h3 & (h3 - 1))) {
+            err = "invalid h1/h2/h3 for the 3-pass layout (h2 in {4,8,16,32}, powers of two)";
+            return PERM_EINVAL;
+        }
+        RowPass& a = P.rp[0];
+        a.phase = 0; a.h = (int32_t)h1; a.ctas = r / h1;
+        a.in = runs(c, 0, h1 * c);
+        a.out = runs(h2, r * h2, h1 * h2);
+        RowPass& b = P.rp[1];
+        b.phase = 1; b.h = (int32_t)h2; b.ctas = c / h2;
+        b.in = cross(r, 0, r * h2);
+        b.out = cross(h3, c * h3, h3 * h2);
+        RowPass& d = P.rp[2];
+        d.phase = 2; d.h = (int32_t)h3; d.ctas = r / h3;
+        d.in = runs(h2, h3 * h2, h3 * c);
+        d.out = runs(c, 0, h3 * c);
+    } else {
+        for (int f = 0; f < 3; ++f) {
+            const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
+            int64_t h = pick(f, std::max<int64_t>(1, pow2_floor(Q / L)));
+            if (h < 1 || h > lines_f || (h & (h - 1))) { err = "invalid h for the 5-pass layout"; return PERM_EINVAL; }
+            RowPass& rp = P.rp[f];
+            rp.phase = f; rp.h = (int32_t)h; rp.ctas = lines_f / h;
+            rp.in = runs(L, 0, h * L);
+            rp.out = runs(L, 0, h * L);
+        }
+    }
+    for (int f = 0; f < 3; ++f) {
+        RowPass& rp = P.rp[f];
+        const PhaseGeom& g = P.ph[rp.phase];
+        if ((int64_t)rp.h * g.L * 4 > 200 * 1024) { err = "a CTA's lines exceed the shared-memory budget"; return PERM_EINVAL; }
+        choose_threads(rp, g.L);
+        choose_pad(rp, g);
+    }
+    return PERM_OK;
+}
+
+}  // namespace perm

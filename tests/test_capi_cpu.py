@@ -1,0 +1,161 @@
+"""CPU-side tests of libperm: the library loads, exports every symbol the header
+declares, validates its inputs, and its C++ planner's exported plans satisfy
+the oracle's invariants (i)-(vii) — checked by oracle/check.py, which shares
+no code with the planner — and drive the paper-faithful emulator to b[P(i)] = a[i].
+No compute call touches a GPU here (perm_plan_create_host)."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import apply as OA
+from oracle import check as OC
+from oracle import emulate as OE
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_icpp_kasagini13_b200 import build
+    build.build()
+    import paper_conf_icpp_kasagini13_b200 as P
+    return P
+
+
+def header_functions():
+    txt = open(os.path.join(ROOT, "include", "perm.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(perm_[a-z_0-9]+)\s*\(", txt)))
+
+
+def test_exports_every_declared_symbol(lib):
+    names = header_functions()
+    assert "perm_plan_create" in names and "perm_apply" in names and "perm_plan_destroy" in names
+    so = ctypes.CDLL(lib.LIB_PATH)
+    missing = [n for n in names if not hasattr(so, n)]
+    assert not missing, missing
+
+
+def test_library_is_sm100a(lib):
+    import subprocess
+    out = subprocess.run(["cuobjdump", "--list-elf", lib.LIB_PATH], capture_output=True, text=True)
+    assert "sm_100a" in out.stdout
+
+
+def decode(sched):
+    s = np.asarray(sched, dtype=np.uint32)
+    return (s >> 16).astype(np.int64), (s & 0xFFFF).astype(np.int64)
+
+
+def export_plan(lib, p, **kw):
+    with lib.Plan(p, device=False, **kw) as pl:
+        info = pl.info()
+        kappa, scheds = pl.export()
+    return info, kappa.astype(np.int64), [decode(s) for s in scheds]
+
+
+@pytest.mark.parametrize("fam", W.FAMILIES)
+@pytest.mark.parametrize("k", [10, 11, 12, 13, 14, 15, 16])
+def test_cpp_plan_passes_oracle_checker(lib, fam, k):
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=42 + k)
+    info, kappa, sched = export_plan(lib, p)
+    r, c = W.view_shape(n)
+    assert (info["rows"], info["cols"]) == (r, c)
+    OC.assert_plan(p, kappa, sched, r, c, 32)
+    for f, L in enumerate((c, r, c)):
+        assert info["entry_bits"][f] == 2 * (L.bit_length() - 1) - 5
+
+
+@pytest.mark.parametrize("k", [12, 13])
+def test_cpp_plan_drives_emulator(lib, k):
+    n = 1 << k
+    r, c = W.view_shape(n)
+    a = W.make_data(n)
+    for fam in W.FAMILIES:
+        p = W.make_perm(fam, n)
+        _, kappa, sched = export_plan(lib, p)
+        b, rc = OE.scheduled(a, sched, r, c, 32)
+        assert np.array_equal(b, OA.apply_ref(p, a))
+        t = rc.table()
+        assert t[("global", "read", "coalesced")] == 11 and t[("global", "write", "coalesced")] == 5
+        assert t[("shared", "read", "conflict-free")] == 8
+        assert t[("shared", "write", "conflict-free")] == 8
+
+
+@pytest.mark.parametrize("k", [18, 20])
+def test_cpp_plan_larger(lib, k):
+    n = 1 << k
+    r, c = W.view_shape(n)
+    for fam in ("random", "bitrev"):
+        p = W.make_perm(fam, n)
+        _, kappa, sched = export_plan(lib, p)
+        OC.assert_plan(p, kappa, sched, r, c, 32)
+
+
+def test_cpp_plan_22_random(lib):
+    n = 1 << 22
+    r, c = W.view_shape(n)
+    p = W.random(n, 42)
+    info, kappa, sched = export_plan(lib, p)
+    OC.assert_plan(p, kappa, sched, r, c, 32)
+    assert info["passes"] == 3
+    # schedule = (2 log2 L - 5) bits per element per phase: 3 * 17 bits at L = 2048
+    assert info["sched_bytes"] == 3 * n * 17 // 8
+
+
+def test_pass_options_and_info(lib):
+    n = 1 << 16
+    p = W.random(n, 1)
+    for passes in (3, 5):
+        with lib.Plan(p, device=False, passes=passes) as pl:
+            info = pl.info()
+            assert info["passes"] == passes
+            assert info["kernels_per_apply"] == passes
+    with lib.Plan(W.random(1 << 12, 1), device=False) as pl:
+        assert pl.info()["passes"] == 1
+    with lib.Plan(p, device=False, passes=3, h=(4, 8, 4)) as pl:
+        assert pl.info()["h"] == [4, 8, 4]
+
+
+def test_errors(lib):
+    with pytest.raises(lib.PermError) as e:
+        lib.Plan(np.array([0, 0] + list(range(2, 1024)), dtype=np.int32), device=False)
+    assert e.value.status == -2
+    with pytest.raises(lib.PermError) as e:
+        lib.Plan(np.arange(1000, dtype=np.int32), device=False)
+    assert e.value.status == -3
+    with pytest.raises(lib.PermError) as e:
+        lib.Plan(np.arange(1024, dtype=np.int32), elem_bytes=2, device=False)
+    assert e.value.status == -3
+    bad = np.arange(1024, dtype=np.int32)
+    bad[5] = 1024
+    with pytest.raises(lib.PermError) as e:
+        lib.Plan(bad, device=False)
+    assert e.value.status == -2
+    with pytest.raises(lib.PermError) as e:
+        lib.Plan(W.random(1 << 16, 1), device=False, passes=3, h=(4, 3, 4))
+    assert e.value.status == -1
+    # a host-only plan cannot apply
+    with lib.Plan(W.random(1 << 12, 1), device=False) as pl:
+        with pytest.raises(lib.PermError) as e:
+            pl.apply(1 << 20, 2 << 20, stream=0)
+        assert e.value.status == -7
+
+
+def test_bruteforce_tiny_via_cpp_euler_split(lib):
+    # the smallest view the library supports is 32 x 32; exhaustively permute
+    # one 8-element block of rows inside an otherwise random permutation
+    import itertools
+    n = 1 << 10
+    base = W.random(n, 5)
+    r, c = W.view_shape(n)
+    for perm in itertools.islice(itertools.permutations(range(8)), 0, 40320, 97):
+        p = base.copy()
+        p[:8] = base[list(perm)]
+        _, kappa, sched = export_plan(lib, p)
+        OC.assert_plan(p, kappa, sched, r, c, 32)

@@ -1,0 +1,209 @@
+"""GPU parity: libperm's CUDA path vs the oracle, bit-exact (tolerance 0).
+
+Inputs come from workloads/ (seeded); expected values from oracle.apply_ref
+(b[P(i)] = a[i]), compared as raw 32-bit words.
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import apply as OA
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_kasagini13_b200 import build
+    build.build()
+    import paper_conf_icpp_kasagini13_b200 as pkg
+    return pkg
+
+
+def dev(x: np.ndarray):
+    return torch.from_numpy(x.view(np.int32)).cuda()
+
+
+def host_words(t) -> np.ndarray:
+    return t.cpu().numpy().view(np.uint32)
+
+
+def run(P, p, a, **kw):
+    with P.Plan(p, **kw) as plan:
+        da = dev(a)
+        db = torch.full_like(da, -1)
+        plan.apply(da, db)
+        torch.cuda.synchronize()
+        return host_words(db), plan.info()
+
+
+@pytest.mark.parametrize("fam", W.FAMILIES)
+@pytest.mark.parametrize("k", [10, 12, 13, 15])
+def test_fused_single_cta(P, fam, k):
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=100 + k)
+    a = W.make_data(n)
+    b, info = run(P, p, a)
+    assert info["passes"] == 1
+    assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+def test_config0_bitrev_4096(P):
+    # BASELINE configs[0]: n = 4096 (64 x 64) bit-reversal, bit-exact against the oracle
+    n = 4096
+    p = W.bitrev(n)
+    a = W.make_data(n)
+    for passes in (0, 3, 5):
+        b, info = run(P, p, a, passes=passes)
+        assert (info["rows"], info["cols"]) == (64, 64)
+        assert np.array_equal(b, OA.apply_ref(p, a)), passes
+
+
+@pytest.mark.parametrize("passes", [3, 5])
+@pytest.mark.parametrize("fam", W.FAMILIES)
+@pytest.mark.parametrize("k", [12, 15, 16, 17, 19, 20])
+def test_multi_pass(P, passes, fam, k):
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=7 + k)
+    a = W.make_data(n)
+    b, info = run(P, p, a, passes=passes)
+    assert info["passes"] == passes
+    assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+@pytest.mark.parametrize("h", [(1, 4, 1), (4, 4, 4), (8, 8, 8), (2, 16, 2), (16, 32, 4), (4, 8, 16)])
+def test_tile_shapes(P, h):
+    n = 1 << 18
+    p = W.random(n, 3)
+    a = W.make_data(n)
+    b, info = run(P, p, a, passes=3, h=h)
+    assert info["h"] == list(h)
+    assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+@pytest.mark.parametrize("fam", W.FAMILIES)
+def test_config1_4M_all_families(P, fam):
+    # BASELINE configs[1]: n = 2^22 float32, the five families of the paper (L373-L389)
+    n = 1 << 22
+    p = W.make_perm(fam, n)
+    a = W.make_data(n)
+    b, info = run(P, p, a)
+    assert np.array_equal(b, OA.apply_ref(p, a))
+    # the conventional kernels agree too
+    da, dp = dev(a), torch.from_numpy(p).cuda()
+    db = torch.empty_like(da)
+    P.scatter_baseline(dp, da, db)
+    torch.cuda.synchronize()
+    assert np.array_equal(host_words(db), OA.apply_ref(p, a))
+    dq = torch.from_numpy(OA.inverse(p)).cuda()
+    db2 = torch.empty_like(da)
+    P.gather_baseline(dq, da, db2)
+    torch.cuda.synchronize()
+    assert np.array_equal(host_words(db2), OA.apply_ref(p, a))
+
+
+def test_config1_random_seeds_and_5pass(P):
+    n = 1 << 22
+    a = W.make_data(n)
+    for seed in (42, 43, 44):
+        p = W.random(n, seed)
+        for passes in (3, 5):
+            b, _ = run(P, p, a, passes=passes)
+            assert np.array_equal(b, OA.apply_ref(p, a)), (seed, passes)
+
+
+@pytest.mark.parametrize("k", [21, 23, 24])
+def test_odd_and_larger_views(P, k):
+    n = 1 << k
+    p = W.random(n, k)
+    a = W.make_data(n)
+    b, _ = run(P, p, a)
+    assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+def test_config2_2pow26_random(P):
+    # BASELINE configs[2]: n = 2^26 random, the launch configuration bench.py times
+    n = 1 << 26
+    p = W.random(n, 42)
+    a = W.make_data(n)
+    b, info = run(P, p, a)
+    assert info["passes"] == 3
+    assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+def test_adversarial_payloads(P):
+    n = 1 << 16
+    a = np.array([0x7FC00001, 0xFFFFFFFF, 0x80000000, 0x00000001, 0x7F800000, 0xFF800000,
+                  0x00000000, 0x7FBFFFFF] * (n // 8), dtype=np.uint32)
+    a ^= np.arange(n, dtype=np.uint32) << np.uint32(20)
+    for fam in W.FAMILIES:
+        p = W.make_perm(fam, n)
+        b, _ = run(P, p, a)
+        assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+def test_repeated_apply_and_streams(P):
+    n = 1 << 20
+    p = W.random(n, 9)
+    a = W.make_data(n)
+    ref = OA.apply_ref(p, a)
+    with P.Plan(p) as plan:
+        da = dev(a)
+        s = torch.cuda.Stream()
+        with torch.cuda.stream(s):
+            outs = []
+            for _ in range(3):
+                db = torch.empty_like(da)
+                plan.apply(da, db, stream=s)
+                outs.append(db)
+        s.synchronize()
+        for db in outs:
+            assert np.array_equal(host_words(db), ref)
+
+
+def test_apply_host_e2e(P):
+    n = 1 << 22
+    p = W.random(n, 5)
+    a = W.make_data(n)
+    b = np.empty_like(a)
+    with P.Plan(p) as plan:
+        plan.apply_host(a, b)
+    assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+def test_profiling_pass_times(P):
+    n = 1 << 22
+    with P.Plan(W.random(n, 1)) as plan:
+        da = torch.zeros(n, dtype=torch.int32, device="cuda")
+        db = torch.empty_like(da)
+        plan.set_profiling(True)
+        plan.apply(da, db)
+        t = plan.pass_times()
+        assert len(t) == 3 and all(x > 0 for x in t)
+
+
+def test_apply_errors(P):
+    n = 1 << 16
+    with P.Plan(W.random(n, 1)) as plan:
+        da = torch.zeros(n + 16, dtype=torch.int32, device="cuda")
+        with pytest.raises(P.PermError) as e:
+            plan.apply(da, da)                      # aliasing
+        assert e.value.status == -1
+        with pytest.raises(P.PermError) as e:
+            plan.apply(da[4:], da[4 + n // 2:])     # overlapping
+        assert e.value.status == -1
+        with pytest.raises(P.PermError) as e:
+            plan.apply(da[1:], torch.empty_like(da))  # misaligned
+        assert e.value.status == -1
+
+
+def test_copy_kernel(P):
+    a = dev(W.make_data(1 << 20))
+    b = torch.empty_like(a)
+    P.copy_kernel(a, b)
+    torch.cuda.synchronize()
+    assert torch.equal(a, b)
