@@ -50,15 +50,28 @@ enum perm_status {
 /* Pass structures a plan may use (perm_plan_info.passes). */
 enum perm_passes {
     PERM_PASSES_AUTO  = 0,
-    PERM_PASSES_FUSED = 1,   /* n <= 2^15: all three phases inside one CTA's shared memory */
+    PERM_PASSES_FUSED = 1,   /* n <= 2^14: all three phases inside one CTA's shared memory */
     PERM_PASSES_3     = 3,   /* R1, R2, R3; both transposes absorbed into tiled layouts */
     PERM_PASSES_5     = 5    /* R, T, R, T, R: the paper's five kernel calls (L699) */
 };
 
+/* Intermediate layouts of the 3-pass pipeline (perm_plan_options.layout). */
+enum perm_layout {
+    PERM_LAYOUT_AUTO  = 0,
+    PERM_LAYOUT_TILED = 1,   /* reader transposes: X1, X2 stored as h1 x h2 / h3 x h2 tiles */
+    PERM_LAYOUT_LINES = 2    /* writer transposes: X1 column-major, X2 row-major; every pass
+                                reads whole lines with TMA bulk copies (persistent, pipelined) */
+};
+
 typedef struct {
     int32_t passes;      /* enum perm_passes; 0 = choose by n */
-    int32_t h1, h2, h3;  /* lines per CTA in the three row passes; 0 = choose */
-    int32_t reserved[8];
+    int32_t h1, h2, h3;  /* lines per CTA tile in the three row passes; 0 = choose */
+    int32_t layout;      /* enum perm_layout; 0 = choose by n */
+    int32_t stages;      /* TMA pipeline depth of the LINES layout (0 = as many as fit, <= 4) */
+    int32_t fuse;        /* LINES layout, square view: 1 = run the three passes as ONE persistent
+                            kernel with grid barriers; 0 = auto (currently three launches
+                            chained with programmatic dependent launch); -1 = never */
+    int32_t reserved[5];
 } perm_plan_options;
 
 typedef struct {
@@ -139,6 +152,14 @@ int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stre
  * most recent apply; returns the number written or a negative status. */
 int perm_plan_set_profiling(perm_plan* plan, int enable);
 int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k);
+
+/* Tracing (diagnostics): when enabled, every CTA of the three row passes
+ * records up to 16 %globaltimer stamps (ns) at its phase boundaries (start,
+ * after griddepcontrol.wait, per tile: data ready / permuted / stored, end).
+ * perm_plan_trace copies [pass][cta][16] stamps of the most recent apply to
+ * host memory (synchronous) and returns the number of entries (3*ctas*16). */
+int     perm_plan_set_tracing(perm_plan* plan, int enable);
+int64_t perm_plan_trace(const perm_plan* plan, uint64_t* out, int64_t max_entries);
 
 /* ------------------------------------------------------- comparators */
 

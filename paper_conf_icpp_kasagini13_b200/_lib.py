@@ -35,7 +35,8 @@ class PermError(RuntimeError):
 
 class PlanOptions(ctypes.Structure):
     _fields_ = [("passes", ctypes.c_int32), ("h1", ctypes.c_int32), ("h2", ctypes.c_int32),
-                ("h3", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+                ("h3", ctypes.c_int32), ("layout", ctypes.c_int32), ("stages", ctypes.c_int32),
+                ("fuse", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -76,6 +77,8 @@ _apply = _sig("perm_apply", ctypes.c_int, _vp, _vp, _vp, _vp)
 _apply_host = _sig("perm_apply_host", ctypes.c_int, _vp, _vp, _vp, _vp)
 _set_prof = _sig("perm_plan_set_profiling", ctypes.c_int, _vp, ctypes.c_int)
 _pass_times = _sig("perm_plan_pass_times", ctypes.c_int, _vp, ctypes.POINTER(ctypes.c_float), ctypes.c_int)
+_set_tracing = _sig("perm_plan_set_tracing", ctypes.c_int, _vp, ctypes.c_int)
+_trace = _sig("perm_plan_trace", _i64, _vp, _vp, _i64)
 _scatter = _sig("perm_scatter_baseline", ctypes.c_int, _vp, _vp, _vp, _i64, _i32, _vp)
 _gather = _sig("perm_gather_baseline", ctypes.c_int, _vp, _vp, _vp, _i64, _i32, _vp)
 _copy = _sig("perm_copy_kernel", ctypes.c_int, _vp, _vp, _i64, _i32, _vp)
@@ -125,11 +128,11 @@ class Plan:
     """perm_plan: the offline schedule of permutation p (int32, host)."""
 
     def __init__(self, p, elem_bytes: int = 4, passes: int = 0, h=(0, 0, 0),
-                 device: bool = True):
+                 device: bool = True, layout: int = 0, stages: int = 0, fuse: int = 0):
         p = _as_int32_host(p)
         self.n = int(p.size)
         self.elem_bytes = elem_bytes
-        opt = PlanOptions(passes, h[0], h[1], h[2])
+        opt = PlanOptions(passes, h[0], h[1], h[2], layout, stages, fuse)
         if device:
             handle = _plan_create_ex(p.ctypes.data, self.n, elem_bytes, ctypes.byref(opt))
         else:
@@ -197,6 +200,22 @@ class Plan:
 
     def set_profiling(self, on: bool = True):
         _check(_set_prof(self._h, 1 if on else 0))
+
+    def set_tracing(self, on: bool = True):
+        _check(_set_tracing(self._h, 1 if on else 0))
+
+    def trace(self) -> np.ndarray:
+        """[3, ctas, 16] uint64 %globaltimer stamps (ns) of the last apply (0 = not recorded)."""
+        n = _trace(self._h, None, 0)
+        if n < 0:
+            _raise(int(n))
+        if n == 0:
+            return np.zeros((3, 0, 16), dtype=np.uint64)
+        buf = np.zeros(n, dtype=np.uint64)
+        k = _trace(self._h, buf.ctypes.data, n)
+        if k < 0:
+            _raise(int(k))
+        return buf.reshape(3, -1, 16)
 
     def pass_times(self) -> list[float]:
         buf = (ctypes.c_float * 8)()

@@ -31,6 +31,10 @@ struct perm_plan {
     int n_events = 0;
     cudaEvent_t ev[8] = {};
     int last_kernels = 0;
+    // tracing: [row pass][cta][16] %globaltimer stamps
+    unsigned long long* d_trace = nullptr;
+    int64_t trace_stride = 0;          // CTAs per pass slot
+    unsigned long long* d_sync = nullptr;   // fused 3-pass grid-barrier counters
 };
 
 namespace {
@@ -58,6 +62,8 @@ void free_device(perm_plan* pl) {
     cudaFree(pl->d_scratch[1]);
     cudaFree(pl->d_stage[0]);
     cudaFree(pl->d_stage[1]);
+    cudaFree(pl->d_trace);
+    cudaFree(pl->d_sync);
     for (int i = 0; i < pl->n_events; ++i) cudaEventDestroy(pl->ev[i]);
     pl->n_events = 0;
     if (cur >= 0) cudaSetDevice(cur);
@@ -69,8 +75,9 @@ int upload(perm_plan* pl) {
     HostPlan& P = pl->host;
     cudaError_t e = cudaGetDevice(&pl->device);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    auto padded = [](int64_t w) { return (w + 32 + 63) / 64 * 64; };   // guard, 256-B aligned phases
     int64_t words = 0;
-    for (int f = 0; f < 3; ++f) words += P.ph[f].words + 32;   // +32: shuffle over-read guard
+    for (int f = 0; f < 3; ++f) words += padded(P.ph[f].words);
     pl->sched_bytes = words * 4;
     e = cudaMalloc(&pl->d_sched, (size_t)pl->sched_bytes);
     if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc schedules: ") + cudaGetErrorString(e));
@@ -83,7 +90,7 @@ int upload(perm_plan* pl) {
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy schedules");
         e = cudaMemset(pl->d_phase[f] + P.ph[f].words, 0, 32 * 4);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemset");
-        off += P.ph[f].words + 32;
+        off += padded(P.ph[f].words);
     }
     if (P.passes != 1) {
         const size_t bytes = (size_t)P.n * P.eb;
@@ -95,6 +102,11 @@ int upload(perm_plan* pl) {
     }
     e = perm::prepare_kernels(P);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
+    if (P.fused3) {
+        e = cudaMalloc(&pl->d_sync, 4 * sizeof(unsigned long long));
+        if (e == cudaSuccess) e = cudaMemset(pl->d_sync, 0, 4 * sizeof(unsigned long long));
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc sync");
+    }
     for (int i = 0; i < 8; ++i) {
         e = cudaEventCreate(&pl->ev[i]);
         if (e != cudaSuccess) return cuda_fail(e, "cudaEventCreate");
@@ -180,7 +192,7 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes == 1 ? 0 : 2 * P.n * P.eb);
     out->elem_bytes = P.eb;
     out->passes = P.passes;
-    out->kernels_per_apply = P.passes;
+    out->kernels_per_apply = P.fused3 ? 1 : P.passes;
     for (int f = 0; f < 3; ++f) {
         out->entry_bits[f] = P.ph[f].E;
         out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
@@ -196,7 +208,8 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
     if (!plan) return fail(PERM_EINVAL, "null plan");
     const HostPlan& P = plan->host;
     std::string s = "{\"n\":" + std::to_string(P.n) + ",\"rows\":" + std::to_string(P.r) +
-                    ",\"cols\":" + std::to_string(P.c) + ",\"passes\":" + std::to_string(P.passes);
+                    ",\"cols\":" + std::to_string(P.c) + ",\"passes\":" + std::to_string(P.passes) +
+                    ",\"layout\":" + std::to_string(P.layout) + ",\"fused3\":" + std::to_string(P.fused3);
     if (P.passes == 1) {
         s += ",\"fused\":{\"threads\":" + std::to_string(P.fused_threads) + ",\"ept\":" +
              std::to_string(P.fused_ept) + ",\"Ls\":" + std::to_string(P.fused_Ls) + "}";
@@ -211,6 +224,8 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
                        std::to_string(m.strideP) + ",\"cta_stride\":" + std::to_string(m.cta_stride) + "}";
             };
             s += std::string(f ? "," : "") + "{\"phase\":" + std::to_string(rp.phase) +
+                 ",\"tma\":" + std::to_string(rp.tma) + ",\"stages\":" + std::to_string(rp.stages) +
+                 ",\"grid\":" + std::to_string(rp.grid) +
                  ",\"L\":" + std::to_string(P.ph[rp.phase].L) + ",\"E\":" +
                  std::to_string(P.ph[rp.phase].E) + ",\"h\":" + std::to_string(rp.h) +
                  ",\"ctas\":" + std::to_string(rp.ctas) + ",\"threads\":" +
@@ -259,6 +274,41 @@ int perm_plan_set_profiling(perm_plan* plan, int enable) {
     return PERM_OK;
 }
 
+int perm_plan_set_tracing(perm_plan* plan, int enable) {
+    if (!plan) return fail(PERM_EINVAL, "null plan");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "host-only plan");
+    if (!enable) {
+        cudaFree(plan->d_trace);
+        plan->d_trace = nullptr;
+        return PERM_OK;
+    }
+    if (plan->d_trace) return PERM_OK;
+    int64_t mx = 1;
+    for (int f = 0; f < 3; ++f) {
+        const perm::RowPass& rp = plan->host.rp[f];
+        mx = std::max<int64_t>(mx, rp.tma ? rp.grid : rp.ctas);
+    }
+    mx = std::max<int64_t>(mx, plan->host.fused3_grid);
+    plan->trace_stride = mx;
+    cudaError_t e = cudaMalloc(&plan->d_trace, (size_t)(3 * mx * 16) * sizeof(unsigned long long));
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc trace");
+    e = cudaMemset(plan->d_trace, 0, (size_t)(3 * mx * 16) * sizeof(unsigned long long));
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMemset trace");
+    return PERM_OK;
+}
+
+int64_t perm_plan_trace(const perm_plan* plan, uint64_t* out, int64_t max_entries) {
+    if (!plan) return fail(PERM_EINVAL, "null plan");
+    if (!plan->d_trace) return 0;
+    const int64_t n = 3 * plan->trace_stride * 16;
+    if (out && max_entries > 0) {
+        cudaError_t e = cudaMemcpy(out, plan->d_trace, (size_t)std::min(n, max_entries) * 8,
+                                   cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy trace");
+    }
+    return n;
+}
+
 int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k) {
     if (!plan || !ms) return fail(PERM_EINVAL, "null argument");
     if (!plan->on_device) return fail(PERM_ENODEVICE, "host-only plan");
@@ -292,6 +342,9 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
     auto mark = [&]() {
         if (prof) cudaEventRecord(plan->ev[ev++], s);
     };
+    auto tr = [&](int f) -> unsigned long long* {
+        return plan->d_trace ? plan->d_trace + (int64_t)f * plan->trace_stride * 16 : nullptr;
+    };
     cudaError_t e = cudaSuccess;
     int k = 0;   // index of the kernel being launched (for the error message)
     mark();
@@ -299,22 +352,27 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
         e = perm::launch_fused(P, sc, in, out, s);
         mark();
+    } else if (P.fused3) {
+        const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
+        e = perm::launch_fused3(P, sc, in, plan->d_scratch[0], plan->d_scratch[1], out, plan->d_sync,
+                                s, tr(0));
+        mark();
     } else if (P.passes == 3) {
         uint32_t* x1 = plan->d_scratch[0];
         uint32_t* x2 = plan->d_scratch[1];
-        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false);
+        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false, tr(0));
         mark();
-        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x1, x2, s, !prof); mark(); }
-        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x1, x2, s, !prof, tr(1)); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof, tr(2)); mark(); }
     } else {
         uint32_t* x1 = plan->d_scratch[0];
         uint32_t* x2 = plan->d_scratch[1];
-        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false);
+        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false, tr(0));
         mark();
         if (e == cudaSuccess) { ++k; e = perm::launch_transpose(x1, x2, P.r, P.c, s, !prof); mark(); }
-        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x2, x1, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x2, x1, s, !prof, tr(1)); mark(); }
         if (e == cudaSuccess) { ++k; e = perm::launch_transpose(x1, x2, P.c, P.r, s, !prof); mark(); }
-        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof, tr(2)); mark(); }
     }
     if (e != cudaSuccess) {
         if (prof) plan->last_kernels = 0;

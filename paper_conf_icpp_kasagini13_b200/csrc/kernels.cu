@@ -43,6 +43,52 @@ __device__ __forceinline__ void prefetch_l2(const void* p) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+// TMA 1-D bulk copy global -> shared, completion counted on an mbarrier
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+// TMA 1-D bulk copy shared -> global (bulk group)
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+                 "r"(smem_u32(src)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
 // streaming 128-bit load of data that is not written by this kernel
 __device__ __forceinline__ uint4 ld_nc_v4(const uint32_t* p) {
     uint4 r;
@@ -71,56 +117,70 @@ __device__ __forceinline__ uint32_t decode_entry(uint32_t word, int w0, int off,
 // (0 <= q < h*L/32) of this CTA is line q >> (logL-5), round q & (L/32 - 1);
 // warp w handles q = w + W*m for m < EPT. addr(l, pos) maps (line, position)
 // to a shared-memory word: ROWS -> l*Ls + pos, COLS -> pos*Ls + l.
-template <int EPT, bool COLS>
+template <bool SMEM>
+__device__ __forceinline__ uint2 sched_load64(const uint2* p) {
+    if constexpr (SMEM) return *p;
+    else return __ldg(p);
+}
+
+// In-place permutation of the lines resident in shared memory. Warp-round q
+// (0 <= q < h*L/32) of this CTA is line q >> (logL-5), round q & (L/32 - 1);
+// warp w handles q = w + W*m for m < EPT. addr(l, pos) maps (line, position)
+// to a shared-memory word: ROWS -> l*Ls + pos, COLS -> pos*Ls + l.
+// Schedule in the W64 format (plan.hpp): lane x reads 64-bit word x/epw of the
+// round and shifts by E*(x % epw): one load, no shuffles. The destination
+// addresses decoded in the read hop stay in registers (two 16-bit addresses
+// per register) for the write hop, so the schedule is read once.
+template <int EPT, bool COLS, bool SCHED_SMEM = false>
 __device__ __forceinline__ void permute_lines(uint32_t* sm, const uint32_t* __restrict__ sched,
-                                              int logL, int E, int Ls) {
-    const int tid = threadIdx.x, lane = tid & 31, W = blockDim.x >> 5;
+                                              int logL, int E, int epw, int w64, int Ls) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, W = blockDim.x >> 5;
     const int logR = logL - 5;                      // log2(rounds per line)
-    const int bit0 = E * lane, w0 = bit0 >> 5, off = bit0 & 31;
+    const int wsel = lane / epw;
+    const int sh = E * (lane - wsel * epw);
     const uint32_t mask = (1u << E) - 1u;
     const uint32_t tmask = (1u << logL) - 1u;
-    const bool has_word = lane < E;
-    const int WE = W * E;
-    constexpr int CH = EPT < 8 ? EPT : 8;
+    const uint2* sp = reinterpret_cast<const uint2*>(sched) + warp * w64 + wsel;
+    const int step = W * w64;
+    // Up to 32 elements per thread the decoded destinations stay in registers
+    // (two 16-bit addresses per register); beyond that they are re-decoded in
+    // the write hop to stay within 128 registers.
+    constexpr bool KEEP = EPT <= 32;
     uint32_t v[EPT];
+    uint32_t ta[KEEP ? (EPT + 1) / 2 : 1];
     // read hop: v[m] = line[32*sigma + lane]   (bank = lane + const: conflict-free)
-    {
-        const int warp = tid >> 5;
-        const uint32_t* sp = sched + warp * E + lane;
 #pragma unroll
-        for (int c0 = 0; c0 < EPT; c0 += CH) {
-            uint32_t sw[CH];
-#pragma unroll
-            for (int u = 0; u < CH; ++u) sw[u] = has_word ? __ldg(sp + (c0 + u) * WE) : 0u;
-#pragma unroll
-            for (int u = 0; u < CH; ++u) {
-                const int l = (warp + W * (c0 + u)) >> logR;
-                const uint32_t e = decode_entry(sw[u], w0, off, mask);
-                const int s = (int)((e >> logL) << 5) + lane;
-                v[c0 + u] = COLS ? sm[s * Ls + l] : sm[l * Ls + s];
-            }
+    for (int m = 0; m < EPT; ++m) {
+        const uint2 wd = sched_load64<SCHED_SMEM>(sp + m * step);
+        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
+        const uint32_t e = (uint32_t)(w >> sh) & mask;
+        const int l = (warp + W * m) >> logR;
+        const int s = (int)((e >> logL) << 5) + lane;
+        v[m] = COLS ? sm[s * Ls + l] : sm[l * Ls + s];
+        if constexpr (KEEP) {
+            const int t = (int)(e & tmask);
+            const uint32_t ad = COLS ? (uint32_t)(t * Ls + l) : (uint32_t)(l * Ls + t);
+            if (m & 1) ta[m >> 1] |= ad << 16;
+            else ta[m >> 1] = ad;
         }
     }
     __syncthreads();
-    // write hop: line[t] = v[m]   (the 32 t of a warp-round hit 32 distinct banks).
-    // The warp index is re-read through a shuffle so the compiler recomputes the
-    // per-round addresses instead of keeping EPT of them live across the barrier.
-    {
-        const int warp = __shfl_sync(kFull, tid >> 5, 0);
-        const uint32_t* sp = sched + warp * E + lane;
+    // write hop: line[t] = v[m]   (the 32 t of a warp-round hit 32 distinct banks)
+    if constexpr (KEEP) {
 #pragma unroll
-        for (int c0 = 0; c0 < EPT; c0 += CH) {
-            uint32_t sw[CH];
+        for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
+    } else {
+        const int warp2 = __shfl_sync(kFull, warp, 0);   // not CSE-able: re-derive addresses
+        const uint2* sp2 = reinterpret_cast<const uint2*>(sched) + warp2 * w64 + wsel;
 #pragma unroll
-            for (int u = 0; u < CH; ++u) sw[u] = has_word ? __ldg(sp + (c0 + u) * WE) : 0u;
-#pragma unroll
-            for (int u = 0; u < CH; ++u) {
-                const int l = (warp + W * (c0 + u)) >> logR;
-                const uint32_t e = decode_entry(sw[u], w0, off, mask);
-                const int t = (int)(e & tmask);
-                if (COLS) sm[t * Ls + l] = v[c0 + u];
-                else      sm[l * Ls + t] = v[c0 + u];
-            }
+        for (int m = 0; m < EPT; ++m) {
+            const uint2 wd = sched_load64<SCHED_SMEM>(sp2 + m * step);
+            const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
+            const uint32_t e = (uint32_t)(w >> sh) & mask;
+            const int l = (warp2 + W * m) >> logR;
+            const int t = (int)(e & tmask);
+            if (COLS) sm[t * Ls + l] = v[m];
+            else      sm[l * Ls + t] = v[m];
         }
     }
     __syncthreads();
@@ -132,7 +192,7 @@ struct FusedArgs {
     const uint32_t* in;
     uint32_t* out;
     const uint32_t* sched[3];
-    int logr, logc, Ls, E[3];
+    int logr, logc, Ls, E[3], epw[3], w64[3];
 };
 
 // PAPER.md Thm 9: row-wise, column-wise, row-wise — all inside one CTA. The
@@ -148,9 +208,9 @@ __global__ void __launch_bounds__(512, 1) fused_kernel(const FusedArgs a) {
     const int cmask = (1 << a.logc) - 1;
     for (int e = tid; e < n; e += T) sm[(e >> a.logc) * a.Ls + (e & cmask)] = __ldg(a.in + e);
     __syncthreads();
-    permute_lines<EPT, false>(sm, a.sched[0], a.logc, a.E[0], a.Ls);   // Step 1: rows
-    permute_lines<EPT, true>(sm, a.sched[1], a.logr, a.E[1], a.Ls);    // Step 2: columns
-    permute_lines<EPT, false>(sm, a.sched[2], a.logc, a.E[2], a.Ls);   // Step 3: rows
+    permute_lines<EPT, false>(sm, a.sched[0], a.logc, a.E[0], a.epw[0], a.w64[0], a.Ls);  // Step 1: rows
+    permute_lines<EPT, true>(sm, a.sched[1], a.logr, a.E[1], a.epw[1], a.w64[1], a.Ls);   // Step 2: columns
+    permute_lines<EPT, false>(sm, a.sched[2], a.logc, a.E[2], a.epw[2], a.w64[2], a.Ls);  // Step 3: rows
     for (int e = tid; e < n; e += T) a.out[e] = sm[(e >> a.logc) * a.Ls + (e & cmask)];
 }
 
@@ -169,10 +229,21 @@ struct RowArgs {
     const uint32_t* in;
     uint32_t* out;
     const uint32_t* sched;     // this pass's packed phase
-    int logL, logh, Ls, E;
+    int logL, logh, Ls, E, epw, w64;
     long long sched_words_per_cta;
     Io i, o;
+    unsigned long long* trace;   // optional: 16 %globaltimer stamps per CTA (tracing)
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+// thread 0 of a CTA records stamp `slot` when tracing is enabled
+__device__ __forceinline__ void stamp(unsigned long long* tr, int slot) {
+    if (tr != nullptr && threadIdx.x == 0) tr[blockIdx.x * 16 + slot] = gtimer();
+}
 
 // Element (line l, position pos) of this CTA <-> global index (see plan.hpp IoMode).
 // Vector v covers elements f = 4v .. 4v+3 of the CTA's flattened I/O order:
@@ -258,7 +329,7 @@ __device__ __forceinline__ void tile_store(const RowArgs& a, const uint32_t* sm,
 // One row-wise permutation pass (Lemma 7): load h lines, permute each line in
 // place with its bank-conflict-free schedule, store them in the next pass's layout.
 template <int EPT>
-__global__ void __launch_bounds__(512, 1) row_pass_kernel(const RowArgs a) {
+__global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_kernel(const RowArgs a) {
     extern __shared__ __align__(16) uint32_t sm[];
     const long long cta = blockIdx.x;
     const uint32_t* sched = a.sched + cta * a.sched_words_per_cta;
@@ -267,12 +338,587 @@ __global__ void __launch_bounds__(512, 1) row_pass_kernel(const RowArgs a) {
     for (long long w = (long long)threadIdx.x * 32; w < a.sched_words_per_cta;
          w += (long long)blockDim.x * 32)
         prefetch_l2(sched + w);
+    stamp(a.trace, 0);
     pdl_wait();
+    stamp(a.trace, 1);
     tile_load<EPT>(a, sm, cta);
     __syncthreads();
+    stamp(a.trace, 2);
     pdl_launch_dependents();
-    permute_lines<EPT, false>(sm, sched, a.logL, a.E, a.Ls);
+    permute_lines<EPT, false>(sm, sched, a.logL, a.E, a.epw, a.w64, a.Ls);
+    stamp(a.trace, 3);
     tile_store<EPT>(a, sm, cta);
+    stamp(a.trace, 14);
+}
+
+// ------------------------------------------------------------------ row pass, TMA pipeline
+
+struct TmaArgs {
+    RowArgs r;                 // geometry + output layout (r.o); r.i unused (input = lines)
+    int ntiles, stages;
+    int data_words;            // h * Ls
+    int sched_words;           // h * (L/32) * E, a multiple of 4
+};
+
+// Persistent, pipelined row-wise permutation pass (Lemma 7) for contiguous input
+// lines. Each CTA walks tiles t = blockIdx.x + i*gridDim.x; a ring of `stages`
+// shared-memory slots holds [h lines | the tile's packed schedule]. One thread
+// arms the slot's mbarrier and issues TMA bulk copies (one per line, or one for
+// the whole tile when unpadded, plus one for the schedule); while tile i is
+// permuted and stored, tiles i+1 .. i+stages-1 are in flight. The schedule
+// copy is issued before griddepcontrol.wait: it does not depend on the
+// previous pass. Output: CROSS gather (column chunks of h elements, 128-bit
+// stores) or, for row-major output, a TMA bulk store.
+template <int EPT, bool OUT_CROSS>
+__global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(const TmaArgs a) {
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x;
+    const int L = 1 << a.r.logL, h = 1 << a.r.logh;
+    const int stage_words = a.data_words + a.sched_words;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + a.stages * stage_words);
+    const int G = gridDim.x;
+    const uint32_t line_bytes = (uint32_t)L * 4u;
+    const bool dense = a.r.Ls == L;
+    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (uint32_t)a.sched_words * 4u;
+
+    auto issue_sched = [&](int s, long long t) {
+        bulk_g2s(smem + s * stage_words + a.data_words, a.r.sched + t * a.sched_words,
+                 (uint32_t)a.sched_words * 4u, &bars[s]);
+    };
+    auto issue_data = [&](int s, long long t) {
+        const uint32_t* src = a.r.in + t * h * (long long)L;
+        uint32_t* dst = smem + s * stage_words;
+        if (dense) {
+            bulk_g2s(dst, src, (uint32_t)h * line_bytes, &bars[s]);
+        } else {
+            for (int l = 0; l < h; ++l) bulk_g2s(dst + l * a.r.Ls, src + (long long)l * L, line_bytes, &bars[s]);
+        }
+    };
+
+    unsigned long long* tr = a.r.trace;
+    stamp(tr, 0);
+    if (tid == 0) {
+        for (int s = 0; s < a.stages; ++s) mbar_init(&bars[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
+        for (int s = 0; s < a.stages; ++s) {
+            const long long t = blockIdx.x + (long long)s * G;
+            if (t < a.ntiles) {
+                mbar_arrive_expect_tx(&bars[s], tile_bytes);
+                issue_sched(s, t);
+            }
+        }
+    }
+    pdl_wait();   // the previous pass's output is complete and visible from here on
+    stamp(tr, 1);
+    if (tid == 0) {
+        for (int s = 0; s < a.stages; ++s) {
+            const long long t = blockIdx.x + (long long)s * G;
+            if (t < a.ntiles) issue_data(s, t);
+        }
+    }
+    pdl_launch_dependents();
+    for (int i = 0;; ++i) {
+        const long long t = blockIdx.x + (long long)i * G;
+        if (t >= a.ntiles) break;
+        const int s = i % a.stages;
+        mbar_wait(&bars[s], (uint32_t)(i / a.stages) & 1u);
+        if (i < 4) stamp(tr, 2 + 3 * i);
+        uint32_t* buf = smem + s * stage_words;
+        permute_lines<EPT, false, true>(buf, buf + a.data_words, a.r.logL, a.r.E, a.r.epw, a.r.w64,
+                                        a.r.Ls);
+        if (i < 4) stamp(tr, 3 + 3 * i);
+        if constexpr (OUT_CROSS) {
+            tile_store<EPT>(a.r, buf, t);
+        } else {
+            if (tid == 0) {
+                fence_proxy_async();     // generic-proxy smem writes -> async-proxy reads
+                uint32_t* dst = a.r.out + t * h * (long long)L;
+                if (dense) {
+                    bulk_s2g(dst, buf, (uint32_t)h * line_bytes);
+                } else {
+                    for (int l = 0; l < h; ++l) bulk_s2g(dst + (long long)l * L, buf + l * a.r.Ls, line_bytes);
+                }
+                bulk_commit();
+            }
+        }
+        __syncthreads();                 // every thread is done with slot s
+        if (i < 4) stamp(tr, 4 + 3 * i);
+        if (tid == 0) {
+            const long long tn = t + (long long)a.stages * G;
+            if (tn < a.ntiles) {
+                if constexpr (!OUT_CROSS) bulk_wait_read0();   // the bulk store has read slot s
+                fence_proxy_async();
+                mbar_arrive_expect_tx(&bars[s], tile_bytes);
+                issue_sched(s, tn);
+                issue_data(s, tn);
+            }
+        }
+    }
+    if constexpr (!OUT_CROSS) {
+        if (tid == 0) bulk_wait0();
+    }
+    stamp(tr, 14);
+}
+
+// ------------------------------------------------------------------ row pass, warp-specialized
+
+__device__ __forceinline__ void named_bar(int id, int count) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void stamp_if(unsigned long long* tr, bool who, int slot) {
+    if (tr != nullptr && who) tr[blockIdx.x * 16 + slot] = gtimer();
+}
+
+constexpr int kWsPerm = 512;    // permuter threads (16 warps)
+constexpr int kWsStore = 256;   // storer threads (8 warps), CROSS output only
+
+struct WsArgs {
+    RowArgs r;                  // geometry, output layout (r.o), trace
+    int ntiles, stages;
+    int data_words;             // h * Ls
+    int sched_words;            // h * (L/32) * w64 * 2
+};
+
+// In-place permute of one tile by the permuter warps: permuter warp pw owns the
+// EPT consecutive warp-rounds q = pw*EPT + m (one line when EPT <= L/32), so the
+// line base is computed once; schedule entries are decoded once (W64 format)
+// and the destination addresses wait in registers across the named barrier.
+template <int EPT>
+__device__ __forceinline__ void permute_tile_ws(uint32_t* sm, const uint32_t* sched, int logL,
+                                                int E, int epw, int w64, int Ls, int pw, int lane) {
+    const int logR = logL - 5;
+    const int wsel = lane / epw;
+    const int sh = E * (lane - wsel * epw);
+    const uint32_t mask = (1u << E) - 1u;
+    const uint32_t tmask = (1u << logL) - 1u;
+    const int q0 = pw * EPT;
+    const uint2* sp = reinterpret_cast<const uint2*>(sched) + q0 * w64 + wsel;
+    constexpr bool KEEP = EPT <= 32;
+    uint32_t v[EPT];
+    uint32_t ta[KEEP ? (EPT + 1) / 2 : 1];
+    const bool one_line = EPT <= (1 << logR);
+    const int lb0 = (q0 >> logR) * Ls + lane;
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) {
+        const uint2 wd = sp[m * w64];
+        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
+        const uint32_t e = (uint32_t)(w >> sh) & mask;
+        const int lb = one_line ? lb0 : ((q0 + m) >> logR) * Ls + lane;
+        v[m] = sm[lb + (int)((e >> logL) << 5)];
+        if constexpr (KEEP) {
+            const uint32_t ad = (uint32_t)(lb - lane) + (e & tmask);
+            if (m & 1) ta[m >> 1] |= ad << 16;
+            else ta[m >> 1] = ad;
+        }
+    }
+    named_bar(1, kWsPerm);
+    if constexpr (KEEP) {
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
+    } else {
+        const int q1 = __shfl_sync(kFull, q0, 0);
+        const uint2* sp2 = reinterpret_cast<const uint2*>(sched) + q1 * w64 + wsel;
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) {
+            const uint2 wd = sp2[m * w64];
+            const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
+            const uint32_t e = (uint32_t)(w >> sh) & mask;
+            sm[((q1 + m) >> logR) * Ls + (int)(e & tmask)] = v[m];
+        }
+    }
+}
+
+// Persistent warp-specialized row-wise permutation pass (Lemma 7) over
+// contiguous input lines. Ring of `stages` shared-memory slots [h lines | the
+// tile's packed schedule]; three mbarriers per slot:
+//   full[s]  TMA bytes landed          (producer thread arms, TMA completes)
+//   perm[s]  tile permuted in place    (512 permuter threads arrive)
+//   empty[s] slot read by the storers  (256 storer threads arrive; CROSS only)
+// warp 0 lane 0: TMA producer (and, for row-major output, the TMA bulk storer);
+// warps 1..16: permuters; warps 17..24: storers (CROSS output gather + 128-bit
+// stores). Loading tile i+1, permuting tile i and storing tile i-1 overlap.
+template <int EPT, bool OUT_CROSS>
+__global__ void __launch_bounds__(OUT_CROSS ? 32 + kWsPerm + kWsStore : 32 + kWsPerm, 1)
+    row_pass_ws_kernel(const WsArgs a) {
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int L = 1 << a.r.logL, h = 1 << a.r.logh;
+    const int NS = a.stages;
+    const int stage_words = a.data_words + a.sched_words;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * stage_words);
+    uint64_t* permd = full + NS;
+    uint64_t* empty = permd + NS;
+    const int G = gridDim.x;
+    const uint32_t line_bytes = (uint32_t)L * 4u;
+    const bool dense = a.r.Ls == L;
+    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (uint32_t)a.sched_words * 4u;
+    unsigned long long* tr = a.r.trace;
+    stamp(tr, 0);
+    if (tid == 0) {
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&permd[s], kWsPerm);
+            mbar_init(&empty[s], OUT_CROSS ? kWsStore : 1);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    auto issue = [&](int s, long long t, bool sched_part, bool data_part) {
+        uint32_t* dst = smem + s * stage_words;
+        if (sched_part)
+            bulk_g2s(dst + a.data_words, a.r.sched + t * a.sched_words, (uint32_t)a.sched_words * 4u,
+                     &full[s]);
+        if (data_part) {
+            const uint32_t* src = a.r.in + t * h * (long long)L;
+            if (dense) {
+                bulk_g2s(dst, src, (uint32_t)h * line_bytes, &full[s]);
+            } else {
+                for (int l = 0; l < h; ++l)
+                    bulk_g2s(dst + l * a.r.Ls, src + (long long)l * L, line_bytes, &full[s]);
+            }
+        }
+    };
+
+    if (warp == 0) {
+        // ---------------- producer (and bulk storer for row-major output)
+        if (lane == 0) {
+            for (int s = 0; s < NS; ++s) {
+                const long long t = blockIdx.x + (long long)s * G;
+                if (t < a.ntiles) {
+                    mbar_arrive_expect_tx(&full[s], tile_bytes);
+                    issue(s, t, true, false);     // schedule does not depend on the previous pass
+                }
+            }
+            pdl_wait();
+            stamp(tr, 1);
+            for (int s = 0; s < NS; ++s) {
+                const long long t = blockIdx.x + (long long)s * G;
+                if (t < a.ntiles) issue(s, t, false, true);
+            }
+            pdl_launch_dependents();
+            if constexpr (OUT_CROSS) {
+                for (int i = NS;; ++i) {
+                    const long long t = blockIdx.x + (long long)i * G;
+                    if (t >= a.ntiles) break;
+                    const int s = i % NS;
+                    mbar_wait(&empty[s], (uint32_t)(i / NS - 1) & 1u);
+                    fence_proxy_async();
+                    mbar_arrive_expect_tx(&full[s], tile_bytes);
+                    issue(s, t, true, true);
+                }
+            } else {
+                for (int i = 0;; ++i) {
+                    const long long t = blockIdx.x + (long long)i * G;
+                    if (t >= a.ntiles) break;
+                    const int s = i % NS;
+                    mbar_wait(&permd[s], (uint32_t)(i / NS) & 1u);
+                    fence_proxy_async();          // permuters' smem writes -> async-proxy reads
+                    const uint32_t* buf = smem + s * stage_words;
+                    uint32_t* dst = a.r.out + t * h * (long long)L;
+                    if (dense) {
+                        bulk_s2g(dst, buf, (uint32_t)h * line_bytes);
+                    } else {
+                        for (int l = 0; l < h; ++l)
+                            bulk_s2g(dst + (long long)l * L, buf + l * a.r.Ls, line_bytes);
+                    }
+                    bulk_commit();
+                    if (i < 4) stamp_if(tr, true, 4 + 3 * i);
+                    const long long tn = t + (long long)NS * G;
+                    if (tn < a.ntiles) {
+                        bulk_wait_read0();
+                        fence_proxy_async();
+                        mbar_arrive_expect_tx(&full[s], tile_bytes);
+                        issue(s, tn, true, true);
+                    }
+                }
+                bulk_wait0();
+            }
+            stamp(tr, 14);
+        }
+    } else if (warp <= kWsPerm / 32) {
+        // ---------------- permuters
+        const int pw = warp - 1;
+        const bool lead = tid == 32;
+        for (int i = 0;; ++i) {
+            const long long t = blockIdx.x + (long long)i * G;
+            if (t >= a.ntiles) break;
+            const int s = i % NS;
+            mbar_wait(&full[s], (uint32_t)(i / NS) & 1u);
+            if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
+            uint32_t* buf = smem + s * stage_words;
+            permute_tile_ws<EPT>(buf, buf + a.data_words, a.r.logL, a.r.E, a.r.epw, a.r.w64, a.r.Ls,
+                                 pw, lane);
+            mbar_arrive(&permd[s]);
+            if (i < 4) stamp_if(tr, lead, 3 + 3 * i);
+        }
+    } else if constexpr (OUT_CROSS) {
+        // ---------------- storers: gather column chunks, 128-bit stores
+        pdl_wait();
+        const int sj = tid - 32 - kWsPerm;
+        const bool lead = sj == 0;
+        const int logh = a.r.logh;
+        const Io& m = a.r.o;
+        const int logBPh = m.logBP + logh;
+        constexpr int NV = (kWsPerm * EPT) / (4 * kWsStore);   // vectors per storer thread
+        for (int i = 0;; ++i) {
+            const long long t = blockIdx.x + (long long)i * G;
+            if (t >= a.ntiles) break;
+            const int s = i % NS;
+            mbar_wait(&permd[s], (uint32_t)(i / NS) & 1u);
+            const uint32_t* buf = smem + s * stage_words;
+            uint32_t* base = a.r.out + t * m.cta_stride;
+            constexpr int CH = NV < 8 ? NV : 8;
+#pragma unroll
+            for (int c0 = 0; c0 < NV; c0 += CH) {
+                uint4 vv[CH];
+#pragma unroll
+                for (int u = 0; u < CH; ++u) {
+                    const int f = 4 * (sj + kWsStore * (c0 + u));
+                    const int pos = f >> logh, l = f & ((1 << logh) - 1);
+                    const uint32_t* src = buf + l * a.r.Ls + pos;
+                    vv[u].x = src[0];
+                    vv[u].y = src[a.r.Ls];
+                    vv[u].z = src[2 * a.r.Ls];
+                    vv[u].w = src[3 * a.r.Ls];
+                }
+                if (c0 + CH >= NV) mbar_arrive(&empty[s]);   // slot may be refilled
+#pragma unroll
+                for (int u = 0; u < CH; ++u) {
+                    const int f = 4 * (sj + kWsStore * (c0 + u));
+                    const int pos = f >> logh;
+                    st_v4(base + (long long)(pos >> m.logBP) * m.strideP + (f & ((1 << logBPh) - 1)),
+                          vv[u]);
+                }
+            }
+            if (i < 4) stamp_if(tr, lead, 4 + 3 * i);
+        }
+        stamp_if(tr, lead, 15);
+    }
+}
+
+// ------------------------------------------------------------------ fused 3-pass persistent kernel
+
+__device__ __forceinline__ void prefetch_l2_bulk(const void* p, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() {
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void red_release_gpu_add(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+struct PassCfg {
+    const uint32_t* in;
+    uint32_t* out;
+    const uint32_t* sched;     // this phase's packed schedule
+    int ntiles;                // lines / h
+    int cross;                 // 1: out[t*h + pos*strideP + l] (column chunks); 0: row-major lines
+    long long strideP;
+};
+
+struct Fused3Args {
+    PassCfg p[3];
+    int logL, logh, Ls, E, epw, w64;
+    int stages, data_words, sched_words;
+    unsigned long long* sync;  // [0], [1]: arrivals at the barriers after pass 0 / pass 1,
+                               // [2]: exits (the last CTA out resets all three)
+    unsigned long long* trace;
+};
+
+// The whole scheduled permutation (Thm 9: row-wise, column-wise, row-wise) in
+// ONE persistent launch, for square views (every phase has lines of length L).
+// Same warp roles and slot ring as row_pass_ws_kernel, continued across the
+// three passes (global tile sequence j). Between pass k and k+1 every element
+// of the intermediate must be written before any is read, so: the storers of a
+// CTA fence and publish their last pass-k store (red.release.gpu on sync[k]);
+// the producer may already arm a slot and TMA the NEXT pass's schedule, but
+// issues the next pass's data copies only after sync[k] reaches the grid size.
+// All CTAs are co-resident (grid = one CTA per SM). The last CTA to exit
+// resets the counters, so the kernel is replayable (e.g. inside a CUDA graph).
+template <int EPT>
+__global__ void __launch_bounds__(32 + kWsPerm + kWsStore, 1) fused3_ws_kernel(const Fused3Args a) {
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int L = 1 << a.logL, h = 1 << a.logh;
+    const int NS = a.stages;
+    const int stage_words = a.data_words + a.sched_words;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * stage_words);
+    uint64_t* permd = full + NS;
+    uint64_t* empty = permd + NS;
+    const int G = gridDim.x;
+    const uint32_t line_bytes = (uint32_t)L * 4u;
+    const bool dense = a.Ls == L;
+    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (uint32_t)a.sched_words * 4u;
+    unsigned long long* tr = a.trace;
+    stamp(tr, 0);
+    if (tid == 0) {
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&permd[s], kWsPerm);
+            mbar_init(&empty[s], kWsStore);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    // tiles of pass k owned by this CTA: t = blockIdx.x + i*G < ntiles_k
+    auto my_tiles = [&](int k) -> int {
+        const int n = a.p[k].ntiles - (int)blockIdx.x;
+        return n > 0 ? (n + G - 1) / G : 0;
+    };
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---------------- producer
+            int j = 0;
+            for (int k = 0; k < 3; ++k) {
+                const PassCfg& pc = a.p[k];
+                const int nt = my_tiles(k);
+                bool data_ok = (k == 0);
+                for (int i = 0; i < nt; ++i, ++j) {
+                    const long long t = blockIdx.x + (long long)i * G;
+                    const int s = j % NS;
+                    if (j >= NS) mbar_wait(&empty[s], (uint32_t)(j / NS - 1) & 1u);
+                    fence_proxy_async();
+                    mbar_arrive_expect_tx(&full[s], tile_bytes);
+                    uint32_t* dst = smem + s * stage_words;
+                    bulk_g2s(dst + a.data_words, pc.sched + t * a.sched_words,
+                             (uint32_t)a.sched_words * 4u, &full[s]);
+                    if (!data_ok) {
+                        // grid barrier: every CTA has published its pass k-1 stores. One
+                        // counter per barrier: a CTA that runs ahead (e.g. owns no tiles)
+                        // must not count toward an earlier barrier.
+                        while (ld_acquire_gpu(&a.sync[k - 1]) < (unsigned long long)G) __nanosleep(64);
+                        fence_proxy_async_global();
+                        data_ok = true;
+                        stamp(tr, 1 + 4 * k);
+                    }
+                    const uint32_t* src = pc.in + t * h * (long long)L;
+                    if (dense) {
+                        bulk_g2s(dst, src, (uint32_t)h * line_bytes, &full[s]);
+                    } else {
+                        for (int l = 0; l < h; ++l)
+                            bulk_g2s(dst + l * a.Ls, src + (long long)l * L, line_bytes, &full[s]);
+                    }
+                }
+                if (k == 0) {
+                    // pass 0's loads are out: the later passes' schedules do not depend on
+                    // the data, so stream them into L2 while pass 0 permutes and stores
+                    for (int k2 = 1; k2 < 3; ++k2)
+                        for (int i = 0; i < my_tiles(k2); ++i) {
+                            const long long t = blockIdx.x + (long long)i * G;
+                            prefetch_l2_bulk(a.p[k2].sched + t * a.sched_words,
+                                             (uint32_t)a.sched_words * 4u);
+                        }
+                }
+            }
+        }
+    } else if (warp <= kWsPerm / 32) {
+        // ---------------- permuters
+        const int pw = warp - 1;
+        const bool lead = tid == 32;
+        int j = 0;
+        for (int k = 0; k < 3; ++k) {
+            const int nt = my_tiles(k);
+            for (int i = 0; i < nt; ++i, ++j) {
+                const int s = j % NS;
+                mbar_wait(&full[s], (uint32_t)(j / NS) & 1u);
+                if (i == 0) stamp_if(tr, lead, 2 + 4 * k);
+                uint32_t* buf = smem + s * stage_words;
+                permute_tile_ws<EPT>(buf, buf + a.data_words, a.logL, a.E, a.epw, a.w64, a.Ls, pw, lane);
+                mbar_arrive(&permd[s]);
+            }
+            stamp_if(tr, lead, 3 + 4 * k);
+        }
+    } else {
+        // ---------------- storers
+        const int sj = tid - 32 - kWsPerm;
+        const bool lead = sj == 0;
+        const int logh = a.logh;
+        constexpr int NV = (kWsPerm * EPT) / (4 * kWsStore);
+        constexpr int CH = NV < 8 ? NV : 8;
+        int j = 0;
+        for (int k = 0; k < 3; ++k) {
+            const PassCfg& pc = a.p[k];
+            const int nt = my_tiles(k);
+            for (int i = 0; i < nt; ++i, ++j) {
+                const long long t = blockIdx.x + (long long)i * G;
+                const int s = j % NS;
+                mbar_wait(&permd[s], (uint32_t)(j / NS) & 1u);
+                const uint32_t* buf = smem + s * stage_words;
+                if (pc.cross) {
+                    uint32_t* base = pc.out + t * h;
+#pragma unroll
+                    for (int c0 = 0; c0 < NV; c0 += CH) {
+                        uint4 vv[CH];
+#pragma unroll
+                        for (int u = 0; u < CH; ++u) {
+                            const int f = 4 * (sj + kWsStore * (c0 + u));
+                            const int pos = f >> logh, l = f & (h - 1);
+                            const uint32_t* src = buf + l * a.Ls + pos;
+                            vv[u].x = src[0];
+                            vv[u].y = src[a.Ls];
+                            vv[u].z = src[2 * a.Ls];
+                            vv[u].w = src[3 * a.Ls];
+                        }
+                        if (c0 + CH >= NV) mbar_arrive(&empty[s]);
+#pragma unroll
+                        for (int u = 0; u < CH; ++u) {
+                            const int f = 4 * (sj + kWsStore * (c0 + u));
+                            const int pos = f >> logh, l = f & (h - 1);
+                            st_v4(base + (long long)pos * pc.strideP + l, vv[u]);
+                        }
+                    }
+                } else {
+                    if (lead) {
+                        fence_proxy_async();
+                        uint32_t* dst = pc.out + t * h * (long long)L;
+                        if (dense) {
+                            bulk_s2g(dst, buf, (uint32_t)h * line_bytes);
+                        } else {
+                            for (int l = 0; l < h; ++l)
+                                bulk_s2g(dst + (long long)l * L, buf + l * a.Ls, line_bytes);
+                        }
+                        bulk_commit();
+                        bulk_wait_read0();
+                    }
+                    mbar_arrive(&empty[s]);
+                }
+            }
+            if (k < 2) {
+                // publish this CTA's pass-k stores to the grid
+                __threadfence();
+                named_bar(2, kWsStore);
+                if (lead) red_release_gpu_add(&a.sync[k], 1ull);
+            }
+            stamp_if(tr, lead, 4 + 4 * k);
+        }
+        if (lead) bulk_wait0();
+    }
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        const unsigned long long old = atomicAdd(&a.sync[2], 1ull);
+        if (old == (unsigned long long)G - 1) {     // last CTA out: every spin has finished
+            a.sync[0] = 0;
+            a.sync[1] = 0;
+            a.sync[2] = 0;
+            __threadfence();
+        }
+    }
+    stamp(tr, 15);
 }
 
 // ------------------------------------------------------------------ transpose
@@ -385,14 +1031,104 @@ Io make_io(const IoMode& m) {
     return o;
 }
 
+template <typename K>
+cudaError_t set_smem(K kernel, size_t bytes) {
+    cudaError_t e = cudaFuncSetAttribute((const void*)kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute((const void*)kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                 100);
+    return e;
+}
+
+size_t tma_smem(const HostPlan& P, int f) {
+    const RowPass& rp = P.rp[f];
+    const PhaseGeom& g = P.ph[rp.phase];
+    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (size_t)rp.h * (g.L / 32) * g.w64 * 8;
+    return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
+}
+
+template <int EPT>
+cudaError_t prep_ws(HostPlan& P, int f) {
+    RowPass& rp = P.rp[f];
+    const size_t smem = tma_smem(P, f);
+    cudaError_t e;
+    int nb = 0;
+    if (rp.out.cross) {
+        e = set_smem(row_pass_ws_kernel<EPT, true>, smem);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_ws_kernel<EPT, true>, rp.threads, smem);
+    } else {
+        e = set_smem(row_pass_ws_kernel<EPT, false>, smem);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_ws_kernel<EPT, false>, rp.threads, smem);
+    }
+    if (e != cudaSuccess) return e;
+    if (nb < 1) return cudaErrorInvalidConfiguration;
+    const long long cap = (long long)nb * sm_count();
+    rp.grid = rp.ctas < cap ? rp.ctas : cap;
+    return cudaSuccess;
+}
+
+template <int EPT>
+cudaError_t set_tma_smem(bool cross, size_t smem) {
+    return cross ? set_smem(row_pass_tma_kernel<EPT, true>, smem)
+                 : set_smem(row_pass_tma_kernel<EPT, false>, smem);
+}
+
+template <int EPT>
+cudaError_t grid_tma(HostPlan& P, int f) {
+    RowPass& rp = P.rp[f];
+    const size_t smem = tma_smem(P, f);
+    int nb = 0;
+    cudaError_t e = rp.out.cross
+        ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_tma_kernel<EPT, true>, rp.threads, smem)
+        : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_tma_kernel<EPT, false>, rp.threads, smem);
+    if (e != cudaSuccess) return e;
+    if (nb < 1) return cudaErrorInvalidConfiguration;
+    const long long cap = (long long)nb * sm_count();
+    rp.grid = rp.ctas < cap ? rp.ctas : cap;
+    return cudaSuccess;
+}
+
+size_t fused3_smem(const HostPlan& P) {
+    const RowPass& rp = P.rp[0];
+    const PhaseGeom& g = P.ph[0];
+    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (size_t)rp.h * (g.L / 32) * g.w64 * 8;
+    return rp.stages * stage + rp.stages * 8 * 3;
+}
+
+template <int EPT>
+cudaError_t prep_fused3(HostPlan& P) {
+    const size_t smem = fused3_smem(P);
+    cudaError_t e = set_smem(fused3_ws_kernel<EPT>, smem);
+    if (e != cudaSuccess) return e;
+    int nb = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fused3_ws_kernel<EPT>, 32 + kWsPerm + kWsStore, smem);
+    if (e != cudaSuccess) return e;
+    if (nb < 1) return cudaErrorInvalidConfiguration;
+    P.fused3_grid = sm_count();      // exactly one co-resident CTA per SM (grid barrier)
+    return cudaSuccess;
+}
+
 }  // namespace
 
-cudaError_t prepare_kernels(const HostPlan& P) {
+cudaError_t prepare_kernels(HostPlan& P) {
     cudaError_t e = cudaSuccess;
     auto set = [&](const void* k, size_t bytes) {
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     };
+    if (P.fused3) {
+        switch (P.rp[0].ept) {
+            case 8: return prep_fused3<8>(P);
+            case 16: return prep_fused3<16>(P);
+            case 32: return prep_fused3<32>(P);
+            default: return cudaErrorInvalidValue;
+        }
+    }
     if (P.passes == 1) {
         const size_t b = fused_smem(P);
         switch (P.fused_ept) {
@@ -400,18 +1136,52 @@ cudaError_t prepare_kernels(const HostPlan& P) {
             case 8: set((const void*)fused_kernel<8>, b); break;
             case 16: set((const void*)fused_kernel<16>, b); break;
             case 32: set((const void*)fused_kernel<32>, b); break;
-            case 64: set((const void*)fused_kernel<64>, b); break;
             default: return cudaErrorInvalidValue;
         }
         return e;
     }
     // one attribute per template instance: use the largest request among the passes
-    size_t need[7] = {0, 0, 0, 0, 0, 0, 0};   // index log2(ept)
+    size_t need[7] = {0, 0, 0, 0, 0, 0, 0};        // plain kernel, index log2(ept)
+    size_t need_t[2][7] = {{0}, {0}};              // TMA kernel [cross][log2(ept)]
     for (int f = 0; f < 3; ++f) {
         const int li = ilog2i(P.rp[f].ept);
         if (li < 2 || li > 6) return cudaErrorInvalidValue;
-        need[li] = need[li] > row_smem(P, f) ? need[li] : row_smem(P, f);
+        if (P.rp[f].tma == 2) {
+            switch (P.rp[f].ept) {
+                case 8: e = prep_ws<8>(P, f); break;
+                case 16: e = prep_ws<16>(P, f); break;
+                case 32: e = prep_ws<32>(P, f); break;
+                case 64: e = prep_ws<64>(P, f); break;
+                default: return cudaErrorInvalidValue;
+            }
+            if (e != cudaSuccess) return e;
+            continue;
+        }
+        if (P.rp[f].tma) {
+            size_t& nt = need_t[P.rp[f].out.cross ? 1 : 0][li];
+            nt = nt > tma_smem(P, f) ? nt : tma_smem(P, f);
+        } else {
+            need[li] = need[li] > row_smem(P, f) ? need[li] : row_smem(P, f);
+        }
     }
+    for (int cx = 0; cx < 2 && e == cudaSuccess; ++cx) {
+        if (need_t[cx][2]) e = set_tma_smem<4>(cx, need_t[cx][2]);
+        if (e == cudaSuccess && need_t[cx][3]) e = set_tma_smem<8>(cx, need_t[cx][3]);
+        if (e == cudaSuccess && need_t[cx][4]) e = set_tma_smem<16>(cx, need_t[cx][4]);
+        if (e == cudaSuccess && need_t[cx][5]) e = set_tma_smem<32>(cx, need_t[cx][5]);
+        if (e == cudaSuccess && need_t[cx][6]) e = set_tma_smem<64>(cx, need_t[cx][6]);
+    }
+    for (int f = 0; f < 3 && e == cudaSuccess; ++f) {
+        if (P.rp[f].tma != 1) continue;
+        switch (P.rp[f].ept) {
+            case 4: e = grid_tma<4>(P, f); break;
+            case 8: e = grid_tma<8>(P, f); break;
+            case 16: e = grid_tma<16>(P, f); break;
+            case 32: e = grid_tma<32>(P, f); break;
+            case 64: e = grid_tma<64>(P, f); break;
+        }
+    }
+    if (e != cudaSuccess) return e;
     if (need[2]) set((const void*)row_pass_kernel<4>, need[2]);
     if (need[3]) set((const void*)row_pass_kernel<8>, need[3]);
     if (need[4]) set((const void*)row_pass_kernel<16>, need[4]);
@@ -428,6 +1198,8 @@ cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], cons
     for (int f = 0; f < 3; ++f) {
         fa.sched[f] = sched[f];
         fa.E[f] = P.ph[f].E;
+        fa.epw[f] = P.ph[f].epw;
+        fa.w64[f] = P.ph[f].w64;
     }
     fa.logr = ilog2i(P.r);
     fa.logc = ilog2i(P.c);
@@ -439,16 +1211,16 @@ cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], cons
         case 8: return launch(fused_kernel<8>, grid, block, smem, s, false, fa);
         case 16: return launch(fused_kernel<16>, grid, block, smem, s, false, fa);
         case 32: return launch(fused_kernel<32>, grid, block, smem, s, false, fa);
-        case 64: return launch(fused_kernel<64>, grid, block, smem, s, false, fa);
     }
     return cudaErrorInvalidValue;
 }
 
 cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, const uint32_t* in,
-                            uint32_t* out, cudaStream_t s, bool pdl) {
+                            uint32_t* out, cudaStream_t s, bool pdl, unsigned long long* trace) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
     RowArgs ra{};
+    ra.trace = trace;
     ra.in = in;
     ra.out = out;
     ra.sched = sched;
@@ -456,10 +1228,60 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
     ra.logh = ilog2i(rp.h);
     ra.Ls = rp.Ls;
     ra.E = g.E;
-    ra.sched_words_per_cta = (long long)rp.h * (g.L / 32) * g.E;
+    ra.epw = g.epw;
+    ra.w64 = g.w64;
+    ra.sched_words_per_cta = (long long)rp.h * (g.L / 32) * g.w64 * 2;
     ra.i = make_io(rp.in);
     ra.o = make_io(rp.out);
-    const dim3 grid((unsigned)rp.ctas), block(rp.threads);
+    const dim3 block(rp.threads);
+    if (rp.tma == 2) {
+        WsArgs wa{};
+        wa.r = ra;
+        wa.ntiles = (int)rp.ctas;
+        wa.stages = rp.stages;
+        wa.data_words = rp.h * rp.Ls;
+        wa.sched_words = (int)ra.sched_words_per_cta;
+        const dim3 grid((unsigned)rp.grid);
+        const size_t smem = tma_smem(P, f);
+        const bool cx = rp.out.cross != 0;
+#define PERM_WS_CASE(E_)                                                                       \
+    case E_:                                                                                   \
+        return cx ? launch(row_pass_ws_kernel<E_, true>, grid, block, smem, s, pdl, wa)        \
+                  : launch(row_pass_ws_kernel<E_, false>, grid, block, smem, s, pdl, wa);
+        switch (rp.ept) {
+            PERM_WS_CASE(8)
+            PERM_WS_CASE(16)
+            PERM_WS_CASE(32)
+            PERM_WS_CASE(64)
+        }
+#undef PERM_WS_CASE
+        return cudaErrorInvalidValue;
+    }
+    if (rp.tma) {
+        TmaArgs ta{};
+        ta.r = ra;
+        ta.ntiles = (int)rp.ctas;
+        ta.stages = rp.stages;
+        ta.data_words = rp.h * rp.Ls;
+        ta.sched_words = (int)ra.sched_words_per_cta;
+        const dim3 grid((unsigned)rp.grid);
+        const size_t smem = tma_smem(P, f);
+        const bool cx = rp.out.cross != 0;
+#define PERM_TMA_CASE(E_)                                                                      \
+    case E_:                                                                                   \
+        return cx ? launch(row_pass_tma_kernel<E_, true>, grid, block, smem, s, pdl, ta)       \
+                  : launch(row_pass_tma_kernel<E_, false>, grid, block, smem, s, pdl, ta);
+        switch (rp.ept) {
+            PERM_TMA_CASE(4)
+            PERM_TMA_CASE(8)
+            PERM_TMA_CASE(16)
+            PERM_TMA_CASE(32)
+            PERM_TMA_CASE(64)
+        }
+#undef PERM_TMA_CASE
+        return cudaErrorInvalidValue;
+    }
+    const dim3 grid((unsigned)rp.ctas);
     const size_t smem = row_smem(P, f);
     switch (rp.ept) {
         case 4: return launch(row_pass_kernel<4>, grid, block, smem, s, pdl, ra);
@@ -467,6 +1289,44 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         case 16: return launch(row_pass_kernel<16>, grid, block, smem, s, pdl, ra);
         case 32: return launch(row_pass_kernel<32>, grid, block, smem, s, pdl, ra);
         case 64: return launch(row_pass_kernel<64>, grid, block, smem, s, pdl, ra);
+    }
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_fused3(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
+                          uint32_t* x1, uint32_t* x2, uint32_t* b, unsigned long long* sync,
+                          cudaStream_t s, unsigned long long* trace) {
+    Fused3Args fa{};
+    const uint32_t* ins[3] = {a, x1, x2};
+    uint32_t* outs[3] = {x1, x2, b};
+    for (int f = 0; f < 3; ++f) {
+        const RowPass& rp = P.rp[f];
+        fa.p[f].in = ins[f];
+        fa.p[f].out = outs[f];
+        fa.p[f].sched = sched[f];
+        fa.p[f].ntiles = (int)rp.ctas;
+        fa.p[f].cross = rp.out.cross;
+        fa.p[f].strideP = rp.out.strideP;
+    }
+    const RowPass& r0 = P.rp[0];
+    const PhaseGeom& g = P.ph[0];
+    fa.logL = g.logL;
+    fa.logh = ilog2i(r0.h);
+    fa.Ls = r0.Ls;
+    fa.E = g.E;
+    fa.epw = g.epw;
+    fa.w64 = g.w64;
+    fa.stages = r0.stages;
+    fa.data_words = r0.h * r0.Ls;
+    fa.sched_words = (int)((long long)r0.h * (g.L / 32) * g.w64 * 2);
+    fa.sync = sync;
+    fa.trace = trace;
+    const dim3 grid((unsigned)P.fused3_grid), block(32 + kWsPerm + kWsStore);
+    const size_t smem = fused3_smem(P);
+    switch (r0.ept) {
+        case 8: return launch(fused3_ws_kernel<8>, grid, block, smem, s, false, fa);
+        case 16: return launch(fused3_ws_kernel<16>, grid, block, smem, s, false, fa);
+        case 32: return launch(fused3_ws_kernel<32>, grid, block, smem, s, false, fa);
     }
     return cudaErrorInvalidValue;
 }

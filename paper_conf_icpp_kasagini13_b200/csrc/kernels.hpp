@@ -10,15 +10,23 @@
 namespace perm {
 
 // Registers max dynamic shared memory for every kernel instantiation the plan uses.
-cudaError_t prepare_kernels(const HostPlan& P);
+cudaError_t prepare_kernels(HostPlan& P);   // also sets persistent grid sizes
 
 // All three phases in one CTA (n <= 2^15): a -> smem -> R1, R2 (columns), R3 -> b.
 cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
                          uint32_t* b, cudaStream_t s);
 
 // One row pass (pass index f in 0..2) of the 3- or 5-pass pipeline.
+// `trace`: optional device buffer of 16 %globaltimer stamps per CTA (nullptr = off).
 cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, const uint32_t* in,
-                            uint32_t* out, cudaStream_t s, bool pdl);
+                            uint32_t* out, cudaStream_t s, bool pdl,
+                            unsigned long long* trace = nullptr);
+
+// The three row passes of the LINES layout in one persistent launch (square
+// views). `sync`: 3 device u64 counters, zero-initialised once (self-resetting).
+cudaError_t launch_fused3(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
+                          uint32_t* x1, uint32_t* x2, uint32_t* b, unsigned long long* sync,
+                          cudaStream_t s, unsigned long long* trace = nullptr);
 
 // out (cols x rows) = transpose of in (rows x cols), 32 x 32 tiles (§V).
 cudaError_t launch_transpose(const uint32_t* in, uint32_t* out, int64_t rows, int64_t cols,

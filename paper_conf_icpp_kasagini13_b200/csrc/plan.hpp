@@ -18,15 +18,19 @@ namespace perm {
 constexpr int kW = 32;                 // HMM width w = warp size = banks (L199-L207)
 
 // One phase of row-wise permutations: `lines` independent lines of length L.
-// Packed schedule: for line g and warp-round k (k < L/32) there are E 32-bit
-// words; the entry of lane x occupies bits [E*x, E*x + E) of those words
-// (LSB first). entry = (sigma << logL) | t: the lane reads source position
-// s = 32*sigma + x (bank x) and writes destination position t (L519, L533).
+// Device schedule ("W64" format): entry = (sigma << logL) | t, E = 2*logL - 5
+// bits: the lane reads source position s = 32*sigma + x (bank x) and writes
+// destination position t (L519, L533). Entries are packed epw = floor(64/E)
+// to a 64-bit word; warp-round (line g, round k) owns W64 = ceil(32/epw)
+// consecutive 64-bit words, lane x's entry sits in word x/epw at bit
+// E*(x % epw). One 64-bit shared load + one shift decodes it.
 struct PhaseGeom {
     int64_t lines = 0;
     int32_t L = 0, logL = 0;
     int32_t E = 0;        // entry bits = logL + (logL - 5)
-    int64_t words = 0;    // lines * (L/32) * E
+    int32_t epw = 0;      // entries per 64-bit word
+    int32_t w64 = 0;      // 64-bit words per warp-round
+    int64_t words = 0;    // 32-bit words: lines * (L/32) * w64 * 2
 };
 
 // Layout of one row pass of the tiled 3-pass pipeline.
@@ -44,7 +48,10 @@ struct IoMode {
 
 struct RowPass {
     int32_t phase = 0;        // 0,1,2 -> Phi1, Phi2, Phi3
-    int32_t h = 0;            // lines per CTA
+    int32_t tma = 0;          // 1: persistent TMA-pipelined kernel (contiguous input lines)
+    int32_t stages = 0;       // TMA ring depth
+    int64_t grid = 0;         // persistent CTAs (set at upload from the occupancy query)
+    int32_t h = 0;            // lines per CTA (tile)
     int32_t Ls = 0;           // shared-memory line stride (elements) = L + pad
     int32_t ept = 0;          // elements per thread
     int32_t threads = 0;
@@ -59,6 +66,9 @@ struct HostPlan {
     int32_t k = 0;             // log2 n
     int64_t r = 0, c = 0;      // view
     int32_t passes = 0;        // 1, 3, 5
+    int32_t layout = 0;        // 3-pass intermediates: 1 tiled, 2 lines (perm_layout)
+    int32_t fused3 = 0;        // LINES layout, square view: all three passes in one launch
+    int64_t fused3_grid = 0;   // one CTA per SM (set at upload)
     PhaseGeom ph[3];
     RowPass rp[3];
     int32_t fused_ept = 0, fused_threads = 0, fused_Ls = 0;
@@ -77,16 +87,20 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 void euler_split_colour(int64_t nodes, int64_t d, int64_t E, const uint32_t* U,
                         const uint32_t* V, uint32_t* colour, bool parallel);
 
-// Decode the entry of (line, slot q = round*32 + lane) from a packed phase.
+// Position of the entry of (line, slot q = round*32 + lane) in a W64 phase.
+inline void entry_pos(const PhaseGeom& g, int64_t line, int64_t q, int64_t& word64, int& bit) {
+    const int64_t round = q >> 5, lane = q & 31;
+    word64 = (line * (g.L >> 5) + round) * g.w64 + lane / g.epw;
+    bit = (int)(g.E * (lane % g.epw));
+}
+
 inline uint32_t unpack_entry(const std::vector<uint32_t>& words, const PhaseGeom& g,
                              int64_t line, int64_t q) {
-    const int64_t round = q >> 5, lane = q & 31;
-    const uint64_t bit = (uint64_t)((line * (g.L >> 5) + round) * (int64_t)g.E) * 32u +
-                         (uint64_t)(g.E * lane);
-    const uint64_t w0 = bit >> 5, off = bit & 31;
-    uint64_t v = words[w0];
-    if (off + g.E > 32) v |= (uint64_t)words[w0 + 1] << 32;
-    return (uint32_t)((v >> off) & ((1ull << g.E) - 1));
+    int64_t w;
+    int bit;
+    entry_pos(g, line, q, w, bit);
+    const uint64_t v = (uint64_t)words[2 * w] | ((uint64_t)words[2 * w + 1] << 32);
+    return (uint32_t)((v >> bit) & ((1ull << g.E) - 1));
 }
 
 // Simulated shared-memory wavefronts per warp request of a pass's load/store

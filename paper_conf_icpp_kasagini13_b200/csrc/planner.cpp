@@ -324,7 +324,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.L = (int32_t)Ls[f];
         g.logL = logLs[f];
         g.E = 2 * g.logL - 5;
-        g.words = g.lines * (g.L / kW) * g.E;
+        g.epw = 64 / g.E;
+        g.w64 = (kW + g.epw - 1) / g.epw;
+        g.words = g.lines * (g.L / kW) * g.w64 * 2;
         P.sched[f].assign((size_t)g.words, 0u);
         const int64_t L = g.L;
         const uint16_t* ph = phi[f].data();
@@ -341,14 +343,15 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                     V[j] = (uint32_t)(phl[j] & 31);
                 }
                 ec.run(kW, L / kW, L, U.data(), V.data(), col.data(), false);
-                uint32_t* Wl = W + line * (L / kW) * g.E;
                 for (int64_t j = 0; j < L; ++j) {
-                    const uint64_t sigma = (uint64_t)(j >> 5), lane = (uint64_t)(j & 31);
+                    const uint64_t sigma = (uint64_t)(j >> 5);
                     const uint64_t entry = (sigma << g.logL) | phl[j];
-                    const uint64_t bit = (uint64_t)col[j] * g.E * 32u + (uint64_t)g.E * lane;
-                    const uint64_t w0 = bit >> 5, off = bit & 31;
-                    Wl[w0] |= (uint32_t)(entry << off);
-                    if (off + g.E > 32) Wl[w0 + 1] |= (uint32_t)(entry >> (32 - off));
+                    int64_t w;
+                    int bit;
+                    entry_pos(g, line, (int64_t)col[j] * kW + (j & 31), w, bit);
+                    const uint64_t sh = entry << bit;
+                    W[2 * w] |= (uint32_t)sh;
+                    W[2 * w + 1] |= (uint32_t)(sh >> 32);
                 }
             }
         }
@@ -357,14 +360,15 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 
     // pass structure
     int passes = opt ? opt->passes : 0;
-    if (passes == 0) passes = (k <= 15) ? 1 : (k <= 26 ? 3 : 5);
-    if (passes == 1 && k > 15) { err = "fused single-CTA pass needs n <= 2^15"; return PERM_EUNSUPPORTED; }
+    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 26 ? 3 : 5);
+    if (passes == 1 && k > 14) { err = "fused single-CTA pass needs n <= 2^14"; return PERM_EUNSUPPORTED; }
     if (passes != 1 && passes != 3 && passes != 5) { err = "passes must be 0, 1, 3 or 5"; return PERM_EINVAL; }
     P.passes = passes;
     if (passes == 1) {
         P.fused_threads = (int32_t)std::min<int64_t>(512, n / 4);
         P.fused_ept = (int32_t)(n / P.fused_threads);
         P.fused_Ls = (int32_t)(c + 1);   // odd stride: rows AND columns conflict-free (Fig. 4 idea)
+        if (r * P.fused_Ls > 65535) { err = "fused tile exceeds 16-bit shared addresses"; return PERM_EUNSUPPORTED; }
         return PERM_OK;
     }
     const int64_t Q = std::min<int64_t>(16384, std::max<int64_t>(2048, pow2_floor(n / 296)));
@@ -372,7 +376,22 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         int64_t v = opt ? (&opt->h1)[idx] : 0;
         return v > 0 ? v : dflt;
     };
+    const int stages = (opt && opt->stages > 0) ? opt->stages : 2;
+    // bytes of one TMA stage: h lines (stride L + pad) + the tile's packed schedule
+    auto stage_bytes = [&](int64_t h, int f, int pad) -> int64_t {
+        const PhaseGeom& g = P.ph[f];
+        return h * (g.L + pad) * 4 + h * (g.L / kW) * g.w64 * 8;
+    };
+    constexpr int64_t kSmemBudget = 220 * 1024;
+    int layout = opt ? opt->layout : 0;
     if (passes == 3) {
+        if (layout == 0) layout = (k <= 24) ? 2 : 1;
+        if (layout != 1 && layout != 2) { err = "layout must be 0, 1 or 2"; return PERM_EINVAL; }
+    } else {
+        layout = 0;
+    }
+    P.layout = layout;
+    if (passes == 3 && layout == 1) {
         int64_t h2 = pick(1, std::min<int64_t>(32, std::max<int64_t>(4, pow2_floor(Q / r))));
         int64_t h1 = pick(0, std::max<int64_t>(1, pow2_floor(Q / c)));
         int64_t h3 = pick(2, h1);
@@ -394,6 +413,31 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         d.phase = 2; d.h = (int32_t)h3; d.ctas = r / h3;
         d.in = runs(h2, h3 * h2, h3 * c);
         d.out = runs(c, 0, h3 * c);
+    } else if (passes == 3) {
+        // LINES: X1 column-major (c x r), X2 row-major; each pass reads whole lines.
+        for (int f = 0; f < 3; ++f) {
+            const int64_t lines_f = P.ph[f].lines, L = P.ph[f].L;
+            const bool cross_out = f < 2;
+            // default: 8 lines (32-byte column chunks = whole L2 sectors) when two
+            // stages fit, else 4
+            const int pad8 = cross_out ? 4 : 0;
+            int64_t h = pick(f, 2 * stage_bytes(8, f, pad8) <= kSmemBudget ? 8 : 4);
+            if (cross_out && h != 4 && h != 8) { err = "LINES layout: h1, h2 must be 4 or 8"; return PERM_EINVAL; }
+            if (h < 1 || h > lines_f || (h & (h - 1))) { err = "invalid h for the LINES layout"; return PERM_EINVAL; }
+            RowPass& rp = P.rp[f];
+            rp.phase = f; rp.h = (int32_t)h; rp.ctas = lines_f / h;
+            rp.in = runs(L, 0, h * L);
+            if (f == 0) rp.out = cross(1, r, h);          // X1[k*r + i]
+            else if (f == 1) rp.out = cross(1, c, h);     // X2[i'*c + k]
+            else rp.out = runs(c, 0, h * c);              // b rows
+            // warp-specialized kernel when the tile splits into 512 permuter threads
+            const int64_t ept = h * L / 512;
+            rp.tma = (h * L % 512 == 0 && ept >= 8 && ept <= 64) ? 2 : 1;
+            const int pad = (cross_out && h == 8) ? 4 : 0;
+            int st = (opt && opt->stages > 0) ? opt->stages
+                                              : (int)std::min<int64_t>(4, kSmemBudget / stage_bytes(h, f, pad));
+            rp.stages = std::max(1, st);
+        }
     } else {
         for (int f = 0; f < 3; ++f) {
             const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
@@ -403,14 +447,62 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.phase = f; rp.h = (int32_t)h; rp.ctas = lines_f / h;
             rp.in = runs(L, 0, h * L);
             rp.out = runs(L, 0, h * L);
+            // TMA pipeline when `stages` tiles (lines + schedule) fit in shared memory
+            rp.tma = (stages * stage_bytes(h, f, 0) <= kSmemBudget &&
+                      (h * (L / kW) * P.ph[f].w64 * 2) % 4 == 0) ? 1 : 0;
+            rp.stages = rp.tma ? stages : 0;
         }
     }
     for (int f = 0; f < 3; ++f) {
         RowPass& rp = P.rp[f];
         const PhaseGeom& g = P.ph[rp.phase];
-        if ((int64_t)rp.h * g.L * 4 > 200 * 1024) { err = "a CTA's lines exceed the shared-memory budget"; return PERM_EINVAL; }
-        choose_threads(rp, g.L);
-        choose_pad(rp, g);
+        if ((int64_t)rp.h * (g.L + 32) > 65535) { err = "tile exceeds 16-bit shared addresses; lower h"; return PERM_EINVAL; }
+        if (rp.tma == 2) {
+            rp.ept = (int32_t)((int64_t)rp.h * g.L / 512);
+            rp.threads = 32 + 512 + (rp.out.cross ? 256 : 0);
+        } else {
+            choose_threads(rp, g.L);
+        }
+        if (rp.tma) {
+            // TMA tiles: lines land at 16-byte aligned strides; a CROSS store of h = 8
+            // lines needs stride = 4 (mod 8) words to be conflict-free, h = 4 any.
+            const int pad = (rp.out.cross && rp.h == 8) ? 4 : 0;
+            rp.Ls = g.L + pad;
+            rp.conflicts_in = 1;   // bulk copies
+            if (rp.tma == 1) {
+                rp.conflicts_out = simulate_conflicts(rp, g, false);
+            } else {
+                // storer gather: 256 threads, vector f = 4*(j + 256*it)
+                RowPass tmp = rp;
+                tmp.threads = 256;
+                rp.conflicts_out = rp.out.cross ? simulate_conflicts(tmp, g, false) : 1;
+            }
+            if ((rp.h * (g.L / kW) * g.w64 * 2) % 4) { err = "TMA tile schedule is not 16-byte sized"; return PERM_EINVAL; }
+            if (rp.stages * stage_bytes(rp.h, rp.phase, pad) > kSmemBudget) {
+                err = "TMA stages exceed the shared-memory budget; lower h or stages";
+                return PERM_EINVAL;
+            }
+        } else {
+            if ((int64_t)rp.h * g.L * 4 > 200 * 1024) { err = "a CTA's lines exceed the shared-memory budget"; return PERM_EINVAL; }
+            choose_pad(rp, g);
+        }
+    }
+    // one persistent launch for all three passes: LINES layout, square view, and
+    // the three passes share tile shape, stride and pipeline depth
+    // auto (0) keeps three launches: measured faster at 2^22 on B200 so far
+    const int fuse = opt ? opt->fuse : 0;
+    if (passes == 3 && layout == 2 && fuse > 0 && r == c) {
+        const RowPass &a0 = P.rp[0], &a1 = P.rp[1], &a2 = P.rp[2];
+        const bool same = a0.tma == 2 && a1.tma == 2 && a2.tma == 2 && a0.h == a1.h &&
+                          a1.h == a2.h && a0.stages == a1.stages && a1.stages == a2.stages &&
+                          a0.ept == a1.ept && a1.ept == a2.ept && (a0.ept == 8 || a0.ept == 16 || a0.ept == 32);
+        if (same) {
+            P.fused3 = 1;
+            for (int f = 0; f < 3; ++f) {   // one shared slot layout (the CROSS stride)
+                P.rp[f].Ls = a0.Ls;
+                P.rp[f].threads = 32 + 512 + 256;
+            }
+        }
     }
     return PERM_OK;
 }

@@ -104,8 +104,9 @@ def test_cpp_plan_22_random(lib):
     info, kappa, sched = export_plan(lib, p)
     OC.assert_plan(p, kappa, sched, r, c, 32)
     assert info["passes"] == 3
-    # schedule = (2 log2 L - 5) bits per element per phase: 3 * 17 bits at L = 2048
-    assert info["sched_bytes"] == 3 * n * 17 // 8
+    # W64 schedule: 17-bit entries, 3 per 64-bit word, 11 words per warp-round of 32
+    assert info["entry_bits"] == [17, 17, 17]
+    assert info["sched_bytes"] == 3 * (n // 32) * 11 * 8
 
 
 def test_pass_options_and_info(lib):
