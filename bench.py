@@ -8,7 +8,7 @@ b[p[i]] = a[i]". Workload (BASELINE configs[1]): n = 2^22 float32 (raw 32-bit
 words), the paper's five permutation families (identity, shuffle, random,
 bit-reversal, transpose). One STEP = one perm_apply of
 each of the five plans (all §8(a) rows: R1 -> R2 -> R3), with L2 flushed
-(256 MiB memset) before every apply, outside the event-timed region.
+(256 MiB write + read) before every apply, outside the event-timed region.
 
 value      = whole-job effective GB/s = sum over ranks of 5 * 2 * n * 4 B / step time
              (device time from CUDA events on the launch stream, max over ranks)
@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--families", default=",".join(W.FAMILIES))
     ap.add_argument("--passes", type=int, default=0)
     ap.add_argument("--h", default="0,0,0")
+    ap.add_argument("--layout", type=int, default=0)
+    ap.add_argument("--fuse", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -148,6 +150,16 @@ def cpu_oracle_baseline(plans_host, n, seconds: float) -> dict:
                       f"({dt:.1f} s, oracle/c/apply_ref.c OpenMP loop)"}
 
 
+def workload_config(args) -> dict:
+    """The `config` object, identical for both arms (--impl ours / reference)."""
+    fams = args.families.split(",")
+    return {"workload": f"n=2^{args.log2n} float32 (raw u32 words), permutation families "
+                        f"{'/'.join(fams)} (PAPER.md L373-L389), one perm_apply of each per step",
+            "n": 1 << args.log2n, "families": fams,
+            "l2": "flushed before every timed apply (256 MiB write + read, > 126 MB L2)",
+            "parallelism": f"replicas x{args.gpus}"}
+
+
 def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
@@ -170,8 +182,7 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
-            "config": {"workload": f"n=2^{args.log2n} float32 words, families {fams}",
-                       "n": n, "families": fams},
+            "config": workload_config(args),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": capply.threads(),
                              "kind": "oracle",
                              "sample": f"full workload, {args.steps} steps (no sampling needed)"},
@@ -204,7 +215,7 @@ def main():
         p = W.make_perm(f, n)
         a = W.make_data(n)
         t0 = time.perf_counter()
-        plans[f] = pkg.Plan(p, passes=args.passes, h=h)
+        plans[f] = pkg.Plan(p, passes=args.passes, h=h, layout=args.layout, fuse=args.fuse)
         build_ms[f] = (time.perf_counter() - t0) * 1e3
         dA[f] = torch.from_numpy(a.view(np.int32)).to(dev)
         dB[f] = torch.empty_like(dA[f])
@@ -213,8 +224,14 @@ def main():
     info = plans[fams[0]].info()
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
 
-    def timed_apply(fn, ev0, ev1):
+    def flush_l2():
+        # write a 256 MiB buffer (> 126 MB L2), then read it back so the L2 holds
+        # clean lines: the timed kernel pays neither stale hits nor write-backs
         flush.zero_()
+        flush.sum()
+
+    def timed_apply(fn, ev0, ev1):
+        flush_l2()
         ev0.record(stream)
         fn()
         ev1.record(stream)
@@ -280,7 +297,7 @@ def main():
     for f in fams:
         plans[f].set_profiling(True)
         for _ in range(args.steps):
-            flush.zero_()
+            flush_l2()
             plans[f].apply(dA[f], dB[f], stream)
             kern[f].append(plans[f].pass_times())
         plans[f].set_profiling(False)
@@ -289,15 +306,22 @@ def main():
               for i in range(nk)]
     dom = int(np.argmax(mean_k))
     E = info["entry_bits"]
-    kinds = (["R1", "R2", "R3"] if info["passes"] == 3 else
-             ["R1", "T", "R2", "T", "R3"] if info["passes"] == 5 else ["fused R1+R2+R3"])
-    if info["passes"] == 3:
-        alg = [2 * n * 4 + n * E[i] / 8 for i in range(3)]
+    # device schedule bytes per element of each phase (W64 format: floor(64/E) entries
+    # per 64-bit word, ceil(32/epw) words per warp-round of 32 elements)
+    sbpe = [8 * (-(-32 // (64 // e))) / 32 for e in E]
+    if info["kernels_per_apply"] == 1 and info["passes"] == 3:
+        kinds = ["fused R1+R2+R3"]
+        alg = [2 * n * 4 + n * sum(sbpe)]
+    elif info["passes"] == 3:
+        kinds = ["R1", "R2", "R3"]
+        alg = [2 * n * 4 + n * sbpe[i] for i in range(3)]
     elif info["passes"] == 5:
-        alg = [2 * n * 4 + n * E[0] / 8, 2 * n * 4, 2 * n * 4 + n * E[1] / 8, 2 * n * 4,
-               2 * n * 4 + n * E[2] / 8]
+        kinds = ["R1", "T", "R2", "T", "R3"]
+        alg = [2 * n * 4 + n * sbpe[0], 2 * n * 4, 2 * n * 4 + n * sbpe[1], 2 * n * 4,
+               2 * n * 4 + n * sbpe[2]]
     else:
-        alg = [2 * n * 4 + n * sum(E) / 8]
+        kinds = ["fused single-CTA"]
+        alg = [2 * n * 4 + n * sum(sbpe)]
     peaks = measured_peaks()
     achieved = alg[dom] / (mean_k[dom] * 1e-3) / 1e9
     traffic = None
@@ -323,7 +347,7 @@ def main():
         for _ in range(args.steps):
             tot = 0.0
             for f in fams:
-                flush.zero_()
+                flush_l2()
                 torch.cuda.synchronize()
                 t0 = time.perf_counter()
                 plans[f].apply_host(pinned[f][0], pinned[f][1], stream)   # syncs the stream
@@ -344,12 +368,10 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": f"n=2^{args.log2n} float32 (raw u32 words), 5 permutation "
-                                   "families, one perm_apply each per step",
-                       "n": n, "families": fams, "view": [info["rows"], info["cols"]],
-                       "passes": info["passes"], "h": info["h"],
-                       "l2": "flushed (256 MiB memset) before every timed apply",
-                       "parallelism": f"replicas x{world}"},
+            "config": workload_config(args),
+            "plan": {"view": [info["rows"], info["cols"]], "passes": info["passes"],
+                     "kernels_per_apply": info["kernels_per_apply"], "h": info["h"],
+                     "entry_bits": info["entry_bits"], "layout": plans[fams[0]].describe().get("layout")},
             "apply_us": per_fam_us,
             "conventional_us": {f: 1e3 * conv[f] for f in fams},
             "s_designated_us": {f: 1e3 * gather[f] for f in fams},
