@@ -109,3 +109,73 @@ def assert_plan(p, kappa, sched, rows, cols, w):
     if bad or missing:
         raise AssertionError(f"plan invariants failed: {bad} missing: {sorted(missing)}")
     return res
+
+
+# ---------------------------------------------------------------- tile-level coloured plans
+#
+# DESIGN.md §5 "TLC": each of the three row-wise permutations runs on tiles of h
+# lines. A tile is read from global memory in its stored order into buffer A and
+# written in the stored order of the pass's output into buffer B; a plan entry
+# (tile T, warp-round q, lane x) is (src offset in A, dst offset in B). The
+# layouts (restated here from DESIGN.md, not imported from the product):
+#   X1[((K*(r/h1) + I)*h1 + i_in)*h2 + k_in]        (K = k div h2, I = i div h1)
+#   X2[((I'*(c/h2) + K)*h3 + i_in')*h2 + k_in]
+#   pass 1, tile I : A = rows I*h1.. of a (i_in*c + j);       B = [K][i_in][k_in]
+#   pass 2, tile K : A = X1 block K   ([i][k_in]);            B = [I'][i_in'][k_in]
+#   pass 3, tile I': A = X2 block I'  ([K][i_in'][k_in]);     B = rows of b (i_in'*c + k')
+# The checker maps every src back to its element, routes the element with the
+# Phi it recomputes from kappa and P, and requires: dst = the layout position of
+# the routed element (i.e. the pass implements Phi), every src and every dst of
+# a tile used once, lane = src mod w, and every round touching w distinct banks
+# in A and in B (L531-L533 generalised from a line to a tile).
+
+def check_tlc(p, kappa, sched, rows: int, cols: int, h, w: int = 32) -> dict:
+    p = np.asarray(p, dtype=np.int64)
+    kappa = np.asarray(kappa, dtype=np.int64)
+    r, c = rows, cols
+    h1, h2, h3 = h
+    n = r * c
+    res = {}
+    res["i_row_colours_bijective"] = _rows_are_perms(kappa.reshape(r, c))
+    key = kappa * r + p // c
+    res["ii_colour_dest_rows_distinct"] = bool(np.unique(key).size == n)
+    if not (res["i_row_colours_bijective"] and res["ii_colour_dest_rows_distinct"]):
+        return res
+    phi1, phi2, phi3 = phases_from_kappa(p, kappa, r, c)
+    ok_map = ok_cover = ok_banks = ok_lane = True
+    for f, (HL, lines, hh) in enumerate(((h1 * c, r, h1), (r * h2, c, h2), (h3 * c, r, h3))):
+        e = np.asarray(sched[f], dtype=np.int64).reshape(lines // hh, HL)
+        src, dst = e >> 16, e & 0xFFFF
+        T = np.arange(lines // hh, dtype=np.int64)[:, None]
+        lane = (np.arange(HL, dtype=np.int64) % w)[None, :]
+        ok_lane &= bool(np.all(src % w == lane))
+        ok_cover &= _rows_are_perms(src) and _rows_are_perms(dst)
+        ok_banks &= _rounds_distinct(src, w) and _rounds_distinct(dst, w)
+        if f == 0:
+            i = T * h1 + src // c
+            j = src % c
+            k = phi1[i, j]
+            want = ((k // h2) * h1 + (i - T * h1)) * h2 + k % h2
+        elif f == 1:
+            i = src // h2
+            k = T * h2 + src % h2
+            ip = phi2[k, i]
+            want = ip * h2 + (k - T * h2)
+        else:
+            K, rem = src // (h3 * h2), src % (h3 * h2)
+            i_in, k_in = rem // h2, rem % h2
+            k = K * h2 + k_in
+            ip = T * h3 + i_in
+            want = i_in * c + phi3[ip, k]
+        ok_map &= bool(np.all(dst == want))
+    res["iii_phases_bijective"] = all(_rows_are_perms(ph) for ph in (phi1, phi2, phi3))
+    x = np.arange(n, dtype=np.int64)
+    i, j = x // c, x % c
+    k = phi1[i, j]
+    row2 = phi2[k, i]
+    res["iv_composition_is_P"] = bool(np.all(row2 * c + phi3[row2, k] == p))
+    res["v_tiles_implement_phi"] = ok_map
+    res["vi_rounds_conflict_free_A_and_B"] = ok_banks
+    res["vii_sources_and_dests_cover_tile"] = ok_cover
+    res["viii_lane_is_source_bank"] = ok_lane
+    return res

@@ -35,6 +35,7 @@ struct perm_plan {
     unsigned long long* d_trace = nullptr;
     int64_t trace_stride = 0;          // CTAs per pass slot
     unsigned long long* d_sync = nullptr;   // fused 3-pass grid-barrier counters
+    alignas(64) CUtensorMap tlc_maps[3];   // TLC layout: TMA tensor maps of X1, X2
 };
 
 namespace {
@@ -77,7 +78,7 @@ int upload(perm_plan* pl) {
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
     auto padded = [](int64_t w) { return (w + 32 + 63) / 64 * 64; };   // guard, 256-B aligned phases
     int64_t words = 0;
-    for (int f = 0; f < 3; ++f) words += padded(P.ph[f].words);
+    for (int f = 0; f < 3; ++f) words += padded((int64_t)P.sched[f].size());
     pl->sched_bytes = words * 4;
     e = cudaMalloc(&pl->d_sched, (size_t)pl->sched_bytes);
     if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc schedules: ") + cudaGetErrorString(e));
@@ -85,12 +86,12 @@ int upload(perm_plan* pl) {
     int64_t off = 0;
     for (int f = 0; f < 3; ++f) {
         pl->d_phase[f] = pl->d_sched + off;
-        e = cudaMemcpy(pl->d_phase[f], P.sched[f].data(), (size_t)P.ph[f].words * 4,
-                       cudaMemcpyHostToDevice);
+        const int64_t wf = (int64_t)P.sched[f].size();
+        e = cudaMemcpy(pl->d_phase[f], P.sched[f].data(), (size_t)wf * 4, cudaMemcpyHostToDevice);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy schedules");
-        e = cudaMemset(pl->d_phase[f] + P.ph[f].words, 0, 32 * 4);
+        e = cudaMemset(pl->d_phase[f] + wf, 0, 32 * 4);
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemset");
-        off += padded(P.ph[f].words);
+        off += padded(wf);
     }
     if (P.passes != 1) {
         const size_t bytes = (size_t)P.n * P.eb;
@@ -102,6 +103,10 @@ int upload(perm_plan* pl) {
     }
     e = perm::prepare_kernels(P);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
+    if (P.layout == 3) {
+        e = perm::make_tlc_maps(P, pl->d_scratch[0], pl->d_scratch[1], pl->tlc_maps);
+        if (e != cudaSuccess) return cuda_fail(e, "cuTensorMapEncodeTiled");
+    }
     if (P.fused3) {
         e = cudaMalloc(&pl->d_sync, 4 * sizeof(unsigned long long));
         if (e == cudaSuccess) e = cudaMemset(pl->d_sync, 0, 4 * sizeof(unsigned long long));
@@ -187,14 +192,14 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->rows = P.r;
     out->cols = P.c;
     int64_t words = 0;
-    for (int f = 0; f < 3; ++f) words += P.ph[f].words;
+    for (int f = 0; f < 3; ++f) words += (int64_t)P.sched[f].size();
     out->sched_bytes = plan->on_device ? plan->sched_bytes : words * 4;
     out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes == 1 ? 0 : 2 * P.n * P.eb);
     out->elem_bytes = P.eb;
     out->passes = P.passes;
     out->kernels_per_apply = P.fused3 ? 1 : P.passes;
     for (int f = 0; f < 3; ++f) {
-        out->entry_bits[f] = P.ph[f].E;
+        out->entry_bits[f] = P.layout == 3 ? P.tp[f].E : P.ph[f].E;
         out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
     }
     out->planner_threads = P.threads_used;
@@ -253,6 +258,23 @@ int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint3
     const HostPlan& P = plan->host;
     if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));
     uint32_t* outs[3] = {s1, s2, s3};
+    if (P.layout == 3) {
+        // TLC: entry (tile T, round q, lane x) -> (src word offset in A << 16) | dst offset in B
+        for (int f = 0; f < 3; ++f) {
+            if (!outs[f]) continue;
+            const perm::TlcPass& tp = P.tp[f];
+#pragma omp parallel for schedule(static)
+            for (int64_t T = 0; T < tp.ntiles; ++T)
+                for (int64_t q = 0; q < tp.HL / 32; ++q)
+                    for (int64_t x = 0; x < 32; ++x) {
+                        const uint32_t e = perm::tlc_entry(P.sched[f], tp, T, q, x);
+                        const uint32_t src = ((e >> tp.logHL) << 5) | (uint32_t)x;
+                        const uint32_t dst = e & (uint32_t)(tp.HL - 1);
+                        outs[f][T * tp.HL + q * 32 + x] = (src << 16) | dst;
+                    }
+        }
+        return PERM_OK;
+    }
     for (int f = 0; f < 3; ++f) {
         if (!outs[f]) continue;
         const perm::PhaseGeom& g = P.ph[f];
@@ -352,6 +374,18 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
         e = perm::launch_fused(P, sc, in, out, s);
         mark();
+    } else if (P.layout == 3 && P.fused3) {
+        const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
+        e = perm::launch_tlc_fused(P, plan->tlc_maps, sc, in, plan->d_scratch[0], plan->d_scratch[1], out,
+                                   plan->d_sync, s, tr(0));
+        mark();
+    } else if (P.layout == 3) {
+        uint32_t* x1 = plan->d_scratch[0];
+        uint32_t* x2 = plan->d_scratch[1];
+        e = perm::launch_tlc_pass(P, 0, plan->tlc_maps, plan->d_phase[0], in, x1, s, false, tr(0));
+        mark();
+        if (e == cudaSuccess) { ++k; e = perm::launch_tlc_pass(P, 1, plan->tlc_maps, plan->d_phase[1], x1, x2, s, !prof, tr(1)); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_tlc_pass(P, 2, plan->tlc_maps, plan->d_phase[2], x2, out, s, !prof, tr(2)); mark(); }
     } else if (P.fused3) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
         e = perm::launch_fused3(P, sc, in, plan->d_scratch[0], plan->d_scratch[1], out, plan->d_sync,

@@ -21,9 +21,13 @@
 //  * passes are chained with programmatic dependent launch: a pass
 //    prefetches its schedule into L2 before griddepcontrol.wait, so the
 //    schedule stream overlaps the previous pass.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
+#include <cstring>
 
 #include "kernels.hpp"
 
@@ -84,6 +88,9 @@ __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.comm
 __device__ __forceinline__ void bulk_wait_read0() {
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
+__device__ __forceinline__ void bulk_wait_read1() {
+    asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+}
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -101,14 +108,6 @@ __device__ __forceinline__ void st_v4(uint32_t* p, uint4 v) {
     asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
                  "r"(v.w)
                  : "memory");
-}
-
-// Entry of this lane from the E words of one warp-round held one per lane
-// (lane j holds word j): bits [E*lane, E*lane + E).
-__device__ __forceinline__ uint32_t decode_entry(uint32_t word, int w0, int off, uint32_t mask) {
-    const uint32_t lo = __shfl_sync(kFull, word, w0);
-    const uint32_t hi = __shfl_sync(kFull, word, w0 + 1);
-    return __funnelshift_r(lo, hi, off) & mask;
 }
 
 // ------------------------------------------------------------------ permute hop
@@ -921,6 +920,379 @@ __global__ void __launch_bounds__(32 + kWsPerm + kWsStore, 1) fused3_ws_kernel(c
     stamp(tr, 15);
 }
 
+// ------------------------------------------------------------------ TLC row pass (tile-level colouring)
+
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void* src, int c0, int c1, int c2) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+            reinterpret_cast<uint64_t>(map)),
+        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2)
+        : "memory");
+}
+__device__ __forceinline__ void tma_store_4d(const CUtensorMap* map, const void* src, int c0, int c1, int c2,
+                                             int c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+            reinterpret_cast<uint64_t>(map)),
+        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+}
+
+__host__ __device__ constexpr int cilog2(int v) { return v <= 1 ? 0 : 1 + cilog2(v >> 1); }
+
+struct TlcArgs {
+    const uint32_t* in;
+    uint32_t* out;             // row-major output (OUT == 0)
+    const uint32_t* sched;
+    int ntiles, stages;
+    long long tile_words;      // schedule words per tile
+    int t_h;                   // lines per tile (tensor-store coordinates)
+    int nbox, box_outer, box_words;
+    unsigned long long* trace;
+};
+
+// One row-wise permutation pass (Lemma 7) with the tile-level bank colouring
+// (plan.hpp TlcPass). A tile of h lines is TMA-loaded into A in its global
+// order; 512 permuter threads move every element A[src] -> B[dst] in
+// warp-rounds that touch 32 distinct banks of A and 32 distinct banks of B;
+// B is already in the global order of the output, so the transposes of the
+// column-wise step (Lemma 8) cost nothing extra: B leaves by TMA (1-D bulk
+// store for row-major output, 3-D / 4-D tensor stores of 64-byte chunks for
+// the intermediates). Roles: warp 0 lane 0 = TMA producer, warp 1 lane 0 =
+// TMA storer, warps 2..17 = permuters; `stages` slots of [A | B].
+template <int EPT, int OUT>
+__global__ void __launch_bounds__(64 + kTlcPerm, 1)
+    row_pass_tlc_kernel(const __grid_constant__ CUtensorMap tmap, const TlcArgs a) {
+    constexpr int HL = kTlcPerm * EPT;
+    constexpr int LOGHL = cilog2(HL);
+    constexpr int E = 2 * LOGHL - 5;
+    constexpr int NWORDS = (EPT * E + 31) / 32;
+    constexpr uint32_t EMASK = (1u << E) - 1u;
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int NS = a.stages;
+    const int G = gridDim.x;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * 2 * HL);
+    uint64_t* permd = full + NS;
+    uint64_t* empty = permd + NS;
+    unsigned long long* tr = a.trace;
+    stamp(tr, 0);
+    if (tid == 0) {
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&permd[s], kTlcPerm);
+            mbar_init(&empty[s], 1);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---------------- producer
+            for (int i = 0; i <= NS; ++i) {      // schedules do not depend on the previous pass
+                const long long t = blockIdx.x + (long long)i * G;
+                if (t < a.ntiles) prefetch_l2_bulk(a.sched + t * a.tile_words, (uint32_t)(a.tile_words * 4));
+            }
+            pdl_wait();
+            stamp(tr, 1);
+            for (int i = 0;; ++i) {
+                const long long t = blockIdx.x + (long long)i * G;
+                if (t >= a.ntiles) break;
+                const int s = i % NS;
+                if (i >= NS) mbar_wait(&empty[s], (uint32_t)(i / NS - 1) & 1u);
+                fence_proxy_async();
+                mbar_arrive_expect_tx(&full[s], (uint32_t)HL * 4u);
+                bulk_g2s(smem + s * 2 * HL, a.in + t * HL, (uint32_t)HL * 4u, &full[s]);
+                const long long tp = t + (long long)(NS + 1) * G;
+                if (tp < a.ntiles) prefetch_l2_bulk(a.sched + tp * a.tile_words, (uint32_t)(a.tile_words * 4));
+                if (i == 0) pdl_launch_dependents();
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ---------------- storer (stores stay one tile deep in flight)
+            pdl_wait();
+            int pend_s = -1;
+            for (int i = 0;; ++i) {
+                const long long t = blockIdx.x + (long long)i * G;
+                if (t >= a.ntiles) break;
+                const int s = i % NS;
+                mbar_wait(&permd[s], (uint32_t)(i / NS) & 1u);
+                fence_proxy_async();       // permuters' smem writes -> async-proxy reads
+                const uint32_t* B = smem + s * 2 * HL + HL;
+                if constexpr (OUT == 0) {
+                    bulk_s2g(a.out + t * HL, B, (uint32_t)HL * 4u);
+                } else if constexpr (OUT == 1) {
+                    for (int b = 0; b < a.nbox; ++b)
+                        tma_store_3d(&tmap, B + b * a.box_words, 0, (int)(t * a.t_h), b * a.box_outer);
+                } else {
+                    for (int b = 0; b < a.nbox; ++b)
+                        tma_store_4d(&tmap, B + b * a.box_words, 0, 0, (int)t, b * a.box_outer);
+                }
+                bulk_commit();
+                if (NS == 1) {                 // a single slot cannot wait for the next tile
+                    bulk_wait_read0();
+                    mbar_arrive(&empty[s]);
+                } else {
+                    if (pend_s >= 0) {
+                        bulk_wait_read1();
+                        mbar_arrive(&empty[pend_s]);
+                    }
+                    pend_s = s;
+                }
+                if (i < 4) stamp_if(tr, true, 4 + 3 * i);
+            }
+            if (pend_s >= 0) {
+                bulk_wait_read0();
+                mbar_arrive(&empty[pend_s]);
+            }
+            bulk_wait0();
+        }
+    } else {
+        // ---------------- permuters
+        const int pw = warp - 2;
+        const bool lead = tid == 64;
+        const uint32_t* sp = a.sched + pw * NWORDS * 32 + lane;
+        uint32_t wc[NWORDS], wn[NWORDS];
+        {
+            const long long t = blockIdx.x;
+            if (t < a.ntiles) {
+#pragma unroll
+                for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + t * a.tile_words + w * 32);
+            }
+        }
+        for (int i = 0;; ++i) {
+            const long long t = blockIdx.x + (long long)i * G;
+            if (t >= a.ntiles) break;
+            const int s = i % NS;
+            const long long tn = t + G;
+            if (tn < a.ntiles) {
+#pragma unroll
+                for (int w = 0; w < NWORDS; ++w) wn[w] = __ldg(sp + tn * a.tile_words + w * 32);
+            }
+            mbar_wait(&full[s], (uint32_t)(i / NS) & 1u);
+            if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
+            const uint32_t* __restrict__ A = smem + s * 2 * HL;
+            uint32_t* __restrict__ B = smem + s * 2 * HL + HL;
+            uint32_t v[EPT];
+            uint32_t d[EPT];
+#pragma unroll
+            for (int m = 0; m < EPT; ++m) {
+                const int bit = m * E, w = bit >> 5, off = bit & 31;
+                uint32_t e;
+                if (off + E <= 32) e = (wc[w] >> off) & EMASK;
+                else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
+                v[m] = A[((e >> LOGHL) << 5) | lane];
+                d[m] = e & (HL - 1);
+            }
+#pragma unroll
+            for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
+            mbar_arrive(&permd[s]);
+#pragma unroll
+            for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
+        }
+        stamp_if(tr, lead, 3);
+    }
+    stamp(tr, 14);
+}
+
+// ------------------------------------------------------------------ TLC, all three passes in one launch
+
+struct TlcPassCfg {
+    const uint32_t* in;
+    uint32_t* out;             // row-major output (kind 0)
+    const uint32_t* sched;
+    int ntiles;
+    int kind;                  // 0: rows (1-D bulk store), 1: X1 3-D tensor, 2: X2 4-D tensor
+    int t_h, nbox, box_outer, box_words;
+};
+
+struct TlcFusedArgs {
+    TlcPassCfg p[3];
+    long long tile_words;
+    int stages;
+    unsigned long long* sync;  // [0], [1]: barrier arrivals after pass 0 / 1; [2]: exits
+    unsigned long long* trace;
+};
+
+// Thm 9 in ONE persistent launch with the TLC passes (square views: the three
+// passes share the tile size HL). Same roles and slot ring as
+// row_pass_tlc_kernel, continued across passes (global tile sequence j). The
+// storer publishes a CTA's pass-k output once its bulk stores have COMPLETED
+// (wait_group 0, then a release at gpu scope on sync[k]); the producer TMA-loads
+// pass k+1 data only after sync[k] reaches the grid size (schedule prefetches go
+// ahead of the barrier). One co-resident CTA per SM; the last CTA out resets
+// the counters, so the launch is replayable (CUDA graphs).
+template <int EPT>
+__global__ void __launch_bounds__(64 + kTlcPerm, 1)
+    fused_tlc_kernel(const __grid_constant__ CUtensorMap map_x1,
+                     const __grid_constant__ CUtensorMap map_x2, const TlcFusedArgs a) {
+    constexpr int HL = kTlcPerm * EPT;
+    constexpr int LOGHL = cilog2(HL);
+    constexpr int E = 2 * LOGHL - 5;
+    constexpr int NWORDS = (EPT * E + 31) / 32;
+    constexpr uint32_t EMASK = (1u << E) - 1u;
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int NS = a.stages;
+    const int G = gridDim.x;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * 2 * HL);
+    uint64_t* permd = full + NS;
+    uint64_t* empty = permd + NS;
+    unsigned long long* tr = a.trace;
+    stamp(tr, 0);
+    if (tid == 0) {
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&permd[s], kTlcPerm);
+            mbar_init(&empty[s], 1);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    auto my_tiles = [&](int k) -> int {
+        const int nt = a.p[k].ntiles - (int)blockIdx.x;
+        return nt > 0 ? (nt + G - 1) / G : 0;
+    };
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---------------- producer
+            for (int i = 0; i < my_tiles(0) && i <= NS; ++i)
+                prefetch_l2_bulk(a.p[0].sched + (blockIdx.x + (long long)i * G) * a.tile_words,
+                                 (uint32_t)(a.tile_words * 4));
+            int j = 0;
+            for (int k = 0; k < 3; ++k) {
+                const TlcPassCfg& pc = a.p[k];
+                const int nt = my_tiles(k);
+                if (k > 0) {
+                    for (int i = 0; i < nt; ++i)      // next pass's schedules: independent of data
+                        prefetch_l2_bulk(pc.sched + (blockIdx.x + (long long)i * G) * a.tile_words,
+                                         (uint32_t)(a.tile_words * 4));
+                    while (ld_acquire_gpu(&a.sync[k - 1]) < (unsigned long long)G) __nanosleep(32);
+                    fence_proxy_async_global();
+                    stamp(tr, 1 + 4 * k);
+                }
+                for (int i = 0; i < nt; ++i, ++j) {
+                    const long long t = blockIdx.x + (long long)i * G;
+                    const int s = j % NS;
+                    if (j >= NS) mbar_wait(&empty[s], (uint32_t)(j / NS - 1) & 1u);
+                    fence_proxy_async();
+                    mbar_arrive_expect_tx(&full[s], (uint32_t)HL * 4u);
+                    bulk_g2s(smem + s * 2 * HL, pc.in + t * HL, (uint32_t)HL * 4u, &full[s]);
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ---------------- storer (stores stay one tile deep in flight)
+            int j = 0;
+            int pend_s = -1;                 // slot of the previous, not yet released store
+            for (int k = 0; k < 3; ++k) {
+                const TlcPassCfg& pc = a.p[k];
+                const int nt = my_tiles(k);
+                for (int i = 0; i < nt; ++i, ++j) {
+                    const long long t = blockIdx.x + (long long)i * G;
+                    const int s = j % NS;
+                    mbar_wait(&permd[s], (uint32_t)(j / NS) & 1u);
+                    fence_proxy_async();
+                    const uint32_t* B = smem + s * 2 * HL + HL;
+                    if (pc.kind == 0) {
+                        bulk_s2g(pc.out + t * HL, B, (uint32_t)HL * 4u);
+                    } else if (pc.kind == 1) {
+                        for (int b = 0; b < pc.nbox; ++b)
+                            tma_store_3d(&map_x1, B + b * pc.box_words, 0, (int)(t * pc.t_h), b * pc.box_outer);
+                    } else {
+                        for (int b = 0; b < pc.nbox; ++b)
+                            tma_store_4d(&map_x2, B + b * pc.box_words, 0, 0, (int)t, b * pc.box_outer);
+                    }
+                    bulk_commit();
+                    if (NS == 1) {
+                        bulk_wait_read0();
+                        mbar_arrive(&empty[s]);
+                    } else {
+                        if (pend_s >= 0) {
+                            bulk_wait_read1();       // the previous store has read its slot
+                            mbar_arrive(&empty[pend_s]);
+                        }
+                        pend_s = s;
+                    }
+                }
+                if (pend_s >= 0) {
+                    bulk_wait_read0();
+                    mbar_arrive(&empty[pend_s]);
+                    pend_s = -1;
+                }
+                if (k < 2) {
+                    bulk_wait0();                    // this CTA's pass-k output is written
+                    fence_proxy_async_global();
+                    __threadfence();
+                    red_release_gpu_add(&a.sync[k], 1ull);
+                    stamp(tr, 4 + 4 * k);
+                }
+            }
+            bulk_wait0();
+        }
+    } else {
+        // ---------------- permuters
+        const int pw = warp - 2;
+        const bool lead = tid == 64;
+        int j = 0;
+        for (int k = 0; k < 3; ++k) {
+            const TlcPassCfg& pc = a.p[k];
+            const int nt = my_tiles(k);
+            const uint32_t* sp = pc.sched + pw * NWORDS * 32 + lane;
+            uint32_t wc[NWORDS], wn[NWORDS];
+            if (nt > 0) {
+#pragma unroll
+                for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + (long long)blockIdx.x * a.tile_words + w * 32);
+            }
+            for (int i = 0; i < nt; ++i, ++j) {
+                const int s = j % NS;
+                if (i + 1 < nt) {
+                    const long long tn = blockIdx.x + (long long)(i + 1) * G;
+#pragma unroll
+                    for (int w = 0; w < NWORDS; ++w) wn[w] = __ldg(sp + tn * a.tile_words + w * 32);
+                }
+                mbar_wait(&full[s], (uint32_t)(j / NS) & 1u);
+                if (i == 0) stamp_if(tr, lead, 2 + 4 * k);
+                const uint32_t* __restrict__ A = smem + s * 2 * HL;
+                uint32_t* __restrict__ B = smem + s * 2 * HL + HL;
+                uint32_t v[EPT];
+                uint32_t d[EPT];
+#pragma unroll
+                for (int m = 0; m < EPT; ++m) {
+                    const int bit = m * E, w = bit >> 5, off = bit & 31;
+                    uint32_t e;
+                    if (off + E <= 32) e = (wc[w] >> off) & EMASK;
+                    else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
+                    v[m] = A[((e >> LOGHL) << 5) | lane];
+                    d[m] = e & (HL - 1);
+                }
+#pragma unroll
+                for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
+                mbar_arrive(&permd[s]);
+#pragma unroll
+                for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
+            }
+            stamp_if(tr, lead, 3 + 4 * k);
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        const unsigned long long old = atomicAdd(&a.sync[2], 1ull);
+        if (old == (unsigned long long)G - 1) {
+            a.sync[0] = 0;
+            a.sync[1] = 0;
+            a.sync[2] = 0;
+            __threadfence();
+        }
+    }
+    stamp(tr, 15);
+}
+
 // ------------------------------------------------------------------ transpose
 
 // PAPER.md §V (Lemma 5): w x w tiles through shared memory. The tile is stored
@@ -1111,9 +1483,196 @@ cudaError_t prep_fused3(HostPlan& P) {
     return cudaSuccess;
 }
 
+size_t tlc_smem(const HostPlan& P, int f) {
+    const TlcPass& tp = P.tp[f];
+    return (size_t)tp.stages * 2 * tp.HL * 4 + (size_t)tp.stages * 8 * 3;
+}
+
+template <int EPT, int OUT>
+cudaError_t prep_tlc_one(HostPlan& P, int f) {
+    const size_t smem = tlc_smem(P, f);
+    cudaError_t e = set_smem(row_pass_tlc_kernel<EPT, OUT>, smem);
+    if (e != cudaSuccess) return e;
+    int nb = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_tlc_kernel<EPT, OUT>, 64 + kTlcPerm, smem);
+    if (e != cudaSuccess) return e;
+    if (nb < 1) return cudaErrorInvalidConfiguration;
+    TlcPass& tp = P.tp[f];
+    const long long cap = (long long)nb * sm_count();
+    tp.grid = tp.ntiles < cap ? tp.ntiles : cap;
+    P.rp[f].grid = tp.grid;
+    return cudaSuccess;
+}
+
+template <int OUT>
+cudaError_t prep_tlc_out(HostPlan& P, int f) {
+    switch (P.tp[f].ept) {
+        case 8: return prep_tlc_one<8, OUT>(P, f);
+        case 16: return prep_tlc_one<16, OUT>(P, f);
+        case 32: return prep_tlc_one<32, OUT>(P, f);
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <int EPT>
+cudaError_t prep_tlc_fused_one(HostPlan& P) {
+    const size_t smem = tlc_smem(P, 0);
+    cudaError_t e = set_smem(fused_tlc_kernel<EPT>, smem);
+    if (e != cudaSuccess) return e;
+    int nb = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fused_tlc_kernel<EPT>, 64 + kTlcPerm, smem);
+    if (e != cudaSuccess) return e;
+    if (nb < 1) return cudaErrorInvalidConfiguration;
+    P.fused3_grid = sm_count();      // one co-resident CTA per SM (grid barriers)
+    return cudaSuccess;
+}
+
+cudaError_t prep_tlc(HostPlan& P) {
+    if (P.fused3) {
+        switch (P.tp[0].ept) {
+            case 8: return prep_tlc_fused_one<8>(P);
+            case 16: return prep_tlc_fused_one<16>(P);
+            case 32: return prep_tlc_fused_one<32>(P);
+        }
+        return cudaErrorInvalidValue;
+    }
+    cudaError_t e = cudaSuccess;
+    for (int f = 0; f < 3 && e == cudaSuccess; ++f) {
+        switch (P.tp[f].out_kind) {
+            case 0: e = prep_tlc_out<0>(P, f); break;
+            case 1: e = prep_tlc_out<1>(P, f); break;
+            case 2: e = prep_tlc_out<2>(P, f); break;
+            default: return cudaErrorInvalidValue;
+        }
+    }
+    return e;
+}
+
 }  // namespace
 
+cudaError_t make_tlc_maps(const HostPlan& P, uint32_t* x1, uint32_t* x2, CUtensorMap* maps) {
+    static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+    if (!encode) {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+        if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn) return cudaErrorNotSupported;
+        encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+    }
+    const cuuint64_t r = (cuuint64_t)P.r, c = (cuuint64_t)P.c;
+    const cuuint64_t h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
+    std::memset(maps, 0, 3 * sizeof(CUtensorMap));
+    {   // X1 = [K][i][k_in]: dims (k_in, i, K)
+        const cuuint64_t dims[3] = {h2, r, c / h2};
+        const cuuint64_t strides[2] = {h2 * 4, r * h2 * 4};
+        const cuuint32_t box[3] = {(cuuint32_t)h2, (cuuint32_t)h1,
+                                   (cuuint32_t)std::min<cuuint64_t>(256, c / h2)};
+        const cuuint32_t es[3] = {1, 1, 1};
+        if (encode(&maps[0], CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, x1, dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return cudaErrorInvalidValue;
+    }
+    {   // X2 = [I'][K][i_in'][k_in]: dims (k_in, i_in', K, I')
+        const cuuint64_t dims[4] = {h2, h3, c / h2, r / h3};
+        const cuuint64_t strides[3] = {h2 * 4, h3 * h2 * 4, c * h3 * 4};
+        const cuuint32_t box[4] = {(cuuint32_t)h2, (cuuint32_t)h3, 1,
+                                   (cuuint32_t)std::min<cuuint64_t>(256, r / h3)};
+        const cuuint32_t es[4] = {1, 1, 1, 1};
+        if (encode(&maps[1], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, x2, dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return cudaErrorInvalidValue;
+    }
+    return cudaSuccess;
+}
+
+cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, const uint32_t* sched,
+                            const uint32_t* in, uint32_t* out, cudaStream_t s, bool pdl,
+                            unsigned long long* trace) {
+    const TlcPass& tp = P.tp[f];
+    TlcArgs ta{};
+    ta.in = in;
+    ta.out = out;
+    ta.sched = sched;
+    ta.ntiles = (int)tp.ntiles;
+    ta.stages = tp.stages;
+    ta.tile_words = tp.tile_words;
+    ta.t_h = tp.h;
+    ta.trace = trace;
+    const long long h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
+    if (tp.out_kind == 1) {
+        const long long outer = P.c / h2, bo = outer < 256 ? outer : 256;
+        ta.box_outer = (int)bo;
+        ta.nbox = (int)(outer / bo);
+        ta.box_words = (int)(bo * h1 * h2);
+    } else if (tp.out_kind == 2) {
+        const long long outer = P.r / h3, bo = outer < 256 ? outer : 256;
+        ta.box_outer = (int)bo;
+        ta.nbox = (int)(outer / bo);
+        ta.box_words = (int)(bo * h3 * h2);
+    }
+    const CUtensorMap& map = maps[tp.out_kind == 2 ? 1 : 0];
+    const dim3 grid((unsigned)tp.grid), block(64 + kTlcPerm);
+    const size_t smem = tlc_smem(P, f);
+#define PERM_TLC_CASE(E_)                                                                             \
+    case E_:                                                                                          \
+        if (tp.out_kind == 0) return launch(row_pass_tlc_kernel<E_, 0>, grid, block, smem, s, pdl, map, ta); \
+        if (tp.out_kind == 1) return launch(row_pass_tlc_kernel<E_, 1>, grid, block, smem, s, pdl, map, ta); \
+        return launch(row_pass_tlc_kernel<E_, 2>, grid, block, smem, s, pdl, map, ta);
+    switch (tp.ept) {
+        PERM_TLC_CASE(8)
+        PERM_TLC_CASE(16)
+        PERM_TLC_CASE(32)
+    }
+#undef PERM_TLC_CASE
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const uint32_t* const sched[3],
+                             const uint32_t* a, uint32_t* x1, uint32_t* x2, uint32_t* b,
+                             unsigned long long* sync, cudaStream_t s, unsigned long long* trace) {
+    TlcFusedArgs fa{};
+    const uint32_t* ins[3] = {a, x1, x2};
+    uint32_t* outs[3] = {x1, x2, b};
+    const long long h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
+    for (int f = 0; f < 3; ++f) {
+        const TlcPass& tp = P.tp[f];
+        TlcPassCfg& pc = fa.p[f];
+        pc.in = ins[f];
+        pc.out = outs[f];
+        pc.sched = sched[f];
+        pc.ntiles = (int)tp.ntiles;
+        pc.kind = tp.out_kind;
+        pc.t_h = tp.h;
+        if (tp.out_kind == 1) {
+            const long long outer = P.c / h2, bo = outer < 256 ? outer : 256;
+            pc.box_outer = (int)bo;
+            pc.nbox = (int)(outer / bo);
+            pc.box_words = (int)(bo * h1 * h2);
+        } else if (tp.out_kind == 2) {
+            const long long outer = P.r / h3, bo = outer < 256 ? outer : 256;
+            pc.box_outer = (int)bo;
+            pc.nbox = (int)(outer / bo);
+            pc.box_words = (int)(bo * h3 * h2);
+        }
+    }
+    fa.tile_words = P.tp[0].tile_words;
+    fa.stages = P.tp[0].stages;
+    fa.sync = sync;
+    fa.trace = trace;
+    const dim3 grid((unsigned)P.fused3_grid), block(64 + kTlcPerm);
+    const size_t smem = tlc_smem(P, 0);
+    switch (P.tp[0].ept) {
+        case 8: return launch(fused_tlc_kernel<8>, grid, block, smem, s, false, maps[0], maps[1], fa);
+        case 16: return launch(fused_tlc_kernel<16>, grid, block, smem, s, false, maps[0], maps[1], fa);
+        case 32: return launch(fused_tlc_kernel<32>, grid, block, smem, s, false, maps[0], maps[1], fa);
+    }
+    return cudaErrorInvalidValue;
+}
+
 cudaError_t prepare_kernels(HostPlan& P) {
+    if (P.layout == 3) return prep_tlc(P);
     cudaError_t e = cudaSuccess;
     auto set = [&](const void* k, size_t bytes) {
         if (e == cudaSuccess)

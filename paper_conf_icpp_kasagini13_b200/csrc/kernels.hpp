@@ -1,6 +1,7 @@
 // kernels.hpp — launchers of the sm_100a kernels (libperm internals).
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -27,6 +28,19 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
 cudaError_t launch_fused3(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
                           uint32_t* x1, uint32_t* x2, uint32_t* b, unsigned long long* sync,
                           cudaStream_t s, unsigned long long* trace = nullptr);
+
+// TLC layout: tensor maps of the intermediates (maps[0]: X1 for pass 1's 3-D
+// stores, maps[1]: X2 for pass 2's 4-D stores) and one pass launch.
+cudaError_t make_tlc_maps(const HostPlan& P, uint32_t* x1, uint32_t* x2, CUtensorMap* maps);
+cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, const uint32_t* sched,
+                            const uint32_t* in, uint32_t* out, cudaStream_t s, bool pdl,
+                            unsigned long long* trace = nullptr);
+
+// TLC layout, square views: the three passes in one persistent launch.
+cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const uint32_t* const sched[3],
+                             const uint32_t* a, uint32_t* x1, uint32_t* x2, uint32_t* b,
+                             unsigned long long* sync, cudaStream_t s,
+                             unsigned long long* trace = nullptr);
 
 // out (cols x rows) = transpose of in (rows x cols), 32 x 32 tiles (§V).
 cudaError_t launch_transpose(const uint32_t* in, uint32_t* out, int64_t rows, int64_t cols,

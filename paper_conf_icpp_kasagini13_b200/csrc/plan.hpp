@@ -60,6 +60,32 @@ struct RowPass {
     int32_t conflicts_in = 1, conflicts_out = 1;   // simulated wavefronts per request
 };
 
+// Tile-level-coloured pass (layout TLC): a tile of h lines is loaded by TMA into
+// buffer A in its global order, permuted out of place into buffer B laid out
+// in the global order of the pass's OUTPUT, and stored by TMA. The bank graph
+// of the whole tile (edge (src mod 32, dst mod 32) per element, src/dst = word
+// offsets in A/B) is (HL/32)-regular; its König colouring gives warp-rounds
+// that read 32 distinct banks of A and write 32 distinct banks of B, whatever
+// the two layouts are. Entry (lane x = src bank, round q) = ((src >> 5) <<
+// logHL) | dst, E = 2*logHL - 5 bits. Permuter warp pw owns rounds
+// [pw*ept, (pw+1)*ept); each lane keeps its ept entries as one bitstream of
+// nwords u32 words; word w of lane x of (tile T, warp pw) is stored at
+// ((T*NW + pw)*nwords + w)*32 + x (coalesced loads).
+constexpr int kTlcPerm = 512;           // permuter threads per CTA
+
+struct TlcPass {
+    int32_t h = 0;            // lines per tile
+    int32_t HL = 0, logHL = 0;
+    int32_t E = 0;
+    int32_t ept = 0;          // HL / kTlcPerm
+    int32_t nwords = 0;       // ceil(ept * E / 32)
+    int64_t ntiles = 0;
+    int64_t tile_words = 0;   // (kTlcPerm / 32) * nwords * 32
+    int32_t out_kind = 0;     // 0: rows (1-D bulk store); 1: X1 3-D tensor store; 2: X2 4-D tensor store
+    int32_t stages = 0;
+    int64_t grid = 0;         // persistent CTAs (set at upload)
+};
+
 struct HostPlan {
     int64_t n = 0;
     int32_t eb = 4;
@@ -68,6 +94,7 @@ struct HostPlan {
     int32_t passes = 0;        // 1, 3, 5
     int32_t layout = 0;        // 3-pass intermediates: 1 tiled, 2 lines (perm_layout)
     int32_t fused3 = 0;        // LINES layout, square view: all three passes in one launch
+    TlcPass tp[3];             // layout TLC (3): the three passes
     int64_t fused3_grid = 0;   // one CTA per SM (set at upload)
     PhaseGeom ph[3];
     RowPass rp[3];
@@ -101,6 +128,17 @@ inline uint32_t unpack_entry(const std::vector<uint32_t>& words, const PhaseGeom
     entry_pos(g, line, q, w, bit);
     const uint64_t v = (uint64_t)words[2 * w] | ((uint64_t)words[2 * w + 1] << 32);
     return (uint32_t)((v >> bit) & ((1ull << g.E) - 1));
+}
+
+// Entry of (tile T, warp-round q, lane x) of a TLC pass.
+inline uint32_t tlc_entry(const std::vector<uint32_t>& words, const TlcPass& tp, int64_t T,
+                          int64_t q, int64_t x) {
+    const int64_t pw = q / tp.ept, m = q % tp.ept;
+    const int64_t bit = m * tp.E, w = bit >> 5, off = bit & 31;
+    const uint32_t* base = words.data() + T * tp.tile_words + pw * tp.nwords * 32 + x;
+    uint64_t v = base[w * 32];
+    if (off + tp.E > 32) v |= (uint64_t)base[(w + 1) * 32] << 32;
+    return (uint32_t)((v >> off) & ((1ull << tp.E) - 1));
 }
 
 // Simulated shared-memory wavefronts per warp request of a pass's load/store

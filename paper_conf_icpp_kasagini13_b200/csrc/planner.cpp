@@ -249,6 +249,113 @@ IoMode cross(int64_t blockP, int64_t strideP, int64_t cta_stride) {
 
 }  // namespace
 
+// ------------------------------------------------------------------ TLC layout
+
+// Word offsets of the element (line, position) of tile T in the A / B buffers of
+// each TLC pass (see plan.hpp and DESIGN.md §5):
+//   X1 = [K][i][k_in] (K < c/h2, i < r, k_in < h2)   X2 = [I'][K][i_in'][k_in]
+//   pass 1: src = i_in*c + j,                     dst = ((k/h2)*h1 + i_in)*h2 + k%h2
+//   pass 2: src = i*h2 + k_in,                    dst = i'*h2 + k_in
+//   pass 3: src = ((k/h2)*h3 + i_in)*h2 + k%h2,   dst = i_in*c + k'
+int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_options* opt,
+              std::string& err) {
+    const int64_t r = P.r, c = P.c;
+    P.layout = 3;
+    const int stages_opt = (opt && opt->stages > 0) ? opt->stages : 0;
+    int64_t hs[3];
+    for (int f = 0; f < 3; ++f) {
+        const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
+        int64_t h = (opt && (&opt->h1)[f] > 0) ? (&opt->h1)[f]
+                                                : std::max<int64_t>(4, 8192 / L);
+        h = std::min(h, lines_f);
+        if (h < 4 || (h & (h - 1)) || lines_f % h) { err = "TLC layout: h must be a power of two >= 4"; return PERM_EINVAL; }
+        hs[f] = h;
+    }
+    const int64_t h1 = hs[0], h2 = hs[1], h3 = hs[2];
+    for (int f = 0; f < 3; ++f) {
+        TlcPass& tp = P.tp[f];
+        tp.h = (int32_t)hs[f];
+        tp.HL = (int32_t)(hs[f] * P.ph[f].L);
+        tp.logHL = ilog2(tp.HL);
+        tp.E = 2 * tp.logHL - 5;
+        tp.ept = tp.HL / kTlcPerm;
+        if (tp.ept != 8 && tp.ept != 16 && tp.ept != 32) {
+            err = "TLC layout: tile must hold 4096, 8192 or 16384 elements (h * L)";
+            return PERM_EINVAL;
+        }
+        tp.nwords = (tp.ept * tp.E + 31) / 32;
+        tp.ntiles = P.ph[f].lines / hs[f];
+        tp.tile_words = (int64_t)(kTlcPerm / 32) * tp.nwords * 32;
+        tp.out_kind = f == 0 ? 1 : (f == 1 ? 2 : 0);
+        const int64_t stage = 2 * (int64_t)tp.HL * 4;
+        int st = stages_opt ? stages_opt : (int)std::min<int64_t>(4, (220 * 1024) / stage);
+        if (st < 1 || st * stage > 220 * 1024) { err = "TLC layout: stages do not fit in shared memory"; return PERM_EINVAL; }
+        tp.stages = st;
+        // keep the generic RowPass view consistent for info/describe
+        RowPass& rp = P.rp[f];
+        rp.phase = f; rp.h = tp.h; rp.ctas = tp.ntiles; rp.tma = 3; rp.stages = st;
+        rp.ept = tp.ept; rp.threads = 64 + kTlcPerm; rp.Ls = P.ph[f].L;
+    }
+    // TMA tensor stores need 16-byte rows: h2 * 4 >= 16 (h2 >= 4 holds)
+    const int64_t NW = kTlcPerm / 32;
+    for (int f = 0; f < 3; ++f) {
+        const TlcPass& tp = P.tp[f];
+        P.sched[f].assign((size_t)(tp.ntiles * tp.tile_words), 0u);
+        uint32_t* W = P.sched[f].data();
+        const uint16_t* ph = phi[f].data();
+        const int64_t HL = tp.HL, h = tp.h;
+        const int E = tp.E, ept = tp.ept, logHL = tp.logHL, nwords = tp.nwords;
+#pragma omp parallel
+        {
+            EulerColourer ec;
+            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL);
+#pragma omp for schedule(dynamic, 1)
+            for (int64_t T = 0; T < tp.ntiles; ++T) {
+                int64_t e = 0;
+                if (f == 0) {
+                    for (int64_t i_in = 0; i_in < h; ++i_in)
+                        for (int64_t j = 0; j < c; ++j, ++e) {
+                            const int64_t kk = ph[(T * h + i_in) * c + j];
+                            src[e] = (uint32_t)(i_in * c + j);
+                            dst[e] = (uint32_t)(((kk / h2) * h1 + i_in) * h2 + kk % h2);
+                        }
+                } else if (f == 1) {
+                    for (int64_t k_in = 0; k_in < h; ++k_in)
+                        for (int64_t i = 0; i < r; ++i, ++e) {
+                            const int64_t ip = ph[(T * h + k_in) * r + i];
+                            src[e] = (uint32_t)(i * h2 + k_in);
+                            dst[e] = (uint32_t)(ip * h2 + k_in);
+                        }
+                } else {
+                    for (int64_t i_in = 0; i_in < h; ++i_in)
+                        for (int64_t kk = 0; kk < c; ++kk, ++e) {
+                            const int64_t kp = ph[(T * h + i_in) * c + kk];
+                            src[e] = (uint32_t)(((kk / h2) * h3 + i_in) * h2 + kk % h2);
+                            dst[e] = (uint32_t)(i_in * c + kp);
+                        }
+                }
+                for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
+                ec.run(kW, HL / kW, HL, U.data(), V.data(), col.data(), false);
+                uint32_t* Wt = W + T * tp.tile_words;
+                for (int64_t x = 0; x < HL; ++x) {
+                    const int64_t q = col[x];                 // warp-round
+                    const int64_t lane = src[x] & 31;         // lane = source bank
+                    const int64_t pw = q / ept, m = q % ept;
+                    const uint64_t entry = ((uint64_t)(src[x] >> 5) << logHL) | dst[x];
+                    const int64_t bit = m * E;
+                    const int64_t w = bit >> 5, off = bit & 31;
+                    const uint64_t sh = entry << off;
+                    uint32_t* base = Wt + (pw * nwords) * 32 + lane;
+                    base[w * 32] |= (uint32_t)sh;
+                    if (off + E > 32) base[(w + 1) * 32] |= (uint32_t)(sh >> 32);
+                }
+            }
+        }
+    }
+    (void)NW;
+    return PERM_OK;
+}
+
 int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
                     HostPlan& P, std::string& err) {
     if (!p || n <= 0) { err = "null p or n <= 0"; return PERM_EINVAL; }
@@ -314,7 +421,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         phi[1][(int64_t)kk * r + i] = (uint16_t)drow;           // Phi2_k(i) = P(x) div c
         phi[2][(int64_t)drow * c + kk] = (uint16_t)dcol;        // Phi3_i'(k) = P(x) mod c
     }
-    // 5-6. bank-level colouring of every line, packed
+    // geometry of the three phases
     const int64_t lines[3] = {r, c, r};
     const int64_t Ls[3] = {c, r, c};
     const int logLs[3] = {logc, logr, logc};
@@ -327,36 +434,41 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.epw = 64 / g.E;
         g.w64 = (kW + g.epw - 1) / g.epw;
         g.words = g.lines * (g.L / kW) * g.w64 * 2;
-        P.sched[f].assign((size_t)g.words, 0u);
-        const int64_t L = g.L;
-        const uint16_t* ph = phi[f].data();
-        uint32_t* W = P.sched[f].data();
+    }
+    // 5-6. bank-level colouring of every line, packed (W64); not needed by TLC plans
+    auto build_line_schedules = [&]() {
+        for (int f = 0; f < 3; ++f) {
+            PhaseGeom& g = P.ph[f];
+            P.sched[f].assign((size_t)g.words, 0u);
+            const int64_t L = g.L;
+            const uint16_t* ph = phi[f].data();
+            uint32_t* W = P.sched[f].data();
 #pragma omp parallel
-        {
-            EulerColourer ec;
-            std::vector<uint32_t> U((size_t)L), V((size_t)L), col((size_t)L);
+            {
+                EulerColourer ec;
+                std::vector<uint32_t> U((size_t)L), V((size_t)L), col((size_t)L);
 #pragma omp for schedule(dynamic, 16)
-            for (int64_t line = 0; line < g.lines; ++line) {
-                const uint16_t* phl = ph + line * L;
-                for (int64_t j = 0; j < L; ++j) {
-                    U[j] = (uint32_t)(j & 31);
-                    V[j] = (uint32_t)(phl[j] & 31);
-                }
-                ec.run(kW, L / kW, L, U.data(), V.data(), col.data(), false);
-                for (int64_t j = 0; j < L; ++j) {
-                    const uint64_t sigma = (uint64_t)(j >> 5);
-                    const uint64_t entry = (sigma << g.logL) | phl[j];
-                    int64_t w;
-                    int bit;
-                    entry_pos(g, line, (int64_t)col[j] * kW + (j & 31), w, bit);
-                    const uint64_t sh = entry << bit;
-                    W[2 * w] |= (uint32_t)sh;
-                    W[2 * w + 1] |= (uint32_t)(sh >> 32);
+                for (int64_t line = 0; line < g.lines; ++line) {
+                    const uint16_t* phl = ph + line * L;
+                    for (int64_t j = 0; j < L; ++j) {
+                        U[j] = (uint32_t)(j & 31);
+                        V[j] = (uint32_t)(phl[j] & 31);
+                    }
+                    ec.run(kW, L / kW, L, U.data(), V.data(), col.data(), false);
+                    for (int64_t j = 0; j < L; ++j) {
+                        const uint64_t sigma = (uint64_t)(j >> 5);
+                        const uint64_t entry = (sigma << g.logL) | phl[j];
+                        int64_t w;
+                        int bit;
+                        entry_pos(g, line, (int64_t)col[j] * kW + (j & 31), w, bit);
+                        const uint64_t sh = entry << bit;
+                        W[2 * w] |= (uint32_t)sh;
+                        W[2 * w + 1] |= (uint32_t)(sh >> 32);
+                    }
                 }
             }
         }
-    }
-    P.ms_bank = ms_since(t0);
+    };
 
     // pass structure
     int passes = opt ? opt->passes : 0;
@@ -369,8 +481,25 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         P.fused_ept = (int32_t)(n / P.fused_threads);
         P.fused_Ls = (int32_t)(c + 1);   // odd stride: rows AND columns conflict-free (Fig. 4 idea)
         if (r * P.fused_Ls > 65535) { err = "fused tile exceeds 16-bit shared addresses"; return PERM_EUNSUPPORTED; }
+        build_line_schedules();
+        P.ms_bank = ms_since(t0);
         return PERM_OK;
     }
+    {
+        int layout0 = opt ? opt->layout : 0;
+        if (passes == 3 && (layout0 == 3 || (layout0 == 0 && k >= 15 && k <= 22))) {
+            const int st = build_tlc(P, phi, opt, err);
+            P.ms_bank = ms_since(t0);
+            // one persistent launch when the three passes share the tile size (square view)
+            const int fuse = opt ? opt->fuse : 0;
+            if (st == PERM_OK && fuse >= 0 && P.tp[0].HL == P.tp[1].HL && P.tp[1].HL == P.tp[2].HL &&
+                P.tp[0].stages == P.tp[1].stages && P.tp[1].stages == P.tp[2].stages)
+                P.fused3 = 1;
+            return st;
+        }
+    }
+    build_line_schedules();
+    P.ms_bank = ms_since(t0);
     const int64_t Q = std::min<int64_t>(16384, std::max<int64_t>(2048, pow2_floor(n / 296)));
     auto pick = [&](int idx, int64_t dflt) -> int64_t {
         int64_t v = opt ? (&opt->h1)[idx] : 0;

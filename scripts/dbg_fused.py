@@ -6,7 +6,7 @@ from oracle import apply as OA
 for k in (18, 20, 22):
     n = 1 << k
     p = W.random(n, k); a = W.make_data(n); ref = OA.apply_ref(p, a)
-    for cfg in ({'h': (8, 8, 8), 'stages': 2}, {'h': (8, 8, 8), 'stages': 2, 'fuse': -1}, {}):
+    for cfg in ({'layout': 2, 'h': (8, 8, 8), 'stages': 2, 'fuse': 1}, {'fuse': -1}, {}, {'layout': 3, 'stages': 1}, {'layout': 3, 'stages': 1, 'fuse': -1}):
         pl = P.Plan(p, **cfg)
         d = pl.describe()
         da = torch.from_numpy(a.view(np.int32)).cuda(); db = torch.full_like(da, -1)

@@ -37,6 +37,8 @@ if d.get('fused3'):
         if v.size:
             print(f"  {fn[c]:>12}: min {v.min():7.2f}  med {np.median(v):7.2f}  max {v.max():7.2f}  (n={v.size})")
     sys.exit(0)
+if d.get('layout') == 3:
+    names = {0: 'start', 1: 'pdl_ok', 2: 'w0', 4: 's0', 5: 'w1', 7: 's1', 8: 'w2', 10: 's2', 3: 'permEnd', 14: 'end'}
 for f in range(3):
     t = tr[f]
     t = t[(t[:, 0] > 0)]

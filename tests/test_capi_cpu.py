@@ -63,7 +63,7 @@ def export_plan(lib, p, **kw):
 def test_cpp_plan_passes_oracle_checker(lib, fam, k):
     n = 1 << k
     p = W.make_perm(fam, n, seed=42 + k)
-    info, kappa, sched = export_plan(lib, p)
+    info, kappa, sched = export_plan(lib, p, layout=2 if k >= 15 else 0)   # per-line schedules
     r, c = W.view_shape(n)
     assert (info["rows"], info["cols"]) == (r, c)
     OC.assert_plan(p, kappa, sched, r, c, 32)
@@ -93,7 +93,7 @@ def test_cpp_plan_larger(lib, k):
     r, c = W.view_shape(n)
     for fam in ("random", "bitrev"):
         p = W.make_perm(fam, n)
-        _, kappa, sched = export_plan(lib, p)
+        _, kappa, sched = export_plan(lib, p, layout=2)
         OC.assert_plan(p, kappa, sched, r, c, 32)
 
 
@@ -101,7 +101,7 @@ def test_cpp_plan_22_random(lib):
     n = 1 << 22
     r, c = W.view_shape(n)
     p = W.random(n, 42)
-    info, kappa, sched = export_plan(lib, p)
+    info, kappa, sched = export_plan(lib, p, layout=2)
     OC.assert_plan(p, kappa, sched, r, c, 32)
     assert info["passes"] == 3
     # W64 schedule: 17-bit entries, 3 per 64-bit word, 11 words per warp-round of 32
@@ -116,10 +116,10 @@ def test_pass_options_and_info(lib):
         with lib.Plan(p, device=False, passes=passes) as pl:
             info = pl.info()
             assert info["passes"] == passes
-            assert info["kernels_per_apply"] == passes
+            assert info["kernels_per_apply"] in (1, passes)   # 1 = single persistent launch
     with lib.Plan(W.random(1 << 12, 1), device=False) as pl:
         assert pl.info()["passes"] == 1
-    with lib.Plan(p, device=False, passes=3, h=(4, 8, 4)) as pl:
+    with lib.Plan(p, device=False, passes=3, layout=1, h=(4, 8, 4)) as pl:
         assert pl.info()["h"] == [4, 8, 4]
 
 
@@ -160,3 +160,55 @@ def test_bruteforce_tiny_via_cpp_euler_split(lib):
         p[:8] = base[list(perm)]
         _, kappa, sched = export_plan(lib, p)
         OC.assert_plan(p, kappa, sched, r, c, 32)
+
+
+# ---------------------------------------------------------------- TLC plans (layout 3)
+
+def export_tlc(lib, p, **kw):
+    with lib.Plan(p, device=False, passes=3, layout=3, **kw) as pl:
+        info = pl.info()
+        d = pl.describe()
+        kappa, scheds = pl.export()
+    return info, d, kappa.astype(np.int64), [s.reshape(-1) for s in scheds]
+
+
+@pytest.mark.parametrize("fam", W.FAMILIES)
+@pytest.mark.parametrize("k", [16, 17, 18, 20])
+def test_tlc_plan_passes_oracle_checker(lib, fam, k):
+    n = 1 << k
+    r, c = W.view_shape(n)
+    p = W.make_perm(fam, n, seed=k)
+    info, d, kappa, sched = export_tlc(lib, p)
+    h = tuple(info["h"])
+    res = OC.check_tlc(p, kappa, sched, r, c, h)
+    assert all(res.values()), res
+    assert len(res) == 8
+
+
+def test_tlc_plan_22(lib):
+    n = 1 << 22
+    r, c = W.view_shape(n)
+    p = W.random(n, 42)
+    info, d, kappa, sched = export_tlc(lib, p)
+    assert info["h"] == [4, 4, 4] and info["entry_bits"] == [21, 21, 21]
+    res = OC.check_tlc(p, kappa, sched, r, c, (4, 4, 4))
+    assert all(res.values()), res
+
+
+def test_tlc_checker_rejects_corruption(lib):
+    n = 1 << 16
+    r, c = W.view_shape(n)
+    p = W.random(n, 7)
+    info, d, kappa, sched = export_tlc(lib, p)
+    h = tuple(info["h"])
+    assert all(OC.check_tlc(p, kappa, sched, r, c, h).values())
+    bad = [s.copy() for s in sched]
+    # swap the destinations of two slots of one round: still a bijection, wrong mapping
+    bad[1][0], bad[1][1] = (bad[1][0] & 0xFFFF0000) | (bad[1][1] & 0xFFFF), (bad[1][1] & 0xFFFF0000) | (bad[1][0] & 0xFFFF)
+    res = OC.check_tlc(p, kappa, bad, r, c, h)
+    assert not res["v_tiles_implement_phi"]
+    # move a slot's source into another lane's bank
+    bad = [s.copy() for s in sched]
+    bad[2][0] = ((((bad[2][0] >> 16) ^ 1)) << 16) | (bad[2][0] & 0xFFFF)
+    res = OC.check_tlc(p, kappa, bad, r, c, h)
+    assert not (res["viii_lane_is_source_bank"] and res["vii_sources_and_dests_cover_tile"])

@@ -225,8 +225,9 @@ def test_copy_kernel(P):
     assert torch.equal(a, b)
 
 
+@pytest.mark.parametrize("layout", [2, 3])
 @pytest.mark.parametrize("k", [16, 18, 20, 22])
-def test_fused3_first_apply_and_graph_replay(P, k):
+def test_fused3_first_apply_and_graph_replay(P, k, layout):
     # the single-launch 3-pass kernel: grid barriers must hold on the FIRST apply of a
     # fresh plan (intermediates not yet valid), for grids with idle CTAs (few tiles),
     # and across CUDA-graph replays (self-resetting counters)
@@ -234,13 +235,17 @@ def test_fused3_first_apply_and_graph_replay(P, k):
     p = W.random(n, 100 + k)
     a = W.make_data(n)
     ref = OA.apply_ref(p, a)
-    with P.Plan(p, h=(8, 8, 8), fuse=1) as plan:
+    if layout == 2 and k < 18:
+        pytest.skip("LINES single-launch kernel needs tiles of >= 4096 elements")
+    h = (8, 8, 8) if layout == 2 else (0, 0, 0)
+    with P.Plan(p, layout=layout, h=h, fuse=1) as plan:
         info = plan.describe()
         da = dev(a)
         db = torch.full_like(da, -1)
         plan.apply(da, db)
         torch.cuda.synchronize()
-        assert np.array_equal(host_words(db), ref), info.get("fused3")
+        assert info.get("fused3") == 1
+        assert np.array_equal(host_words(db), ref)
         s = torch.cuda.Stream()
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
@@ -250,3 +255,15 @@ def test_fused3_first_apply_and_graph_replay(P, k):
             g.replay()
             torch.cuda.synchronize()
             assert np.array_equal(host_words(db), ref)
+
+
+@pytest.mark.parametrize("layout", [1, 2, 3])
+@pytest.mark.parametrize("k", [16, 19, 20, 22])
+def test_every_layout(P, layout, k):
+    n = 1 << k
+    p = W.random(n, 300 + k)
+    a = W.make_data(n)
+    ref = OA.apply_ref(p, a)
+    for fam_p in (p, W.bitrev(n)):
+        b, info = run(P, fam_p, a, passes=3, layout=layout)
+        assert np.array_equal(b, OA.apply_ref(fam_p, a)), (layout, k)
