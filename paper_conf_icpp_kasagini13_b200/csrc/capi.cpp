@@ -215,6 +215,19 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
     std::string s = "{\"n\":" + std::to_string(P.n) + ",\"rows\":" + std::to_string(P.r) +
                     ",\"cols\":" + std::to_string(P.c) + ",\"passes\":" + std::to_string(P.passes) +
                     ",\"layout\":" + std::to_string(P.layout) + ",\"fused3\":" + std::to_string(P.fused3);
+    if (P.layout == 3) {
+        s += ",\"tlc\":[";
+        for (int f = 0; f < 3; ++f) {
+            const perm::TlcPass& tp = P.tp[f];
+            s += std::string(f ? "," : "") + "{\"h\":" + std::to_string(tp.h) + ",\"HL\":" +
+                 std::to_string(tp.HL) + ",\"E\":" + std::to_string(tp.E) + ",\"ept\":" +
+                 std::to_string(tp.ept) + ",\"nwords\":" + std::to_string(tp.nwords) +
+                 ",\"ntiles\":" + std::to_string(tp.ntiles) + ",\"stages\":" +
+                 std::to_string(tp.stages) + ",\"grid\":" + std::to_string(tp.grid) +
+                 ",\"out_kind\":" + std::to_string(tp.out_kind) + "}";
+        }
+        s += "]";
+    }
     if (P.passes == 1) {
         s += ",\"fused\":{\"threads\":" + std::to_string(P.fused_threads) + ",\"ept\":" +
              std::to_string(P.fused_ept) + ",\"Ls\":" + std::to_string(P.fused_Ls) + "}";

@@ -472,7 +472,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 
     // pass structure
     int passes = opt ? opt->passes : 0;
-    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 26 ? 3 : 5);
+    // measured on B200: fused CTA to 2^14, TLC 3-pass 2^15..2^22, LINES
+    // 3-pass 2^23..2^24, the paper's 5-pass structure (TMA row passes) from 2^25
+    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 24 ? 3 : 5);
     if (passes == 1 && k > 14) { err = "fused single-CTA pass needs n <= 2^14"; return PERM_EUNSUPPORTED; }
     if (passes != 1 && passes != 3 && passes != 5) { err = "passes must be 0, 1, 3 or 5"; return PERM_EINVAL; }
     P.passes = passes;
@@ -492,7 +494,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             P.ms_bank = ms_since(t0);
             // one persistent launch when the three passes share the tile size (square view)
             const int fuse = opt ? opt->fuse : 0;
-            if (st == PERM_OK && fuse >= 0 && P.tp[0].HL == P.tp[1].HL && P.tp[1].HL == P.tp[2].HL &&
+            if (st == PERM_OK && fuse > 0 && P.tp[0].HL == P.tp[1].HL && P.tp[1].HL == P.tp[2].HL &&
                 P.tp[0].stages == P.tp[1].stages && P.tp[1].stages == P.tp[2].stages)
                 P.fused3 = 1;
             return st;

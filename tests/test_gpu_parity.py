@@ -147,7 +147,9 @@ def test_config2_2pow26_random(P):
     p = W.random(n, 42)
     a = W.make_data(n)
     b, info = run(P, p, a)
-    assert info["passes"] == 3
+    assert info["passes"] == 5
+    assert np.array_equal(b, OA.apply_ref(p, a))
+    b, info = run(P, p, a, passes=3)
     assert np.array_equal(b, OA.apply_ref(p, a))
 
 
