@@ -190,6 +190,85 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def run_sharded(args, rank, world, local):
+    """N > 1: the row-sharded path on n = 2^log2n * N elements (each GPU
+    holds a 2^log2n shard: weak scaling). Rows stay local for phases 1 and 3; the
+    column phase runs as two NCCL all-to-all exchanges (torch.distributed, NVLink)."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_kasagini13_b200 as pkg
+    from paper_conf_icpp_kasagini13_b200.sharded import ShardedApply
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    ntot = (1 << args.log2n) * world
+    shard = ntot // world
+    fams = args.families.split(",")
+    flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+    runs, bufs, build_ms = {}, {}, {}
+    for f in fams:
+        p = W.make_perm(f, ntot)
+        a = W.make_data(ntot)
+        t0 = time.perf_counter()
+        pl = pkg.Plan(p, world=world, rank=rank)
+        build_ms[f] = (time.perf_counter() - t0) * 1e3
+        a_sh = torch.from_numpy(a[rank * shard:(rank + 1) * shard].view(np.int32).copy()).to(dev)
+        bufs[f] = (pl, a_sh, torch.empty_like(a_sh), torch.empty_like(a_sh), torch.empty_like(a_sh),
+                   p[rank * shard:(rank + 1) * shard], a)
+        runs[f] = ShardedApply(pl)
+    def one(f):
+        pl, a_sh, b_sh, send, recv = bufs[f][:5]
+        runs[f](a_sh, b_sh, send, recv, stream)
+    for _ in range(max(args.warmup, 3)):
+        for f in fams:
+            one(f)
+    torch.cuda.synchronize()
+    # bit-exactness of this rank's shard for the last family (oracle on the host)
+    from oracle import apply as OA
+    f = fams[-1]
+    ref = OA.apply_ref(W.make_perm(f, ntot), bufs[f][6])[rank * shard:(rank + 1) * shard]
+    ok = bool(np.array_equal(bufs[f][2].cpu().numpy().view(np.uint32), ref))
+    evs = {f: [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)] for f in fams}
+    dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clocks:
+        for s in range(args.steps):
+            for f in fams:
+                flush.zero_()
+                flush.sum()
+                dist.barrier()
+                evs[f][s][0].record(stream)
+                one(f)
+                evs[f][s][1].record(stream)
+        torch.cuda.synchronize()
+    dist.barrier()
+    step_ms = [sum(evs[f][s][0].elapsed_time(evs[f][s][1]) for f in fams) for s in range(args.steps)]
+    t = torch.tensor([statistics.mean(step_ms)], device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    okt = torch.tensor([1 if ok else 0], device=dev)
+    dist.all_reduce(okt, op=dist.ReduceOp.MIN)
+    ms_per_step = float(t.item())
+    value = len(fams) * 2 * ntot * 4 / (ms_per_step * 1e-3) / 1e9
+    if rank == 0:
+        cfg = workload_config(args)
+        cfg["workload"] = (f"row-sharded n=2^{args.log2n}*{world} float32 (raw u32 words), one "
+                           f"2^{args.log2n} shard per GPU, families {'/'.join(fams)}, NCCL all-to-all")
+        cfg["n"] = ntot
+        cfg["parallelism"] = f"row-sharded x{world} (NCCL all_to_all_single, 2 exchanges per apply)"
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": cfg, "bitexact_check_all_ranks": bool(okt.item()),
+                "plan_build_ms_rank0": build_ms,
+                "exchange_bytes_per_apply_per_gpu": 2 * (world - 1) * (ntot // (world * world)) * 4,
+                "gpu_launches": args.steps * len(fams) * 5,
+                "clocks": clocks.summary()}
+        print(json.dumps(line), flush=True)
+    for f in fams:
+        bufs[f][0].close()
+    dist.destroy_process_group()
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -201,6 +280,7 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        return run_sharded(args, rank, world, local)
     import paper_conf_icpp_kasagini13_b200 as pkg
 
     n = 1 << args.log2n

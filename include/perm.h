@@ -88,6 +88,9 @@ typedef struct {
     double  build_ms_colour;     /* row-level König colouring (Euler split) */
     double  build_ms_bank;       /* per-line bank-level colourings + packing */
     double  build_ms_upload;     /* device allocation + host->device copy */
+    int32_t world, rank;         /* row sharding (1, 0 for unsharded plans) */
+    int64_t shard_elems;         /* n / world */
+    int64_t block_elems;         /* n / world^2: one all-to-all block */
 } perm_plan_info;
 
 /* ------------------------------------------------------------------ plans */
@@ -160,6 +163,31 @@ int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k);
  * host memory (synchronous) and returns the number of entries (3*ctas*16). */
 int     perm_plan_set_tracing(perm_plan* plan, int enable);
 int64_t perm_plan_trace(const perm_plan* plan, uint64_t* out, int64_t max_entries);
+
+/* ------------------------------------------------- row-sharded (multi-GPU) */
+
+/* rank g of `world` GPUs owns rows [g*r/world, (g+1)*r/world) of the
+ * r x c view, i.e. the contiguous shard a[g*n/world : (g+1)*n/world] (and the
+ * same shard of b). Phases 1 and 3 (row-wise, L537-L539) are local; the
+ * column-wise phase (Lemma 8: transpose, row-wise, transpose) becomes two
+ * all-to-all exchanges. p is the FULL permutation (every rank passes the same p;
+ * every rank colours it identically and keeps its own lines' schedules).
+ * world must be a power of two with r/world >= 32 and c/world >= 32. */
+perm_plan* perm_plan_create_sharded(const int32_t* p, int64_t n, int32_t elem_bytes,
+                                    int32_t world, int32_t rank, const perm_plan_options* opt);
+perm_plan* perm_plan_create_sharded_host(const int32_t* p, int64_t n, int32_t elem_bytes,
+                                         int32_t world, int32_t rank,
+                                         const perm_plan_options* opt);
+
+/* One local step of a sharded apply (device buffers, stream-ordered):
+ *   step 0: in = a shard (n/world elems)  -> out = send buffer (n/world)  [R1, T]
+ *   step 1: in = recv buffer              -> out = send buffer            [R2, T]
+ *   step 2: in = recv buffer              -> out = b shard                [R3]
+ * Between steps 0->1 and 1->2 the caller performs the all-to-all: with
+ * B = n/world^2, for every pair (g, q): recv_q[g*B : (g+1)*B] = send_g[q*B : (q+1)*B]
+ * (NCCL all_to_all over NVLink, or device copies for ranks sharing one GPU). */
+int perm_sharded_step(const perm_plan* plan, int32_t step, const void* in, void* out,
+                      perm_stream_t stream);
 
 /* ------------------------------------------------------- comparators */
 

@@ -46,7 +46,9 @@ class PlanInfo(ctypes.Structure):
                 ("kernels_per_apply", ctypes.c_int32), ("entry_bits", ctypes.c_int32 * 3),
                 ("h", ctypes.c_int32 * 3), ("planner_threads", ctypes.c_int32),
                 ("build_ms_colour", ctypes.c_double), ("build_ms_bank", ctypes.c_double),
-                ("build_ms_upload", ctypes.c_double)]
+                ("build_ms_upload", ctypes.c_double), ("world", ctypes.c_int32),
+                ("rank", ctypes.c_int32), ("shard_elems", ctypes.c_int64),
+                ("block_elems", ctypes.c_int64)]
 
     def as_dict(self) -> dict:
         d = {}
@@ -69,6 +71,11 @@ def _sig(name, res, *args):
 _plan_create = _sig("perm_plan_create", _vp, _vp, _i64, _i32)
 _plan_create_ex = _sig("perm_plan_create_ex", _vp, _vp, _i64, _i32, ctypes.POINTER(PlanOptions))
 _plan_create_host = _sig("perm_plan_create_host", _vp, _vp, _i64, _i32, ctypes.POINTER(PlanOptions))
+_plan_create_sharded = _sig("perm_plan_create_sharded", _vp, _vp, _i64, _i32, _i32, _i32,
+                            ctypes.POINTER(PlanOptions))
+_plan_create_sharded_host = _sig("perm_plan_create_sharded_host", _vp, _vp, _i64, _i32, _i32, _i32,
+                                 ctypes.POINTER(PlanOptions))
+_sharded_step = _sig("perm_sharded_step", ctypes.c_int, _vp, _i32, _vp, _vp, _vp)
 _plan_destroy = _sig("perm_plan_destroy", None, _vp)
 _plan_get_info = _sig("perm_plan_get_info", ctypes.c_int, _vp, ctypes.POINTER(PlanInfo))
 _plan_describe = _sig("perm_plan_describe", _i64, _vp, ctypes.c_char_p, _i64)
@@ -128,12 +135,17 @@ class Plan:
     """perm_plan: the offline schedule of permutation p (int32, host)."""
 
     def __init__(self, p, elem_bytes: int = 4, passes: int = 0, h=(0, 0, 0),
-                 device: bool = True, layout: int = 0, stages: int = 0, fuse: int = 0):
+                 device: bool = True, layout: int = 0, stages: int = 0, fuse: int = 0,
+                 world: int = 0, rank: int = 0):
+        """world > 0: row-sharded plan of rank `rank` (see perm_plan_create_sharded)."""
         p = _as_int32_host(p)
         self.n = int(p.size)
         self.elem_bytes = elem_bytes
         opt = PlanOptions(passes, h[0], h[1], h[2], layout, stages, fuse)
-        if device:
+        if world > 0:
+            fn = _plan_create_sharded if device else _plan_create_sharded_host
+            handle = fn(p.ctypes.data, self.n, elem_bytes, world, rank, ctypes.byref(opt))
+        elif device:
             handle = _plan_create_ex(p.ctypes.data, self.n, elem_bytes, ctypes.byref(opt))
         else:
             handle = _plan_create_host(p.ctypes.data, self.n, elem_bytes, ctypes.byref(opt))
@@ -179,10 +191,11 @@ class Plan:
         """(kappa[n] uint16, [sched1 (r,c), sched2 (c,r), sched3 (r,c)] uint32 (sigma<<16)|t)."""
         inf = self.info()
         r, c = inf["rows"], inf["cols"]
+        G = inf["world"]
         kappa = np.empty(self.n, dtype=np.uint16)
-        s1 = np.empty((r, c), dtype=np.uint32)
-        s2 = np.empty((c, r), dtype=np.uint32)
-        s3 = np.empty((r, c), dtype=np.uint32)
+        s1 = np.empty((r // G, c), dtype=np.uint32)     # sharded plans: this rank's lines
+        s2 = np.empty((c // G, r), dtype=np.uint32)
+        s3 = np.empty((r // G, c), dtype=np.uint32)
         _check(_plan_export(self._h, kappa.ctypes.data, s1.ctypes.data, s2.ctypes.data,
                             s3.ctypes.data))
         return kappa, [s1, s2, s3]
@@ -197,6 +210,11 @@ class Plan:
         """End-to-end: host a -> device -> apply -> host b (synchronises the stream)."""
         _check(_apply_host(self._h, _ptr(a_host), _ptr(b_host), _stream_handle(stream)))
         return b_host
+
+    def sharded_step(self, step: int, inp, out, stream=None):
+        """One local step of a row-sharded apply (see include/perm.h perm_sharded_step)."""
+        _check(_sharded_step(self._h, step, _ptr(inp), _ptr(out), _stream_handle(stream)))
+        return out
 
     def set_profiling(self, on: bool = True):
         _check(_set_prof(self._h, 1 if on else 0))

@@ -94,7 +94,7 @@ int upload(perm_plan* pl) {
         off += padded(wf);
     }
     if (P.passes != 1) {
-        const size_t bytes = (size_t)P.n * P.eb;
+        const size_t bytes = (size_t)(P.r_l ? P.n / P.world : P.n) * P.eb;
         for (int i = 0; i < 2; ++i) {
             e = cudaMalloc(&pl->d_scratch[i], bytes);
             if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc scratch: ") + cudaGetErrorString(e));
@@ -125,13 +125,14 @@ int upload(perm_plan* pl) {
 }
 
 perm_plan* create(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
-                  bool device) {
+                  bool device, int world = 0, int rank = 0) {
     perm_plan* pl = new (std::nothrow) perm_plan();
     if (!pl) { fail(PERM_ENOMEM, "out of host memory"); return nullptr; }
     std::string err;
     int st;
     try {
-        st = perm::build_host_plan(p, n, eb, opt, pl->host, err);
+        st = world > 0 ? perm::build_sharded_plan(p, n, eb, world, rank, opt, pl->host, err)
+                       : perm::build_host_plan(p, n, eb, opt, pl->host, err);
     } catch (const std::bad_alloc&) {
         st = PERM_ENOMEM;
         err = "out of host memory while planning";
@@ -178,6 +179,45 @@ perm_plan* perm_plan_create_host(const int32_t* p, int64_t n, int32_t elem_bytes
     return create(p, n, elem_bytes, opt, false);
 }
 
+perm_plan* perm_plan_create_sharded(const int32_t* p, int64_t n, int32_t elem_bytes, int32_t world,
+                                    int32_t rank, const perm_plan_options* opt) {
+    return create(p, n, elem_bytes, opt, true, world, rank);
+}
+
+perm_plan* perm_plan_create_sharded_host(const int32_t* p, int64_t n, int32_t elem_bytes,
+                                         int32_t world, int32_t rank, const perm_plan_options* opt) {
+    return create(p, n, elem_bytes, opt, false, world, rank);
+}
+
+int perm_sharded_step(const perm_plan* plan, int32_t step, const void* in, void* out,
+                      perm_stream_t stream) {
+    if (!plan || !in || !out) return fail(PERM_EINVAL, "null plan or buffer");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
+    const HostPlan& P = plan->host;
+    if (!P.r_l) return fail(PERM_EINVAL, "not a row-sharded plan");
+    const int64_t shard = P.n / P.world;
+    if (overlap(in, out, shard * P.eb)) return fail(PERM_EINVAL, "in and out overlap");
+    if ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15)
+        return fail(PERM_EINVAL, "buffers must be 16-byte aligned");
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const uint32_t* src = static_cast<const uint32_t*>(in);
+    uint32_t* dst = static_cast<uint32_t*>(out);
+    cudaError_t e;
+    if (step == 0) {          // R1 on my rows, then T-pack: (r_l x c) -> (c x r_l), peer q = rows q*c_l..
+        e = perm::launch_row_pass(P, 0, plan->d_phase[0], src, plan->d_scratch[0], s, false);
+        if (e == cudaSuccess) e = perm::launch_transpose(plan->d_scratch[0], dst, P.r_l, P.c, s, true);
+    } else if (step == 1) {   // R2 on my columns (segments from every sender), T-pack: (c_l x r) -> (r x c_l)
+        e = perm::launch_row_pass(P, 1, plan->d_phase[1], src, plan->d_scratch[1], s, false);
+        if (e == cudaSuccess) e = perm::launch_transpose(plan->d_scratch[1], dst, P.c_l, P.r, s, true);
+    } else if (step == 2) {   // R3 on my rows (segments from every sender) -> b shard
+        e = perm::launch_row_pass(P, 2, plan->d_phase[2], src, dst, s, false);
+    } else {
+        return fail(PERM_EINVAL, "step must be 0, 1 or 2");
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "sharded step launch");
+    return PERM_OK;
+}
+
 void perm_plan_destroy(perm_plan* plan) {
     if (!plan) return;
     free_device(plan);
@@ -206,6 +246,10 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->build_ms_colour = P.ms_colour;
     out->build_ms_bank = P.ms_bank;
     out->build_ms_upload = plan->ms_upload;
+    out->world = P.r_l ? P.world : 1;
+    out->rank = P.r_l ? P.rank : 0;
+    out->shard_elems = P.r_l ? P.n / P.world : P.n;
+    out->block_elems = P.r_l ? P.n / ((int64_t)P.world * P.world) : P.n;
     return PERM_OK;
 }
 

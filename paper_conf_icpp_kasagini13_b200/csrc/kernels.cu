@@ -232,6 +232,8 @@ struct RowArgs {
     long long sched_words_per_cta;
     Io i, o;
     unsigned long long* trace;   // optional: 16 %globaltimer stamps per CTA (tracing)
+    int in_segs;                 // >1: input line l of tile t = in_segs segments of seg_len
+    long long seg_len, seg_stride;   //     at in + s*seg_stride + (t*h + l)*seg_len
 };
 
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -385,8 +387,16 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
                  (uint32_t)a.sched_words * 4u, &bars[s]);
     };
     auto issue_data = [&](int s, long long t) {
-        const uint32_t* src = a.r.in + t * h * (long long)L;
         uint32_t* dst = smem + s * stage_words;
+        if (a.r.in_segs > 1) {
+            const uint32_t sb = (uint32_t)a.r.seg_len * 4u;
+            for (int l = 0; l < h; ++l)
+                for (int g = 0; g < a.r.in_segs; ++g)
+                    bulk_g2s(dst + l * a.r.Ls + g * a.r.seg_len,
+                             a.r.in + g * a.r.seg_stride + (t * h + l) * a.r.seg_len, sb, &bars[s]);
+            return;
+        }
+        const uint32_t* src = a.r.in + t * h * (long long)L;
         if (dense) {
             bulk_g2s(dst, src, (uint32_t)h * line_bytes, &bars[s]);
         } else {
@@ -1792,6 +1802,9 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
     ra.sched_words_per_cta = (long long)rp.h * (g.L / 32) * g.w64 * 2;
     ra.i = make_io(rp.in);
     ra.o = make_io(rp.out);
+    ra.in_segs = rp.in_segs;
+    ra.seg_len = rp.seg_len;
+    ra.seg_stride = rp.seg_stride;
     const dim3 block(rp.threads);
     if (rp.tma == 2) {
         WsArgs wa{};

@@ -48,6 +48,8 @@ struct IoMode {
 
 struct RowPass {
     int32_t phase = 0;        // 0,1,2 -> Phi1, Phi2, Phi3
+    int32_t in_segs = 1;      // >1: each input line is in_segs segments (sharded column phase)
+    int64_t seg_len = 0, seg_stride = 0;
     int32_t tma = 0;          // 1: persistent TMA-pipelined kernel (contiguous input lines)
     int32_t stages = 0;       // TMA ring depth
     int64_t grid = 0;         // persistent CTAs (set at upload from the occupancy query)
@@ -95,6 +97,10 @@ struct HostPlan {
     int32_t layout = 0;        // 3-pass intermediates: 1 tiled, 2 lines (perm_layout)
     int32_t fused3 = 0;        // LINES layout, square view: all three passes in one launch
     TlcPass tp[3];             // layout TLC (3): the three passes
+    // row-sharded plans: this rank owns rows [rank*r_l, +r_l) of a and b,
+    // and columns [rank*c_l, +c_l) in the column phase; schedules are sliced to those lines
+    int32_t world = 1, rank = 0;
+    int64_t r_l = 0, c_l = 0;
     int64_t fused3_grid = 0;   // one CTA per SM (set at upload)
     PhaseGeom ph[3];
     RowPass rp[3];
@@ -108,6 +114,11 @@ struct HostPlan {
 // Builds everything host-side. Returns PERM_OK or a perm_status, with `err` set.
 int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
                     HostPlan& out, std::string& err);
+
+// Row-sharded plan for `rank` of `world` (world a power of two dividing r and c):
+// the global colouring, then this rank's slices of the three phase schedules.
+int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, int32_t rank,
+                       const perm_plan_options* opt, HostPlan& out, std::string& err);
 
 // Colour a d-regular bipartite multigraph (d a power of two) with d colours by
 // recursive Euler splitting. U[e], V[e] < nodes, E = nodes * d edges.

@@ -638,4 +638,57 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     return PERM_OK;
 }
 
+int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, int32_t rank,
+                       const perm_plan_options* opt, HostPlan& P, std::string& err) {
+    if (world < 1 || (world & (world - 1)) || rank < 0 || rank >= world) {
+        err = "world must be a power of two and 0 <= rank < world";
+        return PERM_EINVAL;
+    }
+    // the global plan with per-line schedules (5-pass geometry: whole lines)
+    perm_plan_options o{};
+    if (opt) o = *opt;
+    o.passes = 5;
+    o.layout = 0;
+    int st = build_host_plan(p, n, eb, &o, P, err);
+    if (st != PERM_OK) return st;
+    const int64_t r = P.r, c = P.c;
+    if (r % world || c % world || r / world < 32 || c / world < 32) {
+        err = "row sharding needs r/world >= 32 and c/world >= 32";
+        return PERM_EUNSUPPORTED;
+    }
+    P.world = world;
+    P.rank = rank;
+    P.r_l = r / world;
+    P.c_l = c / world;
+    const int64_t first[3] = {rank * P.r_l, rank * P.c_l, rank * P.r_l};
+    const int64_t count[3] = {P.r_l, P.c_l, P.r_l};
+    for (int f = 0; f < 3; ++f) {
+        PhaseGeom& g = P.ph[f];
+        const int64_t wpl = (int64_t)(g.L / kW) * g.w64 * 2;     // words per line
+        std::vector<uint32_t> slice(P.sched[f].begin() + first[f] * wpl,
+                                    P.sched[f].begin() + (first[f] + count[f]) * wpl);
+        P.sched[f].swap(slice);
+        g.lines = count[f];
+        g.words = count[f] * wpl;
+        RowPass& rp = P.rp[f];
+        if (count[f] % rp.h) rp.h = (int32_t)std::max<int64_t>(1, count[f]);   // degenerate tiny shards
+        rp.ctas = count[f] / rp.h;
+        rp.in = runs(g.L, 0, (int64_t)rp.h * g.L);
+        rp.out = runs(g.L, 0, (int64_t)rp.h * g.L);
+        if (f == 0) {
+            rp.in_segs = 1;
+        } else {
+            // each line arrives as `world` segments, one per sender, block-strided
+            rp.in_segs = world;
+            rp.seg_len = f == 1 ? P.r_l : P.c_l;
+            rp.seg_stride = P.r_l * P.c_l;
+            if (!rp.tma) {
+                err = "row sharding: lines must fit the TMA pass (L <= 16384)";
+                return PERM_EUNSUPPORTED;
+            }
+        }
+    }
+    return PERM_OK;
+}
+
 }  // namespace perm
