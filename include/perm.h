@@ -71,7 +71,9 @@ typedef struct {
     int32_t fuse;        /* LINES layout, square view: 1 = run the three passes as ONE persistent
                             kernel with grid barriers; 0 = auto (currently three launches
                             chained with programmatic dependent launch); -1 = never */
-    int32_t reserved[5];
+    int32_t no_tma;      /* 1: use the plain (non-TMA) row-pass kernels of the 5-pass / sharded
+                            structures even when a TMA stage fits (testing, A/B comparisons) */
+    int32_t reserved[4];
 } perm_plan_options;
 
 typedef struct {

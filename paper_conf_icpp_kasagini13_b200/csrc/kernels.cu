@@ -257,7 +257,19 @@ __device__ __forceinline__ void tile_load(const RowArgs& a, uint32_t* sm, long l
     const uint32_t* base = a.in + cta * m.cta_stride;
     constexpr int NV = EPT / 4;
     uint4 val[NV];
-    if (!m.cross) {
+    if (a.in_segs > 1) {
+        // sharded column phase: line l (global t*h + l) = in_segs segments of seg_len words
+        // at in + s*seg_stride + (t*h + l)*seg_len (whole lines, m.w == L)
+        const int logL = m.logw;
+        const int logS = 31 - __clz((int)a.seg_len);
+#pragma unroll
+        for (int it = 0; it < NV; ++it) {
+            const int f = 4 * (tid + T * it);
+            const int l = f >> logL, pos = f & ((1 << logL) - 1);
+            const int s = pos >> logS, off = pos & ((1 << logS) - 1);
+            val[it] = ld_nc_v4(a.in + s * a.seg_stride + (cta * (1 << a.logh) + l) * a.seg_len + off);
+        }
+    } else if (!m.cross) {
         const int loghw = a.logh + m.logw;
 #pragma unroll
         for (int it = 0; it < NV; ++it) {
@@ -265,6 +277,9 @@ __device__ __forceinline__ void tile_load(const RowArgs& a, uint32_t* sm, long l
             const int K = f >> loghw, rem = f & ((1 << loghw) - 1);
             val[it] = ld_nc_v4(base + (long long)K * m.strideK + rem);
         }
+    }
+    if (!m.cross) {
+        const int loghw = a.logh + m.logw;
 #pragma unroll
         for (int it = 0; it < NV; ++it) {
             const int f = 4 * (tid + T * it);
@@ -959,6 +974,7 @@ struct TlcArgs {
     int t_h;                   // lines per tile (tensor-store coordinates)
     int nbox, box_outer, box_words;
     unsigned long long* trace;
+    int prefetch_in;           // stream the whole input into L2 up front (HBM-resident input)
 };
 
 // One row-wise permutation pass (Lemma 7) with the tile-level bank colouring
@@ -1000,12 +1016,23 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     if (warp == 0) {
         if (lane == 0) {
             // ---------------- producer
-            for (int i = 0; i <= NS; ++i) {      // schedules do not depend on the previous pass
+            // Deep memory-level parallelism without shared memory: every schedule chunk of
+            // this CTA (independent of the previous pass) and, for HBM-resident input, every
+            // input tile are requested into L2 now; the smem ring then streams from L2.
+            for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
-                if (t < a.ntiles) prefetch_l2_bulk(a.sched + t * a.tile_words, (uint32_t)(a.tile_words * 4));
+                if (t >= a.ntiles) break;
+                prefetch_l2_bulk(a.sched + t * a.tile_words, (uint32_t)(a.tile_words * 4));
             }
             pdl_wait();
             stamp(tr, 1);
+            if (a.prefetch_in) {
+                for (int i = NS;; ++i) {
+                    const long long t = blockIdx.x + (long long)i * G;
+                    if (t >= a.ntiles) break;
+                    prefetch_l2_bulk(a.in + t * HL, (uint32_t)HL * 4u);
+                }
+            }
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
@@ -1014,8 +1041,6 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 fence_proxy_async();
                 mbar_arrive_expect_tx(&full[s], (uint32_t)HL * 4u);
                 bulk_g2s(smem + s * 2 * HL, a.in + t * HL, (uint32_t)HL * 4u, &full[s]);
-                const long long tp = t + (long long)(NS + 1) * G;
-                if (tp < a.ntiles) prefetch_l2_bulk(a.sched + tp * a.tile_words, (uint32_t)(a.tile_words * 4));
                 if (i == 0) pdl_launch_dependents();
             }
         }
@@ -1610,6 +1635,7 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
     ta.tile_words = tp.tile_words;
     ta.t_h = tp.h;
     ta.trace = trace;
+    ta.prefetch_in = (f == 0) ? 1 : 0;   // pass 1 reads `a` from HBM; later passes read L2-resident X
     const long long h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
     if (tp.out_kind == 1) {
         const long long outer = P.c / h2, bo = outer < 256 ? outer : 256;

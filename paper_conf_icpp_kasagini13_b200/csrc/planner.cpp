@@ -268,7 +268,11 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
         int64_t h = (opt && (&opt->h1)[f] > 0) ? (&opt->h1)[f]
                                                 : std::max<int64_t>(4, 8192 / L);
         h = std::min(h, lines_f);
-        if (h < 4 || (h & (h - 1)) || lines_f % h) { err = "TLC layout: h must be a power of two >= 4"; return PERM_EINVAL; }
+        // h2 is the inner dimension of the TMA tensor boxes (>= 16 bytes)
+        if (h < (f == 1 ? 4 : 1) || (h & (h - 1)) || lines_f % h) {
+            err = "TLC layout: h must be a power of two (h2 >= 4)";
+            return PERM_EINVAL;
+        }
         hs[f] = h;
     }
     const int64_t h1 = hs[0], h2 = hs[1], h3 = hs[2];
@@ -580,7 +584,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.out = runs(L, 0, h * L);
             // TMA pipeline when `stages` tiles (lines + schedule) fit in shared memory
             rp.tma = (stages * stage_bytes(h, f, 0) <= kSmemBudget &&
-                      (h * (L / kW) * P.ph[f].w64 * 2) % 4 == 0) ? 1 : 0;
+                      (h * (L / kW) * P.ph[f].w64 * 2) % 4 == 0 && !(opt && opt->no_tma)) ? 1 : 0;
             rp.stages = rp.tma ? stages : 0;
         }
     }
@@ -682,10 +686,8 @@ int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, i
             rp.in_segs = world;
             rp.seg_len = f == 1 ? P.r_l : P.c_l;
             rp.seg_stride = P.r_l * P.c_l;
-            if (!rp.tma) {
-                err = "row sharding: lines must fit the TMA pass (L <= 16384)";
-                return PERM_EUNSUPPORTED;
-            }
+            // both the TMA pass (one bulk copy per segment) and the plain pass (128-bit
+            // loads per segment) gather segmented lines
         }
     }
     return PERM_OK;

@@ -127,8 +127,8 @@ def test_config1_random_seeds_and_5pass(P):
     a = W.make_data(n)
     for seed in (42, 43, 44):
         p = W.random(n, seed)
-        for passes in (3, 5):
-            b, _ = run(P, p, a, passes=passes)
+        for passes, no_tma in ((3, 0), (5, 0), (5, 1)):
+            b, _ = run(P, p, a, passes=passes, no_tma=no_tma)
             assert np.array_equal(b, OA.apply_ref(p, a)), (seed, passes)
 
 

@@ -26,16 +26,17 @@ def P():
     return pkg
 
 
+@pytest.mark.parametrize("no_tma", [0, 1])
 @pytest.mark.parametrize("G", [1, 2, 4, 8])
 @pytest.mark.parametrize("k", [16, 19, 22])
-def test_virtual_ranks(P, G, k):
+def test_virtual_ranks(P, G, k, no_tma):
     from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
     n = 1 << k
     shard = n // G
     a = W.make_data(n)
     for fam in ("random", "bitrev", "transpose"):
         p = W.make_perm(fam, n, seed=G + k)
-        plans = [P.Plan(p, world=G, rank=g) for g in range(G)]
+        plans = [P.Plan(p, world=G, rank=g, no_tma=no_tma) for g in range(G)]
         try:
             a_sh = [torch.from_numpy(a[g * shard:(g + 1) * shard].view(np.int32).copy()).cuda() for g in range(G)]
             b_sh = [torch.full((shard,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
