@@ -21,6 +21,8 @@
 // edges on each side. Recurse log2(d) times. O(E log d).
 #include <algorithm>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 
@@ -95,6 +97,180 @@ struct EulerColourer {
         }
     }
 
+    // The same split of one big group by all threads (top recursion levels, where
+    // there are fewer groups than threads). (1) pairing: every thread pairs the edges
+    // of its chunk at each node; the at most one leftover per node per thread is
+    // paired sequentially. (2) the alternating cycles are coloured by concurrent
+    // walks: a walk claims edges (CAS on owner[]) in both directions from its start
+    // and stops at the first edge another walk owns, recording that boundary; every
+    // walk is a segment with tentative bits. (3) the boundaries give parity
+    // constraints between segments (bits of adjacent edges must differ), solved by
+    // BFS; (4) flipped segments' bits are inverted; (5) parallel stable partition.
+    std::vector<int32_t> owner;
+
+    void split_group_par(int64_t base, int64_t S, int64_t nodes) {
+        static const bool verbose = std::getenv("PERM_PLANNER_VERBOSE") != nullptr;
+        auto t0 = clk::now();
+#ifdef _OPENMP
+        const int T = omp_get_max_threads();
+#else
+        const int T = 1;
+#endif
+        std::vector<std::vector<uint32_t>> leftL(T), leftR(T);
+#pragma omp parallel num_threads(T)
+        {
+#ifdef _OPENMP
+            const int t = omp_get_thread_num();
+#else
+            const int t = 0;
+#endif
+            const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
+            std::vector<uint32_t> pend((size_t)nodes, kNone);
+            for (int64_t i = lo; i < hi; ++i) {
+                uint32_t& q = pend[pu[i]];
+                if (q == kNone) q = (uint32_t)i;
+                else { pL[i] = q; pL[q] = (uint32_t)i; q = kNone; }
+            }
+            for (int64_t u = 0; u < nodes; ++u)
+                if (pend[u] != kNone) { leftL[t].push_back(pend[u]); pend[u] = kNone; }
+            for (int64_t i = lo; i < hi; ++i) {
+                uint32_t& q = pend[pv[i]];
+                if (q == kNone) q = (uint32_t)i;
+                else { pR[i] = q; pR[q] = (uint32_t)i; q = kNone; }
+            }
+            for (int64_t u = 0; u < nodes; ++u)
+                if (pend[u] != kNone) leftR[t].push_back(pend[u]);
+        }
+        {
+            std::vector<uint32_t> pend((size_t)nodes, kNone);
+            for (int t = 0; t < T; ++t)
+                for (uint32_t i : leftL[t]) {
+                    uint32_t& q = pend[pu[i]];
+                    if (q == kNone) q = i;
+                    else { pL[i] = q; pL[q] = i; q = kNone; }
+                }
+            std::fill(pend.begin(), pend.end(), kNone);
+            for (int t = 0; t < T; ++t)
+                for (uint32_t i : leftR[t]) {
+                    uint32_t& q = pend[pv[i]];
+                    if (q == kNone) q = i;
+                    else { pR[i] = q; pR[q] = i; q = kNone; }
+                }
+        }
+        const double ms_pair = ms_since(t0);
+        if ((int64_t)owner.size() < S) owner.resize((size_t)S);
+        int32_t* own = owner.data() - base;              // indexed by absolute position
+#pragma omp parallel for schedule(static)
+        for (int64_t i = base; i < base + S; ++i) own[i] = -1;
+        // segment id = t + T * (walk number of thread t): no shared counter
+        struct Bound { uint32_t x, y; };
+        std::vector<std::vector<Bound>> bounds(T);
+        std::vector<int32_t> walks(T, 0);
+        auto claim = [&](uint32_t e, int32_t sid) {
+            int32_t expect = -1;
+            return __atomic_compare_exchange_n(&own[e], &expect, sid, false, __ATOMIC_RELAXED,
+                                               __ATOMIC_RELAXED);
+        };
+#pragma omp parallel num_threads(T)
+        {
+#ifdef _OPENMP
+            const int t = omp_get_thread_num();
+#else
+            const int t = 0;
+#endif
+            const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
+            std::vector<Bound>& bd = bounds[t];
+            int32_t w = 0;
+            for (int64_t e0 = lo; e0 < hi; ++e0) {
+                if (__atomic_load_n(&own[e0], __ATOMIC_RELAXED) != -1) continue;
+                const int32_t sid = t + T * w;
+                if (!claim((uint32_t)e0, sid)) continue;
+                ++w;
+                bit[e0] = 0;
+                for (int dir = 0; dir < 2; ++dir) {       // 0: L first (forward), 1: R first
+                    uint32_t cur = (uint32_t)e0;
+                    while (true) {
+                        const uint32_t a = dir == 0 ? pL[cur] : pR[cur];
+                        if (!claim(a, sid)) { bd.push_back({cur, a}); break; }
+                        bit[a] = bit[cur] ^ 1;
+                        const uint32_t b = dir == 0 ? pR[a] : pL[a];
+                        if (!claim(b, sid)) { bd.push_back({a, b}); break; }
+                        bit[b] = bit[a] ^ 1;
+                        cur = b;
+                    }
+                }
+            }
+            walks[t] = w;
+        }
+        const double ms_walk = ms_since(t0);
+        // parity union-find over segments: flip[A] ^ flip[B] = (bit[x] == bit[y])
+        int32_t maxw = 0;
+        for (int t = 0; t < T; ++t) maxw = std::max(maxw, walks[t]);
+        const int64_t nseg = (int64_t)T * maxw;
+        std::vector<int32_t> parent((size_t)nseg);
+        std::vector<uint8_t> par((size_t)nseg, 0);
+        std::iota(parent.begin(), parent.end(), 0);
+        auto find = [&](int32_t s, uint8_t& px) {
+            uint8_t acc = 0;
+            int32_t r0 = s;
+            while (parent[r0] != r0) { acc ^= par[r0]; r0 = parent[r0]; }
+            // path compression with parity
+            uint8_t acc2 = acc;
+            while (parent[s] != s) {
+                const int32_t nx = parent[s];
+                const uint8_t ps = par[s];
+                parent[s] = r0;
+                par[s] = acc2;
+                acc2 ^= ps;
+                s = nx;
+            }
+            px = acc;
+            return r0;
+        };
+        for (int t = 0; t < T; ++t)
+            for (const Bound& b : bounds[t]) {
+                const int32_t A = own[b.x], B = own[b.y];
+                if (A == B) continue;                     // closed inside one walk: consistent
+                const uint8_t dd = (bit[b.x] == bit[b.y]) ? 1 : 0;
+                uint8_t pa, pb;
+                const int32_t ra = find(A, pa), rb = find(B, pb);
+                if (ra != rb) { parent[ra] = rb; par[ra] = (uint8_t)(pa ^ pb ^ dd); }
+            }
+        std::vector<uint8_t> flip((size_t)nseg, 0);
+        for (int64_t s = 0; s < nseg; ++s) { uint8_t px; find((int32_t)s, px); flip[s] = px; }
+#pragma omp parallel for schedule(static)
+        for (int64_t i = base; i < base + S; ++i)
+            if (flip[own[i]]) bit[i] ^= 1;
+        const double ms_flip = ms_since(t0);
+        // parallel stable partition (zeros first)
+        std::vector<int64_t> zc(T + 1, 0);
+#pragma omp parallel num_threads(T)
+        {
+#ifdef _OPENMP
+            const int t = omp_get_thread_num();
+#else
+            const int t = 0;
+#endif
+            const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
+            int64_t z = 0;
+            for (int64_t i = lo; i < hi; ++i) z += bit[i] == 0;
+            zc[t + 1] = z;
+#pragma omp barrier
+#pragma omp single
+            for (int u = 0; u < T; ++u) zc[u + 1] += zc[u];
+            int64_t zp = base + zc[t], op = base + S / 2 + ((lo - base) - zc[t]);
+            for (int64_t i = lo; i < hi; ++i) {
+                const int64_t dst = bit[i] ? op++ : zp++;
+                ord2[dst] = ord[i];
+                pu2[dst] = pu[i];
+                pv2[dst] = pv[i];
+            }
+        }
+        if (verbose)
+            std::fprintf(stderr, "  split_par S=%lld: pair %.1f walk %.1f flip %.1f total %.1f ms (segments %lld)\n",
+                         (long long)S, ms_pair, ms_walk, ms_flip, ms_since(t0), (long long)nseg);
+    }
+
     void run(int64_t nodes, int64_t d, int64_t E, const uint32_t* U, const uint32_t* V,
              uint32_t* colour, bool parallel) {
         if (d <= 1) {
@@ -107,9 +283,19 @@ struct EulerColourer {
         }
         for (int64_t i = 0; i < E; ++i) { ord[i] = (uint32_t)i; pu[i] = U[i]; pv[i] = V[i]; }
         const int levels = ilog2(d);
+#ifdef _OPENMP
+        const int64_t nthreads = omp_get_max_threads();
+#else
+        const int64_t nthreads = 1;
+#endif
+        static const bool seq_top = std::getenv("PERM_PLANNER_SEQ_TOP") != nullptr;
+        static const bool verbose = std::getenv("PERM_PLANNER_VERBOSE") != nullptr;
         for (int lvl = 0; lvl < levels; ++lvl) {
             const int64_t G = int64_t(1) << lvl, S = E / G;
-            if (parallel && G > 1) {
+            auto tl = clk::now();
+            if (!seq_top && parallel && nthreads > 1 && G < nthreads && S >= (int64_t(1) << 20)) {
+                for (int64_t g = 0; g < G; ++g) split_group_par(g * S, S, nodes);
+            } else if (parallel && G > 1) {
 #pragma omp parallel
                 {
                     std::vector<uint32_t> pend(nodes);
@@ -121,6 +307,9 @@ struct EulerColourer {
                 for (int64_t g = 0; g < G; ++g) split_group(g * S, S, nodes, pend);
             }
             ord.swap(ord2); pu.swap(pu2); pv.swap(pv2);
+            if (verbose && E >= (int64_t(1) << 20))
+                std::fprintf(stderr, "euler level %d: G=%lld S=%lld %.1f ms\n", lvl, (long long)G,
+                             (long long)S, ms_since(tl));
         }
         const int64_t per = E / d;   // a perfect matching per colour
         for (int64_t i = 0; i < E; ++i) colour[ord[i]] = (uint32_t)(i / per);
