@@ -40,7 +40,8 @@ enum perm_status {
     PERM_OK           =  0,
     PERM_EINVAL       = -1,  /* null pointer, n <= 0, a == b / overlapping buffers, bad option */
     PERM_ENOTPERM     = -2,  /* p is not a permutation of 0..n-1 (value out of range or repeated) */
-    PERM_EUNSUPPORTED = -3,  /* n not a power of two in [2^10, 2^30], or elem_bytes != 4 */
+    PERM_EUNSUPPORTED = -3,  /* n not a power of two in [2^10, 2^30] (2^9..2^29 for 8-byte
+                                elements), or elem_bytes not 4 or 8 */
     PERM_ENOMEM       = -4,  /* host or device allocation failed */
     PERM_ECUDA        = -5,  /* a CUDA runtime call failed (message has the CUDA error) */
     PERM_ENCCL        = -6,  /* reserved for the row-sharded multi-GPU path */
@@ -100,7 +101,9 @@ typedef struct {
 /* Build a plan for P on the CURRENT CUDA device: validates p (O(n) bitmap),
  * colours, packs and uploads the schedules and allocates scratch.
  * p: host int32[n], borrowed for the duration of the call only.
- * n: power of two, 2^10 <= n <= 2^30. elem_bytes: 4.
+ * n: power of two, 2^10 <= n <= 2^30. elem_bytes: 4, or 8 (n <= 2^29): an 8-byte
+ * element moves as a pair of 4-byte words (the word permutation 2P(i)+h is
+ * scheduled; info/export then describe 2n words).
  * Returns NULL on error (see perm_last_error). Synchronous. */
 perm_plan* perm_plan_create(const int32_t* p, int64_t n, int32_t elem_bytes);
 

@@ -192,7 +192,7 @@ class Plan:
         inf = self.info()
         r, c = inf["rows"], inf["cols"]
         G = inf["world"]
-        kappa = np.empty(self.n, dtype=np.uint16)
+        kappa = np.empty(r * c, dtype=np.uint16)        # words (2n for 8-byte elements)
         s1 = np.empty((r // G, c), dtype=np.uint32)     # sharded plans: this rank's lines
         s2 = np.empty((c // G, r), dtype=np.uint32)
         s3 = np.empty((r // G, c), dtype=np.uint32)
@@ -243,17 +243,17 @@ class Plan:
         return [float(buf[i]) for i in range(k)]
 
 
-def scatter_baseline(p_dev, a, b, stream=None):
+def scatter_baseline(p_dev, a, b, stream=None, elem_bytes: int = 4):
     """D-designated b[p[i]] = a[i], one kernel. p_dev: int32 CUDA tensor."""
     n = p_dev.numel()
-    _check(_scatter(_ptr(p_dev), _ptr(a), _ptr(b), n, 4, _stream_handle(stream)))
+    _check(_scatter(_ptr(p_dev), _ptr(a), _ptr(b), n, elem_bytes, _stream_handle(stream)))
     return b
 
 
-def gather_baseline(q_dev, a, b, stream=None):
+def gather_baseline(q_dev, a, b, stream=None, elem_bytes: int = 4):
     """S-designated b[i] = a[q[i]], q = P^{-1} on the device."""
     n = q_dev.numel()
-    _check(_gather(_ptr(q_dev), _ptr(a), _ptr(b), n, 4, _stream_handle(stream)))
+    _check(_gather(_ptr(q_dev), _ptr(a), _ptr(b), n, elem_bytes, _stream_handle(stream)))
     return b
 
 

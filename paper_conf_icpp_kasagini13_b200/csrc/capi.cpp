@@ -228,14 +228,14 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     if (!plan || !out) return fail(PERM_EINVAL, "null plan or info");
     const HostPlan& P = plan->host;
     std::memset(out, 0, sizeof(*out));
-    out->n = P.n;
+    out->n = P.user_n;
     out->rows = P.r;
     out->cols = P.c;
     int64_t words = 0;
     for (int f = 0; f < 3; ++f) words += (int64_t)P.sched[f].size();
     out->sched_bytes = plan->on_device ? plan->sched_bytes : words * 4;
     out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes == 1 ? 0 : 2 * P.n * P.eb);
-    out->elem_bytes = P.eb;
+    out->elem_bytes = P.user_eb;
     out->passes = P.passes;
     out->kernels_per_apply = P.fused3 ? 1 : P.passes;
     for (int f = 0; f < 3; ++f) {
@@ -248,8 +248,9 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->build_ms_upload = plan->ms_upload;
     out->world = P.r_l ? P.world : 1;
     out->rank = P.r_l ? P.rank : 0;
-    out->shard_elems = P.r_l ? P.n / P.world : P.n;
-    out->block_elems = P.r_l ? P.n / ((int64_t)P.world * P.world) : P.n;
+    const int64_t wpe = P.user_eb / 4;          // words per caller element
+    out->shard_elems = (P.r_l ? P.n / P.world : P.n) / wpe;
+    out->block_elems = (P.r_l ? P.n / ((int64_t)P.world * P.world) : P.n) / wpe;
     return PERM_OK;
 }
 
@@ -313,7 +314,7 @@ int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint3
                      uint32_t* s3) {
     if (!plan) return fail(PERM_EINVAL, "null plan");
     const HostPlan& P = plan->host;
-    if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));
+    if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));   // words
     uint32_t* outs[3] = {s1, s2, s3};
     if (P.layout == 3) {
         // TLC: entry (tile T, round q, lane x) -> (src word offset in A << 16) | dst offset in B
@@ -502,10 +503,9 @@ int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stre
 int perm_scatter_baseline(const int32_t* p_dev, const void* a, void* b, int64_t n,
                           int32_t elem_bytes, perm_stream_t stream) {
     if (!p_dev || !a || !b || n <= 0) return fail(PERM_EINVAL, "null argument or n <= 0");
-    if (elem_bytes != 4 || (n & 3)) return fail(PERM_EUNSUPPORTED, "elem_bytes 4, n % 4 == 0");
-    cudaError_t e = perm::launch_scatter(p_dev, static_cast<const uint32_t*>(a),
-                                         static_cast<uint32_t*>(b), n,
-                                         static_cast<cudaStream_t>(stream));
+    if ((elem_bytes != 4 && elem_bytes != 8) || (n & 3))
+        return fail(PERM_EUNSUPPORTED, "elem_bytes 4 or 8, n % 4 == 0");
+    cudaError_t e = perm::launch_scatter(p_dev, a, b, n, elem_bytes, static_cast<cudaStream_t>(stream));
     if (e != cudaSuccess) return cuda_fail(e, "scatter launch");
     return PERM_OK;
 }
@@ -513,10 +513,9 @@ int perm_scatter_baseline(const int32_t* p_dev, const void* a, void* b, int64_t 
 int perm_gather_baseline(const int32_t* q_dev, const void* a, void* b, int64_t n,
                          int32_t elem_bytes, perm_stream_t stream) {
     if (!q_dev || !a || !b || n <= 0) return fail(PERM_EINVAL, "null argument or n <= 0");
-    if (elem_bytes != 4 || (n & 3)) return fail(PERM_EUNSUPPORTED, "elem_bytes 4, n % 4 == 0");
-    cudaError_t e = perm::launch_gather(q_dev, static_cast<const uint32_t*>(a),
-                                        static_cast<uint32_t*>(b), n,
-                                        static_cast<cudaStream_t>(stream));
+    if ((elem_bytes != 4 && elem_bytes != 8) || (n & 3))
+        return fail(PERM_EUNSUPPORTED, "elem_bytes 4 or 8, n % 4 == 0");
+    cudaError_t e = perm::launch_gather(q_dev, a, b, n, elem_bytes, static_cast<cudaStream_t>(stream));
     if (e != cudaSuccess) return cuda_fail(e, "gather launch");
     return PERM_OK;
 }

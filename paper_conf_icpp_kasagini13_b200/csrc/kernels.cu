@@ -1384,6 +1384,34 @@ __global__ void __launch_bounds__(256) gather_kernel(const int32_t* __restrict__
     }
 }
 
+// 8-byte element variants (Table II(b)): 2 x 64-bit element loads per 128-bit p/q load
+__global__ void __launch_bounds__(256) scatter64_kernel(const int32_t* __restrict__ p,
+                                                        const uint2* __restrict__ a,
+                                                        uint2* __restrict__ b, long long nv) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nv;
+         v += (long long)gridDim.x * blockDim.x) {
+        const uint4 pv = ld_nc_v4(reinterpret_cast<const uint32_t*>(p) + 4 * v);
+        const uint4 a0 = ld_nc_v4(reinterpret_cast<const uint32_t*>(a + 4 * v));
+        const uint4 a1 = ld_nc_v4(reinterpret_cast<const uint32_t*>(a + 4 * v + 2));
+        b[pv.x] = make_uint2(a0.x, a0.y);
+        b[pv.y] = make_uint2(a0.z, a0.w);
+        b[pv.z] = make_uint2(a1.x, a1.y);
+        b[pv.w] = make_uint2(a1.z, a1.w);
+    }
+}
+
+__global__ void __launch_bounds__(256) gather64_kernel(const int32_t* __restrict__ q,
+                                                       const uint2* __restrict__ a,
+                                                       uint2* __restrict__ b, long long nv) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nv;
+         v += (long long)gridDim.x * blockDim.x) {
+        const uint4 qv = ld_nc_v4(reinterpret_cast<const uint32_t*>(q) + 4 * v);
+        const uint2 x0 = __ldg(a + qv.x), x1 = __ldg(a + qv.y), x2 = __ldg(a + qv.z), x3 = __ldg(a + qv.w);
+        st_v4(reinterpret_cast<uint32_t*>(b + 4 * v), make_uint4(x0.x, x0.y, x1.x, x1.y));
+        st_v4(reinterpret_cast<uint32_t*>(b + 4 * v + 2), make_uint4(x2.x, x2.y, x3.x, x3.y));
+    }
+}
+
 __global__ void __launch_bounds__(256) copy_kernel(const uint32_t* __restrict__ a,
                                                    uint32_t* __restrict__ b, long long nv) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nv;
@@ -1941,16 +1969,24 @@ static unsigned stream_grid(long long nv) {
     return (unsigned)(want < cap ? (want > 0 ? want : 1) : cap);
 }
 
-cudaError_t launch_scatter(const int32_t* p, const uint32_t* a, uint32_t* b, int64_t n,
+cudaError_t launch_scatter(const int32_t* p, const void* a, void* b, int64_t n, int eb,
                            cudaStream_t s) {
     const long long nv = n / 4;
-    return launch(scatter_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, p, a, b, nv);
+    if (eb == 8)
+        return launch(scatter64_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, p,
+                      static_cast<const uint2*>(a), static_cast<uint2*>(b), nv);
+    return launch(scatter_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, p,
+                  static_cast<const uint32_t*>(a), static_cast<uint32_t*>(b), nv);
 }
 
-cudaError_t launch_gather(const int32_t* q, const uint32_t* a, uint32_t* b, int64_t n,
+cudaError_t launch_gather(const int32_t* q, const void* a, void* b, int64_t n, int eb,
                           cudaStream_t s) {
     const long long nv = n / 4;
-    return launch(gather_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, q, a, b, nv);
+    if (eb == 8)
+        return launch(gather64_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, q,
+                      static_cast<const uint2*>(a), static_cast<uint2*>(b), nv);
+    return launch(gather_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, q,
+                  static_cast<const uint32_t*>(a), static_cast<uint32_t*>(b), nv);
 }
 
 cudaError_t launch_copy(const uint32_t* a, uint32_t* b, int64_t n, cudaStream_t s) {

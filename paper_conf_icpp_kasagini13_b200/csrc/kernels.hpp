@@ -47,9 +47,9 @@ cudaError_t launch_transpose(const uint32_t* in, uint32_t* out, int64_t rows, in
                              cudaStream_t s, bool pdl);
 
 // Comparators and a plain vector copy.
-cudaError_t launch_scatter(const int32_t* p, const uint32_t* a, uint32_t* b, int64_t n,
+cudaError_t launch_scatter(const int32_t* p, const void* a, void* b, int64_t n, int eb,
                            cudaStream_t s);
-cudaError_t launch_gather(const int32_t* q, const uint32_t* a, uint32_t* b, int64_t n,
+cudaError_t launch_gather(const int32_t* q, const void* a, void* b, int64_t n, int eb,
                           cudaStream_t s);
 cudaError_t launch_copy(const uint32_t* a, uint32_t* b, int64_t n, cudaStream_t s);
 

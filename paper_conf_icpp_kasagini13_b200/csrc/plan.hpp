@@ -89,8 +89,10 @@ struct TlcPass {
 };
 
 struct HostPlan {
-    int64_t n = 0;
-    int32_t eb = 4;
+    int64_t n = 0;             // words permuted (2 * user_n for 8-byte elements)
+    int32_t eb = 4;            // word size used by the kernels (always 4)
+    int32_t user_eb = 4;       // element size of the caller (4 or 8)
+    int64_t user_n = 0;        // elements of the caller
     int32_t k = 0;             // log2 n
     int64_t r = 0, c = 0;      // view
     int32_t passes = 0;        // 1, 3, 5

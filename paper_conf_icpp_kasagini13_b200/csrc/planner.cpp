@@ -116,15 +116,13 @@ struct EulerColourer {
 #else
         const int T = 1;
 #endif
-        std::vector<std::vector<uint32_t>> leftL(T), leftR(T);
-#pragma omp parallel num_threads(T)
-        {
-#ifdef _OPENMP
-            const int t = omp_get_thread_num();
-#else
-            const int t = 0;
-#endif
-            const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
+        // a fixed chunking (not the thread count) keeps the pairing, and so the colouring,
+        // identical on every rank / machine: sharded plans rely on it
+        constexpr int NCH = 64;
+        std::vector<std::vector<uint32_t>> leftL(NCH), leftR(NCH);
+#pragma omp parallel for schedule(dynamic, 1)
+        for (int ch = 0; ch < NCH; ++ch) {
+            const int64_t lo = base + S * ch / NCH, hi = base + S * (ch + 1) / NCH;
             std::vector<uint32_t> pend((size_t)nodes, kNone);
             for (int64_t i = lo; i < hi; ++i) {
                 uint32_t& q = pend[pu[i]];
@@ -132,26 +130,26 @@ struct EulerColourer {
                 else { pL[i] = q; pL[q] = (uint32_t)i; q = kNone; }
             }
             for (int64_t u = 0; u < nodes; ++u)
-                if (pend[u] != kNone) { leftL[t].push_back(pend[u]); pend[u] = kNone; }
+                if (pend[u] != kNone) { leftL[ch].push_back(pend[u]); pend[u] = kNone; }
             for (int64_t i = lo; i < hi; ++i) {
                 uint32_t& q = pend[pv[i]];
                 if (q == kNone) q = (uint32_t)i;
                 else { pR[i] = q; pR[q] = (uint32_t)i; q = kNone; }
             }
             for (int64_t u = 0; u < nodes; ++u)
-                if (pend[u] != kNone) leftR[t].push_back(pend[u]);
+                if (pend[u] != kNone) leftR[ch].push_back(pend[u]);
         }
         {
             std::vector<uint32_t> pend((size_t)nodes, kNone);
-            for (int t = 0; t < T; ++t)
-                for (uint32_t i : leftL[t]) {
+            for (int ch = 0; ch < NCH; ++ch)
+                for (uint32_t i : leftL[ch]) {
                     uint32_t& q = pend[pu[i]];
                     if (q == kNone) q = i;
                     else { pL[i] = q; pL[q] = i; q = kNone; }
                 }
             std::fill(pend.begin(), pend.end(), kNone);
-            for (int t = 0; t < T; ++t)
-                for (uint32_t i : leftR[t]) {
+            for (int ch = 0; ch < NCH; ++ch)
+                for (uint32_t i : leftR[ch]) {
                     uint32_t& q = pend[pv[i]];
                     if (q == kNone) q = i;
                     else { pR[i] = q; pR[q] = i; q = kNone; }
@@ -165,6 +163,7 @@ struct EulerColourer {
         // segment id = t + T * (walk number of thread t): no shared counter
         struct Bound { uint32_t x, y; };
         std::vector<std::vector<Bound>> bounds(T);
+        std::vector<std::vector<uint32_t>> segmin(T);    // smallest position a walk claimed
         std::vector<int32_t> walks(T, 0);
         auto claim = [&](uint32_t e, int32_t sid) {
             int32_t expect = -1;
@@ -180,6 +179,7 @@ struct EulerColourer {
 #endif
             const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
             std::vector<Bound>& bd = bounds[t];
+            std::vector<uint32_t>& mins = segmin[t];
             int32_t w = 0;
             for (int64_t e0 = lo; e0 < hi; ++e0) {
                 if (__atomic_load_n(&own[e0], __ATOMIC_RELAXED) != -1) continue;
@@ -187,18 +187,22 @@ struct EulerColourer {
                 if (!claim((uint32_t)e0, sid)) continue;
                 ++w;
                 bit[e0] = 0;
+                uint32_t mn = (uint32_t)e0;
                 for (int dir = 0; dir < 2; ++dir) {       // 0: L first (forward), 1: R first
                     uint32_t cur = (uint32_t)e0;
                     while (true) {
                         const uint32_t a = dir == 0 ? pL[cur] : pR[cur];
                         if (!claim(a, sid)) { bd.push_back({cur, a}); break; }
                         bit[a] = bit[cur] ^ 1;
+                        mn = a < mn ? a : mn;
                         const uint32_t b = dir == 0 ? pR[a] : pL[a];
                         if (!claim(b, sid)) { bd.push_back({a, b}); break; }
                         bit[b] = bit[a] ^ 1;
+                        mn = b < mn ? b : mn;
                         cur = b;
                     }
                 }
+                mins.push_back(mn);
             }
             walks[t] = w;
         }
@@ -236,8 +240,24 @@ struct EulerColourer {
                 const int32_t ra = find(A, pa), rb = find(B, pb);
                 if (ra != rb) { parent[ra] = rb; par[ra] = (uint8_t)(pa ^ pb ^ dd); }
             }
+        // canonical polarity: in every cycle (component) the smallest position gets bit 0,
+        // so the colouring does not depend on which walk happened to claim what
         std::vector<uint8_t> flip((size_t)nseg, 0);
-        for (int64_t s = 0; s < nseg; ++s) { uint8_t px; find((int32_t)s, px); flip[s] = px; }
+        std::vector<uint32_t> cmin((size_t)nseg, kNone);
+        std::vector<uint8_t> cbit((size_t)nseg, 0);
+        std::vector<int32_t> root((size_t)nseg, -1);
+        for (int t = 0; t < T; ++t)
+            for (int32_t w = 0; w < walks[t]; ++w) {
+                const int32_t s = t + T * w;
+                uint8_t px;
+                const int32_t rt = find(s, px);
+                root[s] = rt;
+                flip[s] = px;
+                const uint32_t m = segmin[t][w];
+                if (m < cmin[rt]) { cmin[rt] = m; cbit[rt] = (uint8_t)(bit[m] ^ px); }
+            }
+        for (int64_t s = 0; s < nseg; ++s)
+            if (root[s] >= 0) flip[s] ^= cbit[root[s]];
 #pragma omp parallel for schedule(static)
         for (int64_t i = base; i < base + S; ++i)
             if (flip[own[i]]) bit[i] ^= 1;
@@ -283,17 +303,15 @@ struct EulerColourer {
         }
         for (int64_t i = 0; i < E; ++i) { ord[i] = (uint32_t)i; pu[i] = U[i]; pv[i] = V[i]; }
         const int levels = ilog2(d);
-#ifdef _OPENMP
-        const int64_t nthreads = omp_get_max_threads();
-#else
-        const int64_t nthreads = 1;
-#endif
         static const bool seq_top = std::getenv("PERM_PLANNER_SEQ_TOP") != nullptr;
         static const bool verbose = std::getenv("PERM_PLANNER_VERBOSE") != nullptr;
         for (int lvl = 0; lvl < levels; ++lvl) {
             const int64_t G = int64_t(1) << lvl, S = E / G;
             auto tl = clk::now();
-            if (!seq_top && parallel && nthreads > 1 && G < nthreads && S >= (int64_t(1) << 20)) {
+            // big groups: the chunked-pairing split (all threads inside one group). The choice
+            // depends on S only, never on the thread count: every machine and every rank of a
+            // sharded plan produces the same colouring.
+            if (!seq_top && parallel && S >= (int64_t(1) << 20)) {
                 for (int64_t g = 0; g < G; ++g) split_group_par(g * S, S, nodes);
             } else if (parallel && G > 1) {
 #pragma omp parallel
@@ -552,7 +570,34 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
 int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_options* opt,
                     HostPlan& P, std::string& err) {
     if (!p || n <= 0) { err = "null p or n <= 0"; return PERM_EINVAL; }
-    if (eb != 4) { err = "elem_bytes must be 4"; return PERM_EUNSUPPORTED; }
+    if (eb == 8) {
+        // 8-byte elements (Table II(b)): element i is the word pair (2i, 2i+1);
+        // permuting it to P(i) is the word permutation P'(2i + h) = 2P(i) + h, scheduled
+        // like any other (reading #10).
+        if (n > (int64_t(1) << 29)) { err = "n must be <= 2^29 for 8-byte elements"; return PERM_EUNSUPPORTED; }
+        std::vector<uint8_t> seen((size_t)n, 0);
+        for (int64_t i = 0; i < n; ++i) {
+            const int32_t v = p[i];
+            if (v < 0 || v >= n || seen[v]) {
+                err = "p is not a permutation: entry " + std::to_string(i) + " = " + std::to_string(v);
+                return PERM_ENOTPERM;
+            }
+            seen[v] = 1;
+        }
+        std::vector<int32_t> p2((size_t)(2 * n));
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) {
+            p2[2 * i] = 2 * p[i];
+            p2[2 * i + 1] = 2 * p[i] + 1;
+        }
+        const int st = build_host_plan(p2.data(), 2 * n, 4, opt, P, err);
+        P.user_eb = 8;
+        P.user_n = n;
+        return st;
+    }
+    if (eb != 4) { err = "elem_bytes must be 4 or 8"; return PERM_EUNSUPPORTED; }
+    P.user_eb = 4;
+    P.user_n = n;
     const int k = ilog2(n);
     if ((int64_t(1) << k) != n || k < 10 || k > 30) {
         err = "n must be a power of two in [2^10, 2^30]";

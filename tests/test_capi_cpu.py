@@ -212,3 +212,46 @@ def test_tlc_checker_rejects_corruption(lib):
     bad[2][0] = ((((bad[2][0] >> 16) ^ 1)) << 16) | (bad[2][0] & 0xFFFF)
     res = OC.check_tlc(p, kappa, bad, r, c, h)
     assert not (res["viii_lane_is_source_bank"] and res["vii_sources_and_dests_cover_tile"])
+
+
+@pytest.mark.parametrize("k", [10, 13, 16, 19])
+def test_fp64_plan_is_the_word_pair_permutation(lib, k):
+    # Table II(b) (L731-L755): 8-byte elements; element i = words (2i, 2i+1) -> 2P(i)+h
+    n = 1 << k
+    p = W.random(n, k)
+    with lib.Plan(p, elem_bytes=8, device=False, layout=2 if k >= 14 else 0) as pl:
+        info = pl.info()
+        kappa, sched = pl.export()
+    assert info["elem_bytes"] == 8 and info["n"] == n
+    p2 = np.empty(2 * n, dtype=np.int64)
+    p2[0::2] = 2 * p.astype(np.int64)
+    p2[1::2] = 2 * p.astype(np.int64) + 1
+    r, c = W.view_shape(2 * n)
+    OC.assert_plan(p2, kappa.astype(np.int64), [decode(s) for s in sched], r, c, 32)
+
+
+def test_fp64_errors(lib):
+    with pytest.raises(lib.PermError) as e:
+        lib.Plan(np.array([0, 0] + list(range(2, 1024)), dtype=np.int32), elem_bytes=8, device=False)
+    assert e.value.status == -2
+
+
+def test_planner_is_deterministic_across_thread_counts(lib):
+    # sharded ranks colour P independently and must agree exactly (the parallel Euler
+    # split canonicalises every cycle's polarity and does not chunk by thread count)
+    import subprocess, sys, json
+    n = 1 << 21
+    code = (
+        "import sys, hashlib; sys.path.insert(0, %r)\n"
+        "import workloads as W, paper_conf_icpp_kasagini13_b200 as P\n"
+        "pl = P.Plan(W.random(%d, 3), device=False, layout=2)\n"
+        "k, s = pl.export()\n"
+        "print(hashlib.sha256(k.tobytes() + b''.join(x.tobytes() for x in s)).hexdigest())\n"
+    ) % (ROOT, n)
+    digests = set()
+    for threads in ("1", "3", "8"):
+        env = dict(os.environ, OMP_NUM_THREADS=threads)
+        out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env)
+        assert out.returncode == 0, out.stderr
+        digests.add(out.stdout.strip())
+    assert len(digests) == 1

@@ -269,3 +269,29 @@ def test_every_layout(P, layout, k):
     for fam_p in (p, W.bitrev(n)):
         b, info = run(P, fam_p, a, passes=3, layout=layout)
         assert np.array_equal(b, OA.apply_ref(fam_p, a)), (layout, k)
+
+
+@pytest.mark.parametrize("k", [10, 13, 16, 19, 21, 23])
+def test_fp64_elements(P, k):
+    # Table II(b): float64 payloads (raw 64-bit words), every family
+    n = 1 << k
+    a = W.make_data(n, 8)
+    for fam in W.FAMILIES:
+        p = W.make_perm(fam, n, seed=k)
+        with P.Plan(p, elem_bytes=8) as plan:
+            da = torch.from_numpy(a.view(np.int64)).cuda()
+            db = torch.full_like(da, -1)
+            plan.apply(da, db)
+            torch.cuda.synchronize()
+            got = db.cpu().numpy().view(np.uint64)
+        assert np.array_equal(got, OA.apply_ref(p, a)), (fam, k)
+    # conventional kernels on 8-byte elements
+    p = W.random(n, 1)
+    da = torch.from_numpy(a.view(np.int64)).cuda()
+    db = torch.empty_like(da)
+    P.scatter_baseline(torch.from_numpy(p).cuda(), da, db, elem_bytes=8)
+    torch.cuda.synchronize()
+    assert np.array_equal(db.cpu().numpy().view(np.uint64), OA.apply_ref(p, a))
+    P.gather_baseline(torch.from_numpy(OA.inverse(p)).cuda(), da, db, elem_bytes=8)
+    torch.cuda.synchronize()
+    assert np.array_equal(db.cpu().numpy().view(np.uint64), OA.apply_ref(p, a))
