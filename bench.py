@@ -301,7 +301,9 @@ def main():
         dB[f] = torch.empty_like(dA[f])
         dP[f] = torch.from_numpy(p).to(dev)
         host[f] = (p, a, np.empty(n, dtype=np.uint32))
-    info = plans[fams[0]].info()
+    infos = {f: plans[f].info() for f in fams}
+    sched_fams = [f for f in fams if not infos[f]["direct"]] or fams
+    info = infos[sched_fams[0]]
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
 
     def flush_l2():
@@ -373,23 +375,27 @@ def main():
         gather[f] = statistics.median(tg)
 
     # ---- per-kernel durations (events between kernels; PDL overlap disabled here)
-    kern = {f: [] for f in fams}
-    for f in fams:
+    # (families on the low-distribution shortcut run one scatter kernel, not the passes)
+    kern = {f: [] for f in sched_fams}
+    for f in sched_fams:
         plans[f].set_profiling(True)
         for _ in range(args.steps):
             flush_l2()
             plans[f].apply(dA[f], dB[f], stream)
             kern[f].append(plans[f].pass_times())
         plans[f].set_profiling(False)
-    nk = len(kern[fams[0]][0])
-    mean_k = [statistics.mean(kern[f][s][i] for f in fams for s in range(args.steps))
+    nk = min(len(kern[f][0]) for f in sched_fams)
+    mean_k = [statistics.mean(kern[f][s][i] for f in sched_fams for s in range(args.steps))
               for i in range(nk)]
     dom = int(np.argmax(mean_k))
     E = info["entry_bits"]
     # device schedule bytes per element of each phase (W64 format: floor(64/E) entries
     # per 64-bit word, ceil(32/epw) words per warp-round of 32 elements)
     sbpe = [8 * (-(-32 // (64 // e))) / 32 for e in E]
-    if info["kernels_per_apply"] == 1 and info["passes"] == 3:
+    if info["direct"]:
+        kinds = ["D-designated (direct)"]
+        alg = [2 * n * 4 + n * 4]
+    elif info["kernels_per_apply"] == 1 and info["passes"] == 3:
         kinds = ["fused R1+R2+R3"]
         alg = [2 * n * 4 + n * sum(sbpe)]
     elif info["passes"] == 3:
@@ -438,6 +444,24 @@ def main():
                "h2d_bytes_per_step": len(fams) * n * 4, "d2h_bytes_per_step": len(fams) * n * 4,
                "ms_per_step": e2e_s * 1e3}
 
+    # ---- the scheduled passes alone on the shortcut families (direct = -1)
+    sched_only = {}
+    for f in fams:
+        if not infos[f]["direct"]:
+            continue
+        pl = pkg.Plan(host[f][0], passes=args.passes, h=h, layout=args.layout, fuse=args.fuse,
+                      direct=-1)
+        for _ in range(3):
+            pl.apply(dA[f], dB[f], stream)
+        ts = []
+        for _ in range(args.steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            timed_apply(lambda: pl.apply(dA[f], dB[f], stream), e0, e1)
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        sched_only[f] = 1e3 * statistics.median(ts)
+        pl.close()
+
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
         cpu = cpu_oracle_baseline(host, n, args.cpu_seconds)
@@ -453,6 +477,9 @@ def main():
                      "kernels_per_apply": info["kernels_per_apply"], "h": info["h"],
                      "entry_bits": info["entry_bits"], "layout": plans[fams[0]].describe().get("layout")},
             "apply_us": per_fam_us,
+            "direct": {f: infos[f]["direct"] for f in fams},
+            "distribution_over_n": {f: infos[f]["distribution"] / n for f in fams},
+            "scheduled_only_us": sched_only,
             "conventional_us": {f: 1e3 * conv[f] for f in fams},
             "s_designated_us": {f: 1e3 * gather[f] for f in fams},
             "speedup_vs_conventional": {f: conv[f] * 1e3 / per_fam_us[f] for f in fams},
@@ -463,7 +490,7 @@ def main():
             "roofline": roofline,
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": args.steps * len(fams) * info["kernels_per_apply"],
+            "gpu_launches": args.steps * sum(infos[f]["kernels_per_apply"] for f in fams),
             "clocks": clocks.summary(),
             "wall_s_timed_region": t_wall,
         }

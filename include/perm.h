@@ -74,7 +74,11 @@ typedef struct {
                             chained with programmatic dependent launch); -1 = never */
     int32_t no_tma;      /* 1: use the plain (non-TMA) row-pass kernels of the 5-pass / sharded
                             structures even when a TMA stage fits (testing, A/B comparisons) */
-    int32_t reserved[4];
+    int32_t direct;      /* low-distribution shortcut (for P with
+                            D_w(P) <= 2n/w, e.g. identical and shuffle, the D-designated kernel
+                            is coalesced and faster): 0 = auto (on when D_w(P) <= 2n/32),
+                            -1 = never (always run the scheduled passes), 1 = always */
+    int32_t reserved[3];
 } perm_plan_options;
 
 typedef struct {
@@ -94,6 +98,9 @@ typedef struct {
     int32_t world, rank;         /* row sharding (1, 0 for unsharded plans) */
     int64_t shard_elems;         /* n / world */
     int64_t block_elems;         /* n / world^2: one all-to-all block */
+    int64_t distribution;        /* D_w(P), w = 32 (L389-L401): address groups the warps write */
+    int32_t direct;              /* 1: perm_apply runs the D-designated kernel (low D_w) */
+    int32_t pad0;
 } perm_plan_info;
 
 /* ------------------------------------------------------------------ plans */

@@ -35,6 +35,7 @@ struct perm_plan {
     unsigned long long* d_trace = nullptr;
     int64_t trace_stride = 0;          // CTAs per pass slot
     unsigned long long* d_sync = nullptr;   // fused 3-pass grid-barrier counters
+    int32_t* d_p = nullptr;                 // direct (D-designated) shortcut
     alignas(64) CUtensorMap tlc_maps[3];   // TLC layout: TMA tensor maps of X1, X2
 };
 
@@ -65,6 +66,7 @@ void free_device(perm_plan* pl) {
     cudaFree(pl->d_stage[1]);
     cudaFree(pl->d_trace);
     cudaFree(pl->d_sync);
+    cudaFree(pl->d_p);
     for (int i = 0; i < pl->n_events; ++i) cudaEventDestroy(pl->ev[i]);
     pl->n_events = 0;
     if (cur >= 0) cudaSetDevice(cur);
@@ -103,6 +105,13 @@ int upload(perm_plan* pl) {
     }
     e = perm::prepare_kernels(P);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute");
+    if (P.direct) {
+        e = cudaMalloc(&pl->d_p, P.p_copy.size() * sizeof(int32_t));
+        if (e == cudaSuccess)
+            e = cudaMemcpy(pl->d_p, P.p_copy.data(), P.p_copy.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) return cuda_fail(e, "upload p (direct)");
+        std::vector<int32_t>().swap(pl->host.p_copy);
+    }
     if (P.layout == 3) {
         e = perm::make_tlc_maps(P, pl->d_scratch[0], pl->d_scratch[1], pl->tlc_maps);
         if (e != cudaSuccess) return cuda_fail(e, "cuTensorMapEncodeTiled");
@@ -237,7 +246,9 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes == 1 ? 0 : 2 * P.n * P.eb);
     out->elem_bytes = P.user_eb;
     out->passes = P.passes;
-    out->kernels_per_apply = P.fused3 ? 1 : P.passes;
+    out->kernels_per_apply = (plan->d_p || P.fused3) ? 1 : P.passes;
+    out->distribution = P.distribution;
+    out->direct = P.direct;
     for (int f = 0; f < 3; ++f) {
         out->entry_bits[f] = P.layout == 3 ? P.tp[f].E : P.ph[f].E;
         out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
@@ -259,7 +270,9 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
     const HostPlan& P = plan->host;
     std::string s = "{\"n\":" + std::to_string(P.n) + ",\"rows\":" + std::to_string(P.r) +
                     ",\"cols\":" + std::to_string(P.c) + ",\"passes\":" + std::to_string(P.passes) +
-                    ",\"layout\":" + std::to_string(P.layout) + ",\"fused3\":" + std::to_string(P.fused3);
+                    ",\"layout\":" + std::to_string(P.layout) + ",\"fused3\":" + std::to_string(P.fused3) +
+                    ",\"distribution\":" + std::to_string(P.distribution) +
+                    ",\"direct\":" + std::to_string(P.direct);
     if (P.layout == 3) {
         s += ",\"tlc\":[";
         for (int f = 0; f < 3; ++f) {
@@ -428,7 +441,11 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
     cudaError_t e = cudaSuccess;
     int k = 0;   // index of the kernel being launched (for the error message)
     mark();
-    if (P.passes == 1) {
+    if (plan->d_p) {
+        // low distribution (D_w(P) <= 2n/w, L699-L701): the D-designated kernel is coalesced
+        e = perm::launch_scatter(plan->d_p, in, out, P.n, 4, s);
+        mark();
+    } else if (P.passes == 1) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
         e = perm::launch_fused(P, sc, in, out, s);
         mark();

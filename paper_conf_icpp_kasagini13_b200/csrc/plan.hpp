@@ -102,6 +102,10 @@ struct HostPlan {
     // row-sharded plans: this rank owns rows [rank*r_l, +r_l) of a and b,
     // and columns [rank*c_l, +c_l) in the column phase; schedules are sliced to those lines
     int32_t world = 1, rank = 0;
+    // low-distribution shortcut: D_w(P) <= 2n/w -> the D-designated kernel (coalesced)
+    int64_t distribution = 0;
+    int32_t direct = 0;
+    std::vector<int32_t> p_copy;   // uploaded for the direct kernel
     int64_t r_l = 0, c_l = 0;
     int64_t fused3_grid = 0;   // one CTA per SM (set at upload)
     PhaseGeom ph[3];

@@ -616,6 +616,25 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             seen[v] = 1;
         }
     }
+    {
+        // D_w(P) (L389-L401): distinct address groups of b written by each warp of 32
+        int64_t dw = 0;
+#pragma omp parallel for reduction(+ : dw) schedule(static)
+        for (int64_t wj = 0; wj < n / kW; ++wj) {
+            uint32_t g[kW];
+            for (int x = 0; x < kW; ++x) g[x] = (uint32_t)p[wj * kW + x] >> 5;
+            std::sort(g, g + kW);
+            int64_t d = 1;
+            for (int x = 1; x < kW; ++x) d += g[x] != g[x - 1];
+            dw += d;
+        }
+        P.distribution = dw;
+        const int dopt = opt ? opt->direct : 0;
+        if (dopt > 0 || (dopt == 0 && dw <= 2 * n / kW)) {
+            P.direct = 1;
+            P.p_copy.assign(p, p + n);
+        }
+    }
     P.n = n; P.eb = eb; P.k = k;
     P.r = int64_t(1) << (k / 2);
     P.c = int64_t(1) << (k - k / 2);
@@ -896,6 +915,8 @@ int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, i
     }
     P.world = world;
     P.rank = rank;
+    P.direct = 0;                       // the shortcut is a single-device kernel
+    P.p_copy.clear();
     P.r_l = r / world;
     P.c_l = c / world;
     const int64_t first[3] = {rank * P.r_l, rank * P.c_l, rank * P.r_l};

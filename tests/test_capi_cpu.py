@@ -255,3 +255,32 @@ def test_planner_is_deterministic_across_thread_counts(lib):
         assert out.returncode == 0, out.stderr
         digests.add(out.stdout.strip())
     assert len(digests) == 1
+
+
+@pytest.mark.parametrize("k", [10, 14, 16])
+def test_distribution_and_direct_shortcut(lib, k):
+    # D_w(P) reported by the planner equals the oracle's (L389-L401); the shortcut
+    # (L699-L701) is taken exactly when D_w(P) <= 2n/w unless forced either way
+    from oracle import distribution as OD
+    n = 1 << k
+    for fam in W.FAMILIES:
+        p = W.make_perm(fam, n, seed=k)
+        dw = OD.distribution(p, 32)
+        for eb in (4, 8):
+            pp = p if eb == 4 else np.stack([2 * p, 2 * p + 1], axis=1).reshape(-1).astype(np.int32)
+            want_dw = OD.distribution(pp, 32) if eb == 8 else dw
+            with lib.Plan(p, elem_bytes=eb, device=False) as pl:
+                inf = pl.info()
+                assert inf["distribution"] == want_dw, (fam, eb)
+                assert inf["direct"] == int(want_dw <= 2 * pp.size // 32), (fam, eb)
+                assert pl.describe()["direct"] == inf["direct"]
+        with lib.Plan(p, device=False, direct=-1) as pl:
+            assert pl.info()["direct"] == 0
+        with lib.Plan(p, device=False, direct=1) as pl:
+            assert pl.info()["direct"] == 1
+    # identity and shuffle are the paper's low-distribution cases
+    assert lib.Plan(W.identity(n), device=False).info()["direct"] == 1
+    assert lib.Plan(W.make_perm("shuffle", n), device=False).info()["direct"] == 1
+    assert lib.Plan(W.make_perm("bitrev", n), device=False).info()["direct"] == 0
+    if k >= 16:   # sharded plans never take the single-device shortcut
+        assert lib.Plan(W.identity(n), device=False, world=2, rank=0).info()["direct"] == 0

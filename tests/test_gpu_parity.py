@@ -33,6 +33,9 @@ def host_words(t) -> np.ndarray:
 
 
 def run(P, p, a, **kw):
+    # the parity tests exercise the scheduled passes on every family: the
+    # low-distribution shortcut (identity, shuffle) is tested on its own below
+    kw.setdefault("direct", -1)
     with P.Plan(p, **kw) as plan:
         da = dev(a)
         db = torch.full_like(da, -1)
@@ -278,7 +281,7 @@ def test_fp64_elements(P, k):
     a = W.make_data(n, 8)
     for fam in W.FAMILIES:
         p = W.make_perm(fam, n, seed=k)
-        with P.Plan(p, elem_bytes=8) as plan:
+        with P.Plan(p, elem_bytes=8, direct=-1) as plan:
             da = torch.from_numpy(a.view(np.int64)).cuda()
             db = torch.full_like(da, -1)
             plan.apply(da, db)
@@ -295,3 +298,27 @@ def test_fp64_elements(P, k):
     P.gather_baseline(torch.from_numpy(OA.inverse(p)).cuda(), da, db, elem_bytes=8)
     torch.cuda.synchronize()
     assert np.array_equal(db.cpu().numpy().view(np.uint64), OA.apply_ref(p, a))
+
+
+@pytest.mark.parametrize("k", [10, 14, 16, 22])
+@pytest.mark.parametrize("eb", [4, 8])
+def test_direct_shortcut(P, k, eb):
+    # for D_w(P) <= 2n/w (identical, shuffle) the D-designated
+    # kernel is the faster choice; the plan takes it by default and stays bit-exact
+    n = 1 << k
+    a = W.make_data(n, eb)
+    view = np.int32 if eb == 4 else np.int64
+    for fam, direct, want in (("identity", 0, 1), ("shuffle", 0, 1), ("random", 0, 0),
+                              ("random", 1, 1), ("bitrev", 1, 1), ("identity", -1, 0)):
+        p = W.make_perm(fam, n, seed=k)
+        with P.Plan(p, elem_bytes=eb, direct=direct) as plan:
+            info = plan.info()
+            assert info["direct"] == want, (fam, direct)
+            if want:
+                assert info["kernels_per_apply"] == 1
+            da = torch.from_numpy(a.view(view)).cuda()
+            db = torch.full_like(da, -1)
+            plan.apply(da, db)
+            torch.cuda.synchronize()
+            got = db.cpu().numpy().view(a.dtype)
+        assert np.array_equal(got, OA.apply_ref(p, a)), (fam, direct, k, eb)
