@@ -78,7 +78,9 @@ typedef struct {
                             D_w(P) <= 2n/w, e.g. identical and shuffle, the D-designated kernel
                             is coalesced and faster): 0 = auto (on when D_w(P) <= 2n/32),
                             -1 = never (always run the scheduled passes), 1 = always */
-    int32_t reserved[3];
+    int32_t log2c;       /* view r x c with c = 2^log2c (the view "is not
+                            restricted to a square matrix"); 0 = c = 2^ceil(k/2) */
+    int32_t reserved[2];
 } perm_plan_options;
 
 typedef struct {

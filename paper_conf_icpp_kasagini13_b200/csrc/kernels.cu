@@ -954,14 +954,6 @@ __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void*
         "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2)
         : "memory");
 }
-__device__ __forceinline__ void tma_store_4d(const CUtensorMap* map, const void* src, int c0, int c1, int c2,
-                                             int c3) {
-    asm volatile(
-        "cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
-            reinterpret_cast<uint64_t>(map)),
-        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
-        : "memory");
-}
 
 __host__ __device__ constexpr int cilog2(int v) { return v <= 1 ? 0 : 1 + cilog2(v >> 1); }
 
@@ -969,23 +961,99 @@ struct TlcArgs {
     const uint32_t* in;
     uint32_t* out;             // row-major output (OUT == 0)
     const uint32_t* sched;
-    int ntiles, stages;
+    int ntiles, na, nb;        // A slots (loads in flight), B slots (stores in flight)
     long long tile_words;      // schedule words per tile
-    int t_h;                   // lines per tile (tensor-store coordinates)
+    int chunk;                 // box rows per tile chunk (chunk words / box row words)
     int nbox, box_outer, box_words;
     unsigned long long* trace;
     int prefetch_in;           // stream the whole input into L2 up front (HBM-resident input)
 };
 
+// Shared-memory word offsets of the TLC rings: A slots, then B slots, then mbarriers.
+struct TlcRing {
+    uint32_t* A;
+    uint32_t* B;
+    uint64_t* afull;           // TMA bytes of A slot landed        (producer arms, TMA completes)
+    uint64_t* aempty;          // A slot read by all permuters      (kTlcPerm arrivals)
+    uint64_t* bfull;           // B slot written by all permuters   (kTlcPerm arrivals)
+    uint64_t* bempty;          // B slot read by its TMA store      (storer arrives)
+    __device__ TlcRing(uint32_t* smem, int HL, int na, int nb) {
+        A = smem;
+        B = smem + (size_t)na * HL;
+        afull = reinterpret_cast<uint64_t*>(B + (size_t)nb * HL);
+        aempty = afull + na;
+        bfull = aempty + na;
+        bempty = bfull + nb;
+    }
+    __device__ void init(int na, int nb) {
+        for (int s = 0; s < na; ++s) {
+            mbar_init(&afull[s], 1);
+            mbar_init(&aempty[s], kTlcPerm);
+        }
+        for (int s = 0; s < nb; ++s) {
+            mbar_init(&bfull[s], kTlcPerm);
+            mbar_init(&bempty[s], 1);
+        }
+        fence_mbar_init();
+    }
+};
+
+// TMA store of a permuted tile t from B slot `B` (see TlcArgs / make_tlc_maps):
+// kind 0 = one 1-D bulk store of a row-major tile, kind 1/2 = 3-D tensor stores
+// whose box rows are the tile's contiguous chunks (h1*h2 or h3*h2 words, split
+// into `chunk` rows of at most 256 words).
+__device__ __forceinline__ void tlc_store(int kind, const CUtensorMap* map, uint32_t* out, const uint32_t* B,
+                                          long long t, int HL, int chunk, int nbox, int box_outer,
+                                          int box_words) {
+    if (kind == 0) {
+        bulk_s2g(out + t * HL, B, (uint32_t)HL * 4u);
+    } else {
+        for (int b = 0; b < nbox; ++b)
+            tma_store_3d(map, B + b * box_words, 0, (int)(t * chunk), b * box_outer);
+    }
+    bulk_commit();
+}
+
+// Permute one tile: A (TMA-loaded, the pass's input order) -> B (the pass's
+// output order). Warp-round m of permuter warp pw: lane x reads A[32*sigma + x]
+// (bank x) and writes B[dst] (32 distinct banks per round, by construction of
+// the tile-level colouring). Entries are decoded from the lane's bitstream `wc`.
+template <int EPT>
+__device__ __forceinline__ void tlc_permute(const uint32_t* __restrict__ A, uint32_t* __restrict__ B,
+                                            const uint32_t* wc, uint64_t* aempty, uint64_t* bempty_wait,
+                                            uint32_t bparity, int lane) {
+    constexpr int HL = kTlcPerm * EPT;
+    constexpr int LOGHL = cilog2(HL);
+    constexpr int E = 2 * LOGHL - 5;
+    constexpr uint32_t EMASK = (1u << E) - 1u;
+    uint32_t v[EPT];
+    uint32_t d[EPT];
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) {
+        const int bit = m * E, w = bit >> 5, off = bit & 31;
+        uint32_t e;
+        if (off + E <= 32) e = (wc[w] >> off) & EMASK;
+        else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
+        v[m] = A[((e >> LOGHL) << 5) | lane];
+        d[m] = e & (HL - 1);
+    }
+    mbar_arrive(aempty);                      // A slot may be refilled
+    if (bempty_wait) mbar_wait(bempty_wait, bparity);
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
+    fence_proxy_async();                      // generic-proxy writes -> the TMA store's reads
+}
+
 // One row-wise permutation pass (Lemma 7) with the tile-level bank colouring
-// (plan.hpp TlcPass). A tile of h lines is TMA-loaded into A in its global
-// order; 512 permuter threads move every element A[src] -> B[dst] in
+// (plan.hpp TlcPass). A tile of h lines is TMA-loaded into an A slot in its
+// global order; 512 permuter threads move every element A[src] -> B[dst] in
 // warp-rounds that touch 32 distinct banks of A and 32 distinct banks of B;
 // B is already in the global order of the output, so the transposes of the
 // column-wise step (Lemma 8) cost nothing extra: B leaves by TMA (1-D bulk
-// store for row-major output, 3-D / 4-D tensor stores of 64-byte chunks for
-// the intermediates). Roles: warp 0 lane 0 = TMA producer, warp 1 lane 0 =
-// TMA storer, warps 2..17 = permuters; `stages` slots of [A | B].
+// store for row-major output, 2-D tensor stores of 64-byte chunks for the
+// intermediates). Roles: warp 0 lane 0 = TMA producer, warp 1 lane 0 = TMA
+// storer, warps 2..17 = permuters. Separate rings: `na` A slots (a CTA's whole
+// share of tiles is requested up front when it fits) and `nb` B slots.
 template <int EPT, int OUT>
 __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     row_pass_tlc_kernel(const __grid_constant__ CUtensorMap tmap, const TlcArgs a) {
@@ -993,32 +1061,22 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     constexpr int LOGHL = cilog2(HL);
     constexpr int E = 2 * LOGHL - 5;
     constexpr int NWORDS = (EPT * E + 31) / 32;
-    constexpr uint32_t EMASK = (1u << E) - 1u;
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int NS = a.stages;
+    const int NA = a.na, NB = a.nb;
     const int G = gridDim.x;
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * 2 * HL);
-    uint64_t* permd = full + NS;
-    uint64_t* empty = permd + NS;
+    TlcRing R(smem, HL, NA, NB);
     unsigned long long* tr = a.trace;
     stamp(tr, 0);
-    if (tid == 0) {
-        for (int s = 0; s < NS; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&permd[s], kTlcPerm);
-            mbar_init(&empty[s], 1);
-        }
-        fence_mbar_init();
-    }
+    if (tid == 0) R.init(NA, NB);
     __syncthreads();
 
     if (warp == 0) {
         if (lane == 0) {
             // ---------------- producer
-            // Deep memory-level parallelism without shared memory: every schedule chunk of
-            // this CTA (independent of the previous pass) and, for HBM-resident input, every
-            // input tile are requested into L2 now; the smem ring then streams from L2.
+            // every schedule chunk of this CTA (independent of the previous pass) is
+            // requested into L2 now; for HBM-resident input, so are the input tiles
+            // beyond the ring
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
@@ -1027,7 +1085,7 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             pdl_wait();
             stamp(tr, 1);
             if (a.prefetch_in) {
-                for (int i = NS;; ++i) {
+                for (int i = NA;; ++i) {
                     const long long t = blockIdx.x + (long long)i * G;
                     if (t >= a.ntiles) break;
                     prefetch_l2_bulk(a.in + t * HL, (uint32_t)HL * 4u);
@@ -1036,94 +1094,63 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
-                const int s = i % NS;
-                if (i >= NS) mbar_wait(&empty[s], (uint32_t)(i / NS - 1) & 1u);
-                fence_proxy_async();
-                mbar_arrive_expect_tx(&full[s], (uint32_t)HL * 4u);
-                bulk_g2s(smem + s * 2 * HL, a.in + t * HL, (uint32_t)HL * 4u, &full[s]);
+                const int s = i % NA;
+                if (i >= NA) mbar_wait(&R.aempty[s], (uint32_t)(i / NA - 1) & 1u);
+                fence_proxy_async();           // permuters' generic reads of the slot -> TMA write
+                mbar_arrive_expect_tx(&R.afull[s], (uint32_t)HL * 4u);
+                bulk_g2s(R.A + (size_t)s * HL, a.in + t * HL, (uint32_t)HL * 4u, &R.afull[s]);
                 if (i == 0) pdl_launch_dependents();
             }
         }
     } else if (warp == 1) {
         if (lane == 0) {
-            // ---------------- storer (stores stay one tile deep in flight)
+            // ---------------- storer: at most one store un-read while the next is issued
             pdl_wait();
-            int pend_s = -1;
+            int prev = -1;
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
-                const int s = i % NS;
-                mbar_wait(&permd[s], (uint32_t)(i / NS) & 1u);
-                fence_proxy_async();       // permuters' smem writes -> async-proxy reads
-                const uint32_t* B = smem + s * 2 * HL + HL;
-                if constexpr (OUT == 0) {
-                    bulk_s2g(a.out + t * HL, B, (uint32_t)HL * 4u);
-                } else if constexpr (OUT == 1) {
-                    for (int b = 0; b < a.nbox; ++b)
-                        tma_store_3d(&tmap, B + b * a.box_words, 0, (int)(t * a.t_h), b * a.box_outer);
-                } else {
-                    for (int b = 0; b < a.nbox; ++b)
-                        tma_store_4d(&tmap, B + b * a.box_words, 0, 0, (int)t, b * a.box_outer);
-                }
-                bulk_commit();
-                if (NS == 1) {                 // a single slot cannot wait for the next tile
+                const int s = i % NB;
+                mbar_wait(&R.bfull[s], (uint32_t)(i / NB) & 1u);
+                tlc_store(OUT, &tmap, a.out, R.B + (size_t)s * HL, t, HL, a.chunk, a.nbox, a.box_outer,
+                          a.box_words);
+                if (NB == 1) {
                     bulk_wait_read0();
-                    mbar_arrive(&empty[s]);
+                    mbar_arrive(&R.bempty[s]);
                 } else {
-                    if (pend_s >= 0) {
+                    if (prev >= 0) {
                         bulk_wait_read1();
-                        mbar_arrive(&empty[pend_s]);
+                        mbar_arrive(&R.bempty[prev]);
                     }
-                    pend_s = s;
+                    prev = s;
                 }
                 if (i < 4) stamp_if(tr, true, 4 + 3 * i);
-            }
-            if (pend_s >= 0) {
-                bulk_wait_read0();
-                mbar_arrive(&empty[pend_s]);
             }
             bulk_wait0();
         }
     } else {
         // ---------------- permuters
-        const int pw = warp - 2;
         const bool lead = tid == 64;
-        const uint32_t* sp = a.sched + pw * NWORDS * 32 + lane;
+        const uint32_t* sp = a.sched + (warp - 2) * NWORDS * 32 + lane;
         uint32_t wc[NWORDS], wn[NWORDS];
-        {
-            const long long t = blockIdx.x;
-            if (t < a.ntiles) {
+        if (blockIdx.x < a.ntiles) {
 #pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + t * a.tile_words + w * 32);
-            }
+            for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + (long long)blockIdx.x * a.tile_words + w * 32);
         }
         for (int i = 0;; ++i) {
             const long long t = blockIdx.x + (long long)i * G;
             if (t >= a.ntiles) break;
-            const int s = i % NS;
+            const int s = i % NA, sb = i % NB;
             const long long tn = t + G;
             if (tn < a.ntiles) {
 #pragma unroll
                 for (int w = 0; w < NWORDS; ++w) wn[w] = __ldg(sp + tn * a.tile_words + w * 32);
             }
-            mbar_wait(&full[s], (uint32_t)(i / NS) & 1u);
+            mbar_wait(&R.afull[s], (uint32_t)(i / NA) & 1u);
             if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
-            const uint32_t* __restrict__ A = smem + s * 2 * HL;
-            uint32_t* __restrict__ B = smem + s * 2 * HL + HL;
-            uint32_t v[EPT];
-            uint32_t d[EPT];
-#pragma unroll
-            for (int m = 0; m < EPT; ++m) {
-                const int bit = m * E, w = bit >> 5, off = bit & 31;
-                uint32_t e;
-                if (off + E <= 32) e = (wc[w] >> off) & EMASK;
-                else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
-                v[m] = A[((e >> LOGHL) << 5) | lane];
-                d[m] = e & (HL - 1);
-            }
-#pragma unroll
-            for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
-            mbar_arrive(&permd[s]);
+            tlc_permute<EPT>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wc, &R.aempty[s],
+                             i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
+            mbar_arrive(&R.bfull[sb]);
 #pragma unroll
             for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
         }
@@ -1139,26 +1166,26 @@ struct TlcPassCfg {
     uint32_t* out;             // row-major output (kind 0)
     const uint32_t* sched;
     int ntiles;
-    int kind;                  // 0: rows (1-D bulk store), 1: X1 3-D tensor, 2: X2 4-D tensor
-    int t_h, nbox, box_outer, box_words;
+    int kind;                  // 0: rows (1-D bulk store), 1: X1, 2: X2 (3-D tensor stores)
+    int chunk, nbox, box_outer, box_words;
 };
 
 struct TlcFusedArgs {
     TlcPassCfg p[3];
     long long tile_words;
-    int stages;
+    int na, nb;
     unsigned long long* sync;  // [0], [1]: barrier arrivals after pass 0 / 1; [2]: exits
     unsigned long long* trace;
 };
 
 // Thm 9 in ONE persistent launch with the TLC passes (square views: the three
-// passes share the tile size HL). Same roles and slot ring as
-// row_pass_tlc_kernel, continued across passes (global tile sequence j). The
-// storer publishes a CTA's pass-k output once its bulk stores have COMPLETED
-// (wait_group 0, then a release at gpu scope on sync[k]); the producer TMA-loads
-// pass k+1 data only after sync[k] reaches the grid size (schedule prefetches go
-// ahead of the barrier). One co-resident CTA per SM; the last CTA out resets
-// the counters, so the launch is replayable (CUDA graphs).
+// passes share the tile size HL). Same roles and rings as row_pass_tlc_kernel,
+// continued across passes (global tile sequence j). The storer publishes a
+// CTA's pass-k output once its bulk stores have COMPLETED (wait_group 0, then a
+// release at gpu scope on sync[k]); the producer TMA-loads pass k+1 data only
+// after sync[k] reaches the grid size (schedule prefetches go ahead of the
+// barrier). One co-resident CTA per SM; the last CTA out resets the counters,
+// so the launch is replayable (CUDA graphs).
 template <int EPT>
 __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     fused_tlc_kernel(const __grid_constant__ CUtensorMap map_x1,
@@ -1167,24 +1194,14 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     constexpr int LOGHL = cilog2(HL);
     constexpr int E = 2 * LOGHL - 5;
     constexpr int NWORDS = (EPT * E + 31) / 32;
-    constexpr uint32_t EMASK = (1u << E) - 1u;
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int NS = a.stages;
+    const int NA = a.na, NB = a.nb;
     const int G = gridDim.x;
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * 2 * HL);
-    uint64_t* permd = full + NS;
-    uint64_t* empty = permd + NS;
+    TlcRing R(smem, HL, NA, NB);
     unsigned long long* tr = a.trace;
     stamp(tr, 0);
-    if (tid == 0) {
-        for (int s = 0; s < NS; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&permd[s], kTlcPerm);
-            mbar_init(&empty[s], 1);
-        }
-        fence_mbar_init();
-    }
+    if (tid == 0) R.init(NA, NB);
     __syncthreads();
     auto my_tiles = [&](int k) -> int {
         const int nt = a.p[k].ntiles - (int)blockIdx.x;
@@ -1194,73 +1211,68 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     if (warp == 0) {
         if (lane == 0) {
             // ---------------- producer
-            for (int i = 0; i < my_tiles(0) && i <= NS; ++i)
-                prefetch_l2_bulk(a.p[0].sched + (blockIdx.x + (long long)i * G) * a.tile_words,
-                                 (uint32_t)(a.tile_words * 4));
+            // every schedule of this CTA is independent of the data: pass 0's is requested
+            // first, passes 1 and 2 right after the first ring of pass-0 loads
+            auto prefetch_sched = [&](int k) {
+                for (int i = 0; i < my_tiles(k); ++i)
+                    prefetch_l2_bulk(a.p[k].sched + (blockIdx.x + (long long)i * G) * a.tile_words,
+                                     (uint32_t)(a.tile_words * 4));
+            };
+            prefetch_sched(0);
+            const int first_ring = my_tiles(0) < NA ? my_tiles(0) : NA;
+            if (first_ring == 0) { prefetch_sched(1); prefetch_sched(2); }
             int j = 0;
             for (int k = 0; k < 3; ++k) {
                 const TlcPassCfg& pc = a.p[k];
                 const int nt = my_tiles(k);
                 if (k > 0) {
-                    for (int i = 0; i < nt; ++i)      // next pass's schedules: independent of data
-                        prefetch_l2_bulk(pc.sched + (blockIdx.x + (long long)i * G) * a.tile_words,
-                                         (uint32_t)(a.tile_words * 4));
                     while (ld_acquire_gpu(&a.sync[k - 1]) < (unsigned long long)G) __nanosleep(32);
                     fence_proxy_async_global();
                     stamp(tr, 1 + 4 * k);
                 }
                 for (int i = 0; i < nt; ++i, ++j) {
                     const long long t = blockIdx.x + (long long)i * G;
-                    const int s = j % NS;
-                    if (j >= NS) mbar_wait(&empty[s], (uint32_t)(j / NS - 1) & 1u);
-                    fence_proxy_async();
-                    mbar_arrive_expect_tx(&full[s], (uint32_t)HL * 4u);
-                    bulk_g2s(smem + s * 2 * HL, pc.in + t * HL, (uint32_t)HL * 4u, &full[s]);
+                    const int s = j % NA;
+                    if (j >= NA) mbar_wait(&R.aempty[s], (uint32_t)(j / NA - 1) & 1u);
+                    fence_proxy_async();       // permuters' generic reads of the slot -> TMA write
+                    mbar_arrive_expect_tx(&R.afull[s], (uint32_t)HL * 4u);
+                    bulk_g2s(R.A + (size_t)s * HL, pc.in + t * HL, (uint32_t)HL * 4u, &R.afull[s]);
+                    if (k == 0 && i + 1 == first_ring) { prefetch_sched(1); prefetch_sched(2); }
                 }
             }
         }
     } else if (warp == 1) {
         if (lane == 0) {
-            // ---------------- storer (stores stay one tile deep in flight)
+            // ---------------- storer
             int j = 0;
-            int pend_s = -1;                 // slot of the previous, not yet released store
+            int prev = -1;                   // B slot of the previous, not yet released store
             for (int k = 0; k < 3; ++k) {
                 const TlcPassCfg& pc = a.p[k];
+                const CUtensorMap* map = pc.kind == 2 ? &map_x2 : &map_x1;
                 const int nt = my_tiles(k);
                 for (int i = 0; i < nt; ++i, ++j) {
                     const long long t = blockIdx.x + (long long)i * G;
-                    const int s = j % NS;
-                    mbar_wait(&permd[s], (uint32_t)(j / NS) & 1u);
-                    fence_proxy_async();
-                    const uint32_t* B = smem + s * 2 * HL + HL;
-                    if (pc.kind == 0) {
-                        bulk_s2g(pc.out + t * HL, B, (uint32_t)HL * 4u);
-                    } else if (pc.kind == 1) {
-                        for (int b = 0; b < pc.nbox; ++b)
-                            tma_store_3d(&map_x1, B + b * pc.box_words, 0, (int)(t * pc.t_h), b * pc.box_outer);
-                    } else {
-                        for (int b = 0; b < pc.nbox; ++b)
-                            tma_store_4d(&map_x2, B + b * pc.box_words, 0, 0, (int)t, b * pc.box_outer);
-                    }
-                    bulk_commit();
-                    if (NS == 1) {
+                    const int s = j % NB;
+                    mbar_wait(&R.bfull[s], (uint32_t)(j / NB) & 1u);
+                    tlc_store(pc.kind, map, pc.out, R.B + (size_t)s * HL, t, HL, pc.chunk, pc.nbox,
+                              pc.box_outer, pc.box_words);
+                    if (NB == 1) {
                         bulk_wait_read0();
-                        mbar_arrive(&empty[s]);
+                        mbar_arrive(&R.bempty[s]);
                     } else {
-                        if (pend_s >= 0) {
+                        if (prev >= 0) {
                             bulk_wait_read1();       // the previous store has read its slot
-                            mbar_arrive(&empty[pend_s]);
+                            mbar_arrive(&R.bempty[prev]);
                         }
-                        pend_s = s;
+                        prev = s;
                     }
-                }
-                if (pend_s >= 0) {
-                    bulk_wait_read0();
-                    mbar_arrive(&empty[pend_s]);
-                    pend_s = -1;
                 }
                 if (k < 2) {
                     bulk_wait0();                    // this CTA's pass-k output is written
+                    if (prev >= 0) {
+                        mbar_arrive(&R.bempty[prev]);
+                        prev = -1;
+                    }
                     fence_proxy_async_global();
                     __threadfence();
                     red_release_gpu_add(&a.sync[k], 1ull);
@@ -1271,43 +1283,29 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         }
     } else {
         // ---------------- permuters
-        const int pw = warp - 2;
         const bool lead = tid == 64;
         int j = 0;
         for (int k = 0; k < 3; ++k) {
             const TlcPassCfg& pc = a.p[k];
             const int nt = my_tiles(k);
-            const uint32_t* sp = pc.sched + pw * NWORDS * 32 + lane;
+            const uint32_t* sp = pc.sched + (warp - 2) * NWORDS * 32 + lane;
             uint32_t wc[NWORDS], wn[NWORDS];
             if (nt > 0) {
 #pragma unroll
                 for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + (long long)blockIdx.x * a.tile_words + w * 32);
             }
             for (int i = 0; i < nt; ++i, ++j) {
-                const int s = j % NS;
+                const int s = j % NA, sb = j % NB;
                 if (i + 1 < nt) {
                     const long long tn = blockIdx.x + (long long)(i + 1) * G;
 #pragma unroll
                     for (int w = 0; w < NWORDS; ++w) wn[w] = __ldg(sp + tn * a.tile_words + w * 32);
                 }
-                mbar_wait(&full[s], (uint32_t)(j / NS) & 1u);
+                mbar_wait(&R.afull[s], (uint32_t)(j / NA) & 1u);
                 if (i == 0) stamp_if(tr, lead, 2 + 4 * k);
-                const uint32_t* __restrict__ A = smem + s * 2 * HL;
-                uint32_t* __restrict__ B = smem + s * 2 * HL + HL;
-                uint32_t v[EPT];
-                uint32_t d[EPT];
-#pragma unroll
-                for (int m = 0; m < EPT; ++m) {
-                    const int bit = m * E, w = bit >> 5, off = bit & 31;
-                    uint32_t e;
-                    if (off + E <= 32) e = (wc[w] >> off) & EMASK;
-                    else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
-                    v[m] = A[((e >> LOGHL) << 5) | lane];
-                    d[m] = e & (HL - 1);
-                }
-#pragma unroll
-                for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
-                mbar_arrive(&permd[s]);
+                tlc_permute<EPT>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wc, &R.aempty[s],
+                                 j >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(j / NB - 1) & 1u, lane);
+                mbar_arrive(&R.bfull[sb]);
 #pragma unroll
                 for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
             }
@@ -1548,7 +1546,7 @@ cudaError_t prep_fused3(HostPlan& P) {
 
 size_t tlc_smem(const HostPlan& P, int f) {
     const TlcPass& tp = P.tp[f];
-    return (size_t)tp.stages * 2 * tp.HL * 4 + (size_t)tp.stages * 8 * 3;
+    return (size_t)(tp.stages + tp.bslots) * tp.HL * 4 + (size_t)(tp.stages + tp.bslots) * 8 * 2;
 }
 
 template <int EPT, int OUT>
@@ -1625,24 +1623,23 @@ cudaError_t make_tlc_maps(const HostPlan& P, uint32_t* x1, uint32_t* x2, CUtenso
     const cuuint64_t r = (cuuint64_t)P.r, c = (cuuint64_t)P.c;
     const cuuint64_t h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
     std::memset(maps, 0, 3 * sizeof(CUtensorMap));
-    {   // X1 = [K][i][k_in]: dims (k_in, i, K)
-        const cuuint64_t dims[3] = {h2, r, c / h2};
-        const cuuint64_t strides[2] = {h2 * 4, r * h2 * 4};
-        const cuuint32_t box[3] = {(cuuint32_t)h2, (cuuint32_t)h1,
-                                   (cuuint32_t)std::min<cuuint64_t>(256, c / h2)};
+    // Maps whose box rows are a tile's contiguous chunks (64 bytes at h1*h2 = 16 words; at
+    // most 256 words per row): a 16-byte innermost box dimension makes the TMA unit emit
+    // 16-byte rows (measured 1.5x slower per pass, scripts/micro/tile_io.py).
+    //   X1 = [K][i][k_in]: K-blocks of r*h2 words; pass-1 tile t writes [t*h1*h2, +h1*h2) of each
+    //   X2 = [I'][K][i_in'][k_in]: I'-blocks of c*h3 words; pass-2 tile K writes [K*h3*h2, +h3*h2)
+    const cuuint64_t ch[2] = {h1 * h2, h3 * h2};
+    const cuuint64_t blk[2] = {r * h2, c * h3};
+    const cuuint64_t nblk[2] = {c / h2, r / h3};
+    void* base[2] = {x1, x2};
+    for (int m = 0; m < 2; ++m) {
+        const cuuint64_t rw = std::min<cuuint64_t>(ch[m], 256);
+        const cuuint64_t dims[3] = {rw, blk[m] / rw, nblk[m]};
+        const cuuint64_t strides[2] = {rw * 4, blk[m] * 4};
+        const cuuint32_t box[3] = {(cuuint32_t)rw, (cuuint32_t)(ch[m] / rw),
+                                   (cuuint32_t)std::min<cuuint64_t>(256, nblk[m])};
         const cuuint32_t es[3] = {1, 1, 1};
-        if (encode(&maps[0], CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, x1, dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                   CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-            return cudaErrorInvalidValue;
-    }
-    {   // X2 = [I'][K][i_in'][k_in]: dims (k_in, i_in', K, I')
-        const cuuint64_t dims[4] = {h2, h3, c / h2, r / h3};
-        const cuuint64_t strides[3] = {h2 * 4, h3 * h2 * 4, c * h3 * 4};
-        const cuuint32_t box[4] = {(cuuint32_t)h2, (cuuint32_t)h3, 1,
-                                   (cuuint32_t)std::min<cuuint64_t>(256, r / h3)};
-        const cuuint32_t es[4] = {1, 1, 1, 1};
-        if (encode(&maps[1], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, x2, dims, strides, box, es,
+        if (encode(&maps[m], CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, base[m], dims, strides, box, es,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                    CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
             return cudaErrorInvalidValue;
@@ -1659,9 +1656,9 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
     ta.out = out;
     ta.sched = sched;
     ta.ntiles = (int)tp.ntiles;
-    ta.stages = tp.stages;
+    ta.na = tp.stages;
+    ta.nb = tp.bslots;
     ta.tile_words = tp.tile_words;
-    ta.t_h = tp.h;
     ta.trace = trace;
     ta.prefetch_in = (f == 0) ? 1 : 0;   // pass 1 reads `a` from HBM; later passes read L2-resident X
     const long long h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
@@ -1670,11 +1667,13 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
         ta.box_outer = (int)bo;
         ta.nbox = (int)(outer / bo);
         ta.box_words = (int)(bo * h1 * h2);
+        ta.chunk = (int)(h1 * h2 / std::min<long long>(h1 * h2, 256));
     } else if (tp.out_kind == 2) {
         const long long outer = P.r / h3, bo = outer < 256 ? outer : 256;
         ta.box_outer = (int)bo;
         ta.nbox = (int)(outer / bo);
         ta.box_words = (int)(bo * h3 * h2);
+        ta.chunk = (int)(h3 * h2 / std::min<long long>(h3 * h2, 256));
     }
     const CUtensorMap& map = maps[tp.out_kind == 2 ? 1 : 0];
     const dim3 grid((unsigned)tp.grid), block(64 + kTlcPerm);
@@ -1708,21 +1707,23 @@ cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const u
         pc.sched = sched[f];
         pc.ntiles = (int)tp.ntiles;
         pc.kind = tp.out_kind;
-        pc.t_h = tp.h;
         if (tp.out_kind == 1) {
             const long long outer = P.c / h2, bo = outer < 256 ? outer : 256;
             pc.box_outer = (int)bo;
             pc.nbox = (int)(outer / bo);
             pc.box_words = (int)(bo * h1 * h2);
+            pc.chunk = (int)(h1 * h2 / std::min<long long>(h1 * h2, 256));
         } else if (tp.out_kind == 2) {
             const long long outer = P.r / h3, bo = outer < 256 ? outer : 256;
             pc.box_outer = (int)bo;
             pc.nbox = (int)(outer / bo);
             pc.box_words = (int)(bo * h3 * h2);
+            pc.chunk = (int)(h3 * h2 / std::min<long long>(h3 * h2, 256));
         }
     }
     fa.tile_words = P.tp[0].tile_words;
-    fa.stages = P.tp[0].stages;
+    fa.na = P.tp[0].stages;
+    fa.nb = P.tp[0].bslots;
     fa.sync = sync;
     fa.trace = trace;
     const dim3 grid((unsigned)P.fused3_grid), block(64 + kTlcPerm);

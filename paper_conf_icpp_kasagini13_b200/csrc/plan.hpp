@@ -83,8 +83,9 @@ struct TlcPass {
     int32_t nwords = 0;       // ceil(ept * E / 32)
     int64_t ntiles = 0;
     int64_t tile_words = 0;   // (kTlcPerm / 32) * nwords * 32
-    int32_t out_kind = 0;     // 0: rows (1-D bulk store); 1: X1 3-D tensor store; 2: X2 4-D tensor store
-    int32_t stages = 0;
+    int32_t out_kind = 0;     // 0: rows (1-D bulk store); 1: X1 / 2: X2 2-D tensor store (64-byte box rows)
+    int32_t stages = 0;       // A slots (TMA loads in flight); B slots = bslots
+    int32_t bslots = 0;       // B slots (permuted tiles waiting for / under their TMA store)
     int64_t grid = 0;         // persistent CTAs (set at upload)
 };
 

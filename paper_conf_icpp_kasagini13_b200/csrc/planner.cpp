@@ -498,10 +498,16 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
         tp.ntiles = P.ph[f].lines / hs[f];
         tp.tile_words = (int64_t)(kTlcPerm / 32) * tp.nwords * 32;
         tp.out_kind = f == 0 ? 1 : (f == 1 ? 2 : 0);
-        const int64_t stage = 2 * (int64_t)tp.HL * 4;
-        int st = stages_opt ? stages_opt : (int)std::min<int64_t>(4, (220 * 1024) / stage);
-        if (st < 1 || st * stage > 220 * 1024) { err = "TLC layout: stages do not fit in shared memory"; return PERM_EINVAL; }
+        // separate rings: A slots take TMA loads (a CTA's whole share of tiles in flight
+        // when it fits), B slots hold permuted tiles until their TMA store has read them
+        const int64_t slot = (int64_t)tp.HL * 4;
+        const int64_t budget = 220 * 1024;
+        const int nb = slot * 4 <= budget ? 2 : 1;
+        const int64_t fit = budget / slot - nb;
+        int st = stages_opt ? stages_opt : (int)std::min<int64_t>(6, fit);
+        if (st < 1 || (st + nb) * slot > budget) { err = "TLC layout: stages do not fit in shared memory"; return PERM_EINVAL; }
         tp.stages = st;
+        tp.bslots = nb;
         // keep the generic RowPass view consistent for info/describe
         RowPass& rp = P.rp[f];
         rp.phase = f; rp.h = tp.h; rp.ctas = tp.ntiles; rp.tma = 3; rp.stages = st;
@@ -636,10 +642,12 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         }
     }
     P.n = n; P.eb = eb; P.k = k;
-    P.r = int64_t(1) << (k / 2);
-    P.c = int64_t(1) << (k - k / 2);
+    // view r x c (L603: "not restricted to a square matrix"); default c = 2^ceil(k/2)
+    const int logc = (opt && opt->log2c > 0) ? opt->log2c : k - k / 2, logr = k - logc;
+    if (logc < 5 || logr < 5) { err = "view: log2c must leave r, c >= 32"; return PERM_EINVAL; }
+    P.r = int64_t(1) << logr;
+    P.c = int64_t(1) << logc;
     const int64_t r = P.r, c = P.c;
-    const int logc = k - k / 2, logr = k / 2;
 #ifdef _OPENMP
     P.threads_used = omp_get_max_threads();
 #endif
@@ -729,8 +737,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 
     // pass structure
     int passes = opt ? opt->passes : 0;
-    // measured on B200: fused CTA to 2^14, TLC 3-pass 2^15..2^22, LINES
-    // 3-pass 2^23..2^24, the paper's 5-pass structure (TMA row passes) from 2^25
+    // measured on B200: fused CTA to 2^14, TLC 3-pass 2^15..2^24 (LINES /
+    // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^25
     if (passes == 0) passes = (k <= 14) ? 1 : (k <= 24 ? 3 : 5);
     if (passes == 1 && k > 14) { err = "fused single-CTA pass needs n <= 2^14"; return PERM_EUNSUPPORTED; }
     if (passes != 1 && passes != 3 && passes != 5) { err = "passes must be 0, 1, 3 or 5"; return PERM_EINVAL; }
@@ -746,13 +754,14 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     }
     {
         int layout0 = opt ? opt->layout : 0;
-        if (passes == 3 && (layout0 == 3 || (layout0 == 0 && k >= 15 && k <= 22))) {
+        if (passes == 3 && (layout0 == 3 || (layout0 == 0 && k >= 15 && k <= 24))) {
             const int st = build_tlc(P, phi, opt, err);
             P.ms_bank = ms_since(t0);
             // one persistent launch when the three passes share the tile size (square view)
             const int fuse = opt ? opt->fuse : 0;
             if (st == PERM_OK && fuse > 0 && P.tp[0].HL == P.tp[1].HL && P.tp[1].HL == P.tp[2].HL &&
-                P.tp[0].stages == P.tp[1].stages && P.tp[1].stages == P.tp[2].stages)
+                P.tp[0].stages == P.tp[1].stages && P.tp[1].stages == P.tp[2].stages &&
+                P.tp[0].bslots == P.tp[1].bslots && P.tp[1].bslots == P.tp[2].bslots)
                 P.fused3 = 1;
             return st;
         }

@@ -195,6 +195,19 @@ def test_tlc_plan_22(lib):
     assert all(res.values()), res
 
 
+@pytest.mark.parametrize("k,log2c,h", [(16, 10, (0, 0, 0)), (16, 6, (0, 0, 0)), (18, 12, (1, 64, 1)),
+                                         (19, 12, (2, 64, 2))])
+def test_tlc_non_square_view(lib, k, log2c, h):
+    # the r x c view "is not restricted to a square matrix"
+    n = 1 << k
+    r, c = n >> log2c, 1 << log2c
+    p = W.make_perm("random", n, seed=k)
+    info, d, kappa, sched = export_tlc(lib, p, log2c=log2c, h=h)
+    assert (info["rows"], info["cols"]) == (r, c)
+    res = OC.check_tlc(p, kappa, sched, r, c, tuple(info["h"]))
+    assert all(res.values()), res
+
+
 def test_tlc_checker_rejects_corruption(lib):
     n = 1 << 16
     r, c = W.view_shape(n)

@@ -322,3 +322,28 @@ def test_direct_shortcut(P, k, eb):
             torch.cuda.synchronize()
             got = db.cpu().numpy().view(a.dtype)
         assert np.array_equal(got, OA.apply_ref(p, a)), (fam, direct, k, eb)
+
+
+# TLC ring configurations: tiles per CTA > A slots and > B slots, so both rings wrap
+# (a missing async-proxy fence before a slot's TMA refill only shows up then)
+@pytest.mark.parametrize("k,h,stages,fuse,log2c", [
+    (20, (16, 16, 16), 1, 0, 0),      # EPT 32, NA 1, NB 1
+    (20, (8, 8, 8), 1, 0, 0),         # EPT 16, NA 1, NB 2
+    (22, (8, 8, 8), 0, 0, 0),         # EPT 32, NA 2, NB 1, ~2 tiles per CTA
+    (22, (2, 4, 2), 0, 0, 0),         # EPT 8 / 16 / 8, NA 6, ~7 tiles per CTA, 32-byte chunks
+    (22, (2, 2, 2), 0, 0, 0),         # rejected: h2 < 4
+    (22, (4, 4, 4), 2, 1, 0),         # fused single launch, NA 2
+    (24, (4, 4, 4), 0, 0, 0),         # EPT 32, ~7 tiles per CTA
+    (24, (4, 4, 4), 0, 1, 0),
+    (24, (1, 4, 1), 0, 0, 13),        # non-square view 2048 x 8192, 16-byte chunks
+])
+def test_tlc_rings_wrap(P, k, h, stages, fuse, log2c):
+    n = 1 << k
+    p = W.random(n, 77 + k)
+    a = W.make_data(n)
+    try:
+        b, info = run(P, p, a, passes=3, layout=3, h=h, stages=stages, fuse=fuse, log2c=log2c)
+    except P.PermError as e:
+        assert h[1] < 4 and "h" in str(e)      # h2 >= 4 (16-byte tensor-store rows)
+        return
+    assert np.array_equal(b, OA.apply_ref(p, a)), (k, h, stages, fuse, log2c)
