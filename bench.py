@@ -389,9 +389,13 @@ def main():
               for i in range(nk)]
     dom = int(np.argmax(mean_k))
     E = info["entry_bits"]
-    # device schedule bytes per element of each phase (W64 format: floor(64/E) entries
-    # per 64-bit word, ceil(32/epw) words per warp-round of 32 elements)
-    sbpe = [8 * (-(-32 // (64 // e))) / 32 for e in E]
+    desc = plans[sched_fams[0]].describe()
+    if desc.get("layout") == 3:
+        # TLC format: each lane's ept entries are one bitstream of nwords 32-bit words
+        sbpe = [4 * t["nwords"] / t["ept"] for t in desc["tlc"]]
+    else:
+        # W64 format: floor(64/E) entries per 64-bit word, ceil(32/epw) words per warp-round
+        sbpe = [8 * (-(-32 // (64 // e))) / 32 for e in E]
     if info["direct"]:
         kinds = ["D-designated (direct)"]
         alg = [2 * n * 4 + n * 4]

@@ -80,7 +80,11 @@ typedef struct {
                             -1 = never (always run the scheduled passes), 1 = always */
     int32_t log2c;       /* view r x c with c = 2^log2c (the view "is not
                             restricted to a square matrix"); 0 = c = 2^ceil(k/2) */
-    int32_t reserved[2];
+    int32_t sched_format; /* TLC layout entry format: 0 = full (source row << log2(tile) |
+                             destination); 1 = compact (the line index inside the tile is implied
+                             by the source offset: 19 instead of 21 bits at n = 2^22) wherever a
+                             kernel is compiled for its width (not with fuse = 1) */
+    int32_t reserved[1];
 } perm_plan_options;
 
 typedef struct {

@@ -339,8 +339,8 @@ int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint3
                 for (int64_t q = 0; q < tp.HL / 32; ++q)
                     for (int64_t x = 0; x < 32; ++x) {
                         const uint32_t e = perm::tlc_entry(P.sched[f], tp, T, q, x);
-                        const uint32_t src = ((e >> tp.logHL) << 5) | (uint32_t)x;
-                        const uint32_t dst = e & (uint32_t)(tp.HL - 1);
+                        const uint32_t src = ((e >> tp.dec.lt) << 5) | (uint32_t)x;
+                        const uint32_t dst = perm::tlc_dst(tp.dec, e & ((1u << tp.dec.lt) - 1u), src);
                         outs[f][T * tp.HL + q * 32 + x] = (src << 16) | dst;
                     }
         }

@@ -967,6 +967,7 @@ struct TlcArgs {
     int nbox, box_outer, box_words;
     unsigned long long* trace;
     int prefetch_in;           // stream the whole input into L2 up front (HBM-resident input)
+    TlcDecode dec;             // entry -> destination (plan.hpp)
 };
 
 // Shared-memory word offsets of the TLC rings: A slots, then B slots, then mbarriers.
@@ -1018,14 +1019,30 @@ __device__ __forceinline__ void tlc_store(int kind, const CUtensorMap* map, uint
 // output order). Warp-round m of permuter warp pw: lane x reads A[32*sigma + x]
 // (bank x) and writes B[dst] (32 distinct banks per round, by construction of
 // the tile-level colouring). Entries are decoded from the lane's bitstream `wc`.
-template <int EPT>
+// Entry decode variants (plan.hpp TlcDecode), chosen at compile time:
+//   TLC_FULL: entry = (sigma << log2 HL) | dst
+//   TLC_X1 / TLC_X2 / TLC_ROWS: compact entries of pass 1 / 2 / 3, entry = (sigma << lt) | t,
+//   dst rebuilt with the line index taken from sigma (X1) or from the lane (X2, ROWS; a
+//   per-lane constant `lc`, so those decodes cost no more than the full format)
+enum { TLC_FULL = 0, TLC_X1 = 1, TLC_X2 = 2, TLC_ROWS = 3 };
+
+__device__ __forceinline__ uint32_t tlc_lane_const(int kind, const TlcDecode& dc, int lane) {
+    if (kind == TLC_X2) return (uint32_t)lane & dc.m2;
+    if (kind == TLC_ROWS) return (((uint32_t)lane >> dc.s4) & dc.m2) << dc.s3;
+    return 0u;
+}
+
+template <int EPT, int E, int KIND>
 __device__ __forceinline__ void tlc_permute(const uint32_t* __restrict__ A, uint32_t* __restrict__ B,
-                                            const uint32_t* wc, uint64_t* aempty, uint64_t* bempty_wait,
-                                            uint32_t bparity, int lane) {
+                                            const uint32_t* wc, const TlcDecode& dc, uint32_t lc,
+                                            uint64_t* aempty, uint64_t* bempty_wait, uint32_t bparity,
+                                            int lane) {
     constexpr int HL = kTlcPerm * EPT;
     constexpr int LOGHL = cilog2(HL);
-    constexpr int E = 2 * LOGHL - 5;
     constexpr uint32_t EMASK = (1u << E) - 1u;
+    const int lt = KIND == TLC_FULL ? LOGHL : dc.lt;
+    const uint32_t tmask = KIND == TLC_FULL ? (uint32_t)(HL - 1) : (1u << dc.lt) - 1u;
+    const int sh_line = dc.lt + dc.s4 - 5;    // TLC_X1: line index = e >> sh_line
     uint32_t v[EPT];
     uint32_t d[EPT];
 #pragma unroll
@@ -1034,8 +1051,12 @@ __device__ __forceinline__ void tlc_permute(const uint32_t* __restrict__ A, uint
         uint32_t e;
         if (off + E <= 32) e = (wc[w] >> off) & EMASK;
         else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
-        v[m] = A[((e >> LOGHL) << 5) | lane];
-        d[m] = e & (HL - 1);
+        const uint32_t t = e & tmask;
+        v[m] = A[((e >> lt) << 5) | (uint32_t)lane];
+        if constexpr (KIND == TLC_FULL) d[m] = t;
+        else if constexpr (KIND == TLC_X2) d[m] = (t << dc.s2) | lc;
+        else if constexpr (KIND == TLC_ROWS) d[m] = t | lc;
+        else d[m] = ((t >> dc.s1) << dc.s2) | ((e >> sh_line) << dc.s3) | (t & dc.m1);
     }
     mbar_arrive(aempty);                      // A slot may be refilled
     if (bempty_wait) mbar_wait(bempty_wait, bparity);
@@ -1054,12 +1075,10 @@ __device__ __forceinline__ void tlc_permute(const uint32_t* __restrict__ A, uint
 // intermediates). Roles: warp 0 lane 0 = TMA producer, warp 1 lane 0 = TMA
 // storer, warps 2..17 = permuters. Separate rings: `na` A slots (a CTA's whole
 // share of tiles is requested up front when it fits) and `nb` B slots.
-template <int EPT, int OUT>
+template <int EPT, int OUT, int E>
 __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     row_pass_tlc_kernel(const __grid_constant__ CUtensorMap tmap, const TlcArgs a) {
     constexpr int HL = kTlcPerm * EPT;
-    constexpr int LOGHL = cilog2(HL);
-    constexpr int E = 2 * LOGHL - 5;
     constexpr int NWORDS = (EPT * E + 31) / 32;
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -1130,6 +1149,9 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         }
     } else {
         // ---------------- permuters
+        constexpr int KIND = (E == 2 * cilog2(HL) - 5) ? TLC_FULL
+                             : (OUT == 1 ? TLC_X1 : (OUT == 2 ? TLC_X2 : TLC_ROWS));
+        const uint32_t lc = tlc_lane_const(KIND, a.dec, lane);
         const bool lead = tid == 64;
         const uint32_t* sp = a.sched + (warp - 2) * NWORDS * 32 + lane;
         uint32_t wc[NWORDS], wn[NWORDS];
@@ -1148,8 +1170,8 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             }
             mbar_wait(&R.afull[s], (uint32_t)(i / NA) & 1u);
             if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
-            tlc_permute<EPT>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wc, &R.aempty[s],
-                             i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
+            tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wc, a.dec, lc, &R.aempty[s],
+                                      i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
             mbar_arrive(&R.bfull[sb]);
 #pragma unroll
             for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
@@ -1168,6 +1190,7 @@ struct TlcPassCfg {
     int ntiles;
     int kind;                  // 0: rows (1-D bulk store), 1: X1, 2: X2 (3-D tensor stores)
     int chunk, nbox, box_outer, box_words;
+    TlcDecode dec;
 };
 
 struct TlcFusedArgs {
@@ -1186,13 +1209,11 @@ struct TlcFusedArgs {
 // after sync[k] reaches the grid size (schedule prefetches go ahead of the
 // barrier). One co-resident CTA per SM; the last CTA out resets the counters,
 // so the launch is replayable (CUDA graphs).
-template <int EPT>
+template <int EPT, int E>
 __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     fused_tlc_kernel(const __grid_constant__ CUtensorMap map_x1,
                      const __grid_constant__ CUtensorMap map_x2, const TlcFusedArgs a) {
     constexpr int HL = kTlcPerm * EPT;
-    constexpr int LOGHL = cilog2(HL);
-    constexpr int E = 2 * LOGHL - 5;
     constexpr int NWORDS = (EPT * E + 31) / 32;
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -1288,6 +1309,8 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         for (int k = 0; k < 3; ++k) {
             const TlcPassCfg& pc = a.p[k];
             const int nt = my_tiles(k);
+            const uint32_t lc = tlc_lane_const(pc.kind == 1 ? TLC_X1 : (pc.kind == 2 ? TLC_X2 : TLC_ROWS),
+                                               pc.dec, lane);
             const uint32_t* sp = pc.sched + (warp - 2) * NWORDS * 32 + lane;
             uint32_t wc[NWORDS], wn[NWORDS];
             if (nt > 0) {
@@ -1303,8 +1326,18 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 }
                 mbar_wait(&R.afull[s], (uint32_t)(j / NA) & 1u);
                 if (i == 0) stamp_if(tr, lead, 2 + 4 * k);
-                tlc_permute<EPT>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wc, &R.aempty[s],
-                                 j >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(j / NB - 1) & 1u, lane);
+                uint32_t* const Bs = R.B + (size_t)sb * HL;
+                const uint32_t* const As = R.A + (size_t)s * HL;
+                uint64_t* const bw = j >= NB ? &R.bempty[sb] : nullptr;
+                const uint32_t bp = (uint32_t)(j / NB - 1) & 1u;
+                if (E == 2 * cilog2(HL) - 5)
+                    tlc_permute<EPT, E, TLC_FULL>(As, Bs, wc, pc.dec, 0u, &R.aempty[s], bw, bp, lane);
+                else if (pc.kind == 1)
+                    tlc_permute<EPT, E, TLC_X1>(As, Bs, wc, pc.dec, lc, &R.aempty[s], bw, bp, lane);
+                else if (pc.kind == 2)
+                    tlc_permute<EPT, E, TLC_X2>(As, Bs, wc, pc.dec, lc, &R.aempty[s], bw, bp, lane);
+                else
+                    tlc_permute<EPT, E, TLC_ROWS>(As, Bs, wc, pc.dec, lc, &R.aempty[s], bw, bp, lane);
                 mbar_arrive(&R.bfull[sb]);
 #pragma unroll
                 for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
@@ -1549,62 +1582,62 @@ size_t tlc_smem(const HostPlan& P, int f) {
     return (size_t)(tp.stages + tp.bslots) * tp.HL * 4 + (size_t)(tp.stages + tp.bslots) * 8 * 2;
 }
 
-template <int EPT, int OUT>
-cudaError_t prep_tlc_one(HostPlan& P, int f) {
-    const size_t smem = tlc_smem(P, f);
-    cudaError_t e = set_smem(row_pass_tlc_kernel<EPT, OUT>, smem);
-    if (e != cudaSuccess) return e;
-    int nb = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_tlc_kernel<EPT, OUT>, 64 + kTlcPerm, smem);
-    if (e != cudaSuccess) return e;
-    if (nb < 1) return cudaErrorInvalidConfiguration;
-    TlcPass& tp = P.tp[f];
-    const long long cap = (long long)nb * sm_count();
-    tp.grid = tp.ntiles < cap ? tp.ntiles : cap;
-    P.rp[f].grid = tp.grid;
-    return cudaSuccess;
-}
-
-template <int OUT>
-cudaError_t prep_tlc_out(HostPlan& P, int f) {
-    switch (P.tp[f].ept) {
-        case 8: return prep_tlc_one<8, OUT>(P, f);
-        case 16: return prep_tlc_one<16, OUT>(P, f);
-        case 32: return prep_tlc_one<32, OUT>(P, f);
+// Calls f(EPT, E) (std::integral_constant) for the compiled (elements per thread,
+// entry bits) pairs of the TLC kernels: the full formats 2*log2(512*EPT) - 5 and
+// the compact widths of plan.hpp tlc_compact_supported().
+template <class F>
+cudaError_t tlc_dispatch(int ept, int E, F&& f) {
+    using std::integral_constant;
+    if (ept == 8 && E == 19) return f(integral_constant<int, 8>{}, integral_constant<int, 19>{});
+    if (ept == 16) {
+        switch (E) {
+            case 21: return f(integral_constant<int, 16>{}, integral_constant<int, 21>{});
+            case 19: return f(integral_constant<int, 16>{}, integral_constant<int, 19>{});
+            case 18: return f(integral_constant<int, 16>{}, integral_constant<int, 18>{});
+            case 17: return f(integral_constant<int, 16>{}, integral_constant<int, 17>{});
+            case 16: return f(integral_constant<int, 16>{}, integral_constant<int, 16>{});
+            case 15: return f(integral_constant<int, 16>{}, integral_constant<int, 15>{});
+        }
     }
+    if (ept == 32 && E == 23) return f(integral_constant<int, 32>{}, integral_constant<int, 23>{});
+    if (ept == 32 && E == 21) return f(integral_constant<int, 32>{}, integral_constant<int, 21>{});
     return cudaErrorInvalidValue;
 }
 
-template <int EPT>
-cudaError_t prep_tlc_fused_one(HostPlan& P) {
-    const size_t smem = tlc_smem(P, 0);
-    cudaError_t e = set_smem(fused_tlc_kernel<EPT>, smem);
+template <class K>
+cudaError_t prep_tlc_kernel(K kernel, size_t smem, long long ntiles, long long& grid) {
+    cudaError_t e = set_smem(kernel, smem);
     if (e != cudaSuccess) return e;
     int nb = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fused_tlc_kernel<EPT>, 64 + kTlcPerm, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, 64 + kTlcPerm, smem);
     if (e != cudaSuccess) return e;
     if (nb < 1) return cudaErrorInvalidConfiguration;
-    P.fused3_grid = sm_count();      // one co-resident CTA per SM (grid barriers)
+    const long long cap = (long long)nb * sm_count();
+    grid = ntiles < cap ? ntiles : cap;
     return cudaSuccess;
 }
 
 cudaError_t prep_tlc(HostPlan& P) {
     if (P.fused3) {
-        switch (P.tp[0].ept) {
-            case 8: return prep_tlc_fused_one<8>(P);
-            case 16: return prep_tlc_fused_one<16>(P);
-            case 32: return prep_tlc_fused_one<32>(P);
-        }
-        return cudaErrorInvalidValue;
+        return tlc_dispatch(P.tp[0].ept, P.tp[0].E, [&](auto ept, auto E) {
+            long long g = 0;
+            const cudaError_t e = prep_tlc_kernel(fused_tlc_kernel<ept, E>, tlc_smem(P, 0), 1, g);
+            P.fused3_grid = sm_count();      // one co-resident CTA per SM (grid barriers)
+            return e;
+        });
     }
     cudaError_t e = cudaSuccess;
     for (int f = 0; f < 3 && e == cudaSuccess; ++f) {
-        switch (P.tp[f].out_kind) {
-            case 0: e = prep_tlc_out<0>(P, f); break;
-            case 1: e = prep_tlc_out<1>(P, f); break;
-            case 2: e = prep_tlc_out<2>(P, f); break;
-            default: return cudaErrorInvalidValue;
-        }
+        TlcPass& tp = P.tp[f];
+        long long g = 0;
+        e = tlc_dispatch(tp.ept, tp.E, [&](auto ept, auto E) {
+            const size_t smem = tlc_smem(P, f);
+            if (tp.out_kind == 0) return prep_tlc_kernel(row_pass_tlc_kernel<ept, 0, E>, smem, tp.ntiles, g);
+            if (tp.out_kind == 1) return prep_tlc_kernel(row_pass_tlc_kernel<ept, 1, E>, smem, tp.ntiles, g);
+            return prep_tlc_kernel(row_pass_tlc_kernel<ept, 2, E>, smem, tp.ntiles, g);
+        });
+        tp.grid = g;
+        P.rp[f].grid = g;
     }
     return e;
 }
@@ -1678,18 +1711,12 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
     const CUtensorMap& map = maps[tp.out_kind == 2 ? 1 : 0];
     const dim3 grid((unsigned)tp.grid), block(64 + kTlcPerm);
     const size_t smem = tlc_smem(P, f);
-#define PERM_TLC_CASE(E_)                                                                             \
-    case E_:                                                                                          \
-        if (tp.out_kind == 0) return launch(row_pass_tlc_kernel<E_, 0>, grid, block, smem, s, pdl, map, ta); \
-        if (tp.out_kind == 1) return launch(row_pass_tlc_kernel<E_, 1>, grid, block, smem, s, pdl, map, ta); \
-        return launch(row_pass_tlc_kernel<E_, 2>, grid, block, smem, s, pdl, map, ta);
-    switch (tp.ept) {
-        PERM_TLC_CASE(8)
-        PERM_TLC_CASE(16)
-        PERM_TLC_CASE(32)
-    }
-#undef PERM_TLC_CASE
-    return cudaErrorInvalidValue;
+    ta.dec = tp.dec;
+    return tlc_dispatch(tp.ept, tp.E, [&](auto ept, auto E) {
+        if (tp.out_kind == 0) return launch(row_pass_tlc_kernel<ept, 0, E>, grid, block, smem, s, pdl, map, ta);
+        if (tp.out_kind == 1) return launch(row_pass_tlc_kernel<ept, 1, E>, grid, block, smem, s, pdl, map, ta);
+        return launch(row_pass_tlc_kernel<ept, 2, E>, grid, block, smem, s, pdl, map, ta);
+    });
 }
 
 cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const uint32_t* const sched[3],
@@ -1707,6 +1734,7 @@ cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const u
         pc.sched = sched[f];
         pc.ntiles = (int)tp.ntiles;
         pc.kind = tp.out_kind;
+        pc.dec = tp.dec;
         if (tp.out_kind == 1) {
             const long long outer = P.c / h2, bo = outer < 256 ? outer : 256;
             pc.box_outer = (int)bo;
@@ -1728,12 +1756,9 @@ cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const u
     fa.trace = trace;
     const dim3 grid((unsigned)P.fused3_grid), block(64 + kTlcPerm);
     const size_t smem = tlc_smem(P, 0);
-    switch (P.tp[0].ept) {
-        case 8: return launch(fused_tlc_kernel<8>, grid, block, smem, s, false, maps[0], maps[1], fa);
-        case 16: return launch(fused_tlc_kernel<16>, grid, block, smem, s, false, maps[0], maps[1], fa);
-        case 32: return launch(fused_tlc_kernel<32>, grid, block, smem, s, false, maps[0], maps[1], fa);
-    }
-    return cudaErrorInvalidValue;
+    return tlc_dispatch(P.tp[0].ept, P.tp[0].E, [&](auto ept, auto E) {
+        return launch(fused_tlc_kernel<ept, E>, grid, block, smem, s, false, maps[0], maps[1], fa);
+    });
 }
 
 cudaError_t prepare_kernels(HostPlan& P) {

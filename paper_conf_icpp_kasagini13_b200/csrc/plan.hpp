@@ -75,6 +75,27 @@ struct RowPass {
 // ((T*NW + pw)*nwords + w)*32 + x (coalesced loads).
 constexpr int kTlcPerm = 512;           // permuter threads per CTA
 
+// Destination of a TLC entry. An element never leaves its line in a row-wise
+// permutation (L517), so the line's index inside the tile is a function of the
+// source offset; the entry keeps only t = the destination position in the line
+// (log2 L bits) and the kernel rebuilds
+//   dst = ((t >> s1) << s2) | (((src >> s4) & m2) << s3) | (t & m1),
+// E = (logHL - 5) + lt bits ("compact"; 19 at n = 2^22 vs 21). The full format
+// (lt = logHL, dst = t: s1 = s2 = s3 = s4 = m1 = m2 = 0) is kept for entry
+// widths without a compiled kernel (tlc_compact_supported).
+struct TlcDecode {
+    int32_t lt = 0;
+    int32_t s1 = 0, s2 = 0, s3 = 0, s4 = 0;
+    uint32_t m1 = 0, m2 = 0;
+};
+inline uint32_t tlc_dst(const TlcDecode& d, uint32_t t, uint32_t src) {
+    return ((t >> d.s1) << d.s2) | (((src >> d.s4) & d.m2) << d.s3) | (t & d.m1);
+}
+// (elements per permuter thread, compact entry bits) pairs with a compiled kernel
+inline bool tlc_compact_supported(int ept, int E) {
+    return (ept == 16 && E >= 15 && E <= 19) || (ept == 32 && E == 21);
+}
+
 struct TlcPass {
     int32_t h = 0;            // lines per tile
     int32_t HL = 0, logHL = 0;
@@ -84,6 +105,7 @@ struct TlcPass {
     int64_t ntiles = 0;
     int64_t tile_words = 0;   // (kTlcPerm / 32) * nwords * 32
     int32_t out_kind = 0;     // 0: rows (1-D bulk store); 1: X1 / 2: X2 2-D tensor store (64-byte box rows)
+    TlcDecode dec;            // entry -> destination offset (compact or full format)
     int32_t stages = 0;       // A slots (TMA loads in flight); B slots = bslots
     int32_t bslots = 0;       // B slots (permuted tiles waiting for / under their TMA store)
     int64_t grid = 0;         // persistent CTAs (set at upload)

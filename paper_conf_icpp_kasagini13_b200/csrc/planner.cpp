@@ -472,8 +472,10 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
     int64_t hs[3];
     for (int f = 0; f < 3; ++f) {
         const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
+        // default tiles: 8192 words up to 2^24 (64-byte transposed chunks), 16384 words at
+        // 2^25 (32-byte chunks: h1*h2*4 bytes with h1*L, h2*r <= 16384 words)
         int64_t h = (opt && (&opt->h1)[f] > 0) ? (&opt->h1)[f]
-                                                : std::max<int64_t>(4, 8192 / L);
+                    : (P.k <= 24 ? std::max<int64_t>(4, 8192 / L) : std::max<int64_t>(1, 16384 / L));
         h = std::min(h, lines_f);
         // h2 is the inner dimension of the TMA tensor boxes (>= 16 bytes)
         if (h < (f == 1 ? 4 : 1) || (h & (h - 1)) || lines_f % h) {
@@ -488,12 +490,39 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
         tp.h = (int32_t)hs[f];
         tp.HL = (int32_t)(hs[f] * P.ph[f].L);
         tp.logHL = ilog2(tp.HL);
-        tp.E = 2 * tp.logHL - 5;
         tp.ept = tp.HL / kTlcPerm;
         if (tp.ept != 8 && tp.ept != 16 && tp.ept != 32) {
             err = "TLC layout: tile must hold 4096, 8192 or 16384 elements (h * L)";
             return PERM_EINVAL;
         }
+        // entry format (plan.hpp TlcDecode): compact when a kernel is compiled for its width
+        const int logL = P.ph[f].logL;
+        const int cmp_opt = opt ? opt->sched_format : 0;
+        const int Ec = tp.logHL - 5 + logL;
+        TlcDecode d;
+        // the kernels take pass 2's and pass 3's line index from the lane alone (free decode):
+        // needs h2 <= 32 (pass 2) and h2 * h3 <= 32 (pass 3)
+        const bool lane_line = (f != 1 || hs[1] <= kW) && (f != 2 || hs[1] * hs[2] <= kW);
+        // (measured on B200: no faster than the full format at 2^22..2^25, so opt-in)
+        const bool fused_req = opt && opt->fuse > 0;
+        if (cmp_opt > 0 && !fused_req && tlc_compact_supported(tp.ept, Ec) && lane_line) {
+            const int lh1 = ilog2(hs[0]), lh2 = ilog2(hs[1]), lc = ilog2(P.c);
+            d.lt = logL;
+            if (f == 0) {          // dst = ((k/h2)*h1 + i_in)*h2 + k%h2, i_in = src >> log c
+                d.s1 = lh2; d.s2 = lh1 + lh2; d.s4 = lc; d.m2 = (uint32_t)hs[0] - 1; d.s3 = lh2;
+                d.m1 = (uint32_t)hs[1] - 1;
+            } else if (f == 1) {   // dst = i'*h2 + k_in, k_in = src mod h2
+                d.s1 = 0; d.s2 = lh2; d.s4 = 0; d.m2 = (uint32_t)hs[1] - 1; d.s3 = 0; d.m1 = 0;
+            } else {               // dst = i_in*c + k', i_in = (src >> log h2) mod h3
+                d.s1 = lc; d.s2 = 0; d.s4 = lh2; d.m2 = (uint32_t)hs[2] - 1; d.s3 = lc;
+                d.m1 = (uint32_t)P.c - 1;
+            }
+            tp.E = Ec;
+        } else {
+            d.lt = tp.logHL;       // full format: dst = t
+            tp.E = 2 * tp.logHL - 5;
+        }
+        tp.dec = d;
         tp.nwords = (tp.ept * tp.E + 31) / 32;
         tp.ntiles = P.ph[f].lines / hs[f];
         tp.tile_words = (int64_t)(kTlcPerm / 32) * tp.nwords * 32;
@@ -521,11 +550,15 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
         uint32_t* W = P.sched[f].data();
         const uint16_t* ph = phi[f].data();
         const int64_t HL = tp.HL, h = tp.h;
-        const int E = tp.E, ept = tp.ept, logHL = tp.logHL, nwords = tp.nwords;
-#pragma omp parallel
+        const int E = tp.E, ept = tp.ept, nwords = tp.nwords;
+        const TlcDecode dec = tp.dec;
+        const bool full = dec.lt == tp.logHL && dec.s2 == 0 && dec.s3 == 0 && dec.m1 == 0;
+        int bad = 0;
+#pragma omp parallel reduction(| : bad)
         {
             EulerColourer ec;
-            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL);
+            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL),
+                tval((size_t)HL);
 #pragma omp for schedule(dynamic, 1)
             for (int64_t T = 0; T < tp.ntiles; ++T) {
                 int64_t e = 0;
@@ -535,6 +568,7 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
                             const int64_t kk = ph[(T * h + i_in) * c + j];
                             src[e] = (uint32_t)(i_in * c + j);
                             dst[e] = (uint32_t)(((kk / h2) * h1 + i_in) * h2 + kk % h2);
+                            tval[e] = full ? dst[e] : (uint32_t)kk;
                         }
                 } else if (f == 1) {
                     for (int64_t k_in = 0; k_in < h; ++k_in)
@@ -542,6 +576,7 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
                             const int64_t ip = ph[(T * h + k_in) * r + i];
                             src[e] = (uint32_t)(i * h2 + k_in);
                             dst[e] = (uint32_t)(ip * h2 + k_in);
+                            tval[e] = full ? dst[e] : (uint32_t)ip;
                         }
                 } else {
                     for (int64_t i_in = 0; i_in < h; ++i_in)
@@ -549,6 +584,7 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
                             const int64_t kp = ph[(T * h + i_in) * c + kk];
                             src[e] = (uint32_t)(((kk / h2) * h3 + i_in) * h2 + kk % h2);
                             dst[e] = (uint32_t)(i_in * c + kp);
+                            tval[e] = full ? dst[e] : (uint32_t)kp;
                         }
                 }
                 for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
@@ -558,7 +594,9 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
                     const int64_t q = col[x];                 // warp-round
                     const int64_t lane = src[x] & 31;         // lane = source bank
                     const int64_t pw = q / ept, m = q % ept;
-                    const uint64_t entry = ((uint64_t)(src[x] >> 5) << logHL) | dst[x];
+                    const uint32_t t = tval[x];
+                    if (tlc_dst(dec, t, src[x]) != dst[x]) bad = 1;   // decode self-check
+                    const uint64_t entry = ((uint64_t)(src[x] >> 5) << dec.lt) | t;
                     const int64_t bit = m * E;
                     const int64_t w = bit >> 5, off = bit & 31;
                     const uint64_t sh = entry << off;
@@ -568,6 +606,7 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
                 }
             }
         }
+        if (bad) { err = "TLC layout: internal error (entry decode mismatch)"; return PERM_ECUDA; }
     }
     (void)NW;
     return PERM_OK;
@@ -737,9 +776,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 
     // pass structure
     int passes = opt ? opt->passes : 0;
-    // measured on B200: fused CTA to 2^14, TLC 3-pass 2^15..2^24 (LINES /
-    // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^25
-    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 24 ? 3 : 5);
+    // measured on B200: fused CTA to 2^14, TLC 3-pass 2^15..2^25 (LINES /
+    // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^26
+    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 25 ? 3 : 5);
     if (passes == 1 && k > 14) { err = "fused single-CTA pass needs n <= 2^14"; return PERM_EUNSUPPORTED; }
     if (passes != 1 && passes != 3 && passes != 5) { err = "passes must be 0, 1, 3 or 5"; return PERM_EINVAL; }
     P.passes = passes;
@@ -754,14 +793,15 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     }
     {
         int layout0 = opt ? opt->layout : 0;
-        if (passes == 3 && (layout0 == 3 || (layout0 == 0 && k >= 15 && k <= 24))) {
+        if (passes == 3 && (layout0 == 3 || (layout0 == 0 && k >= 15 && k <= 25))) {
             const int st = build_tlc(P, phi, opt, err);
             P.ms_bank = ms_since(t0);
             // one persistent launch when the three passes share the tile size (square view)
             const int fuse = opt ? opt->fuse : 0;
             if (st == PERM_OK && fuse > 0 && P.tp[0].HL == P.tp[1].HL && P.tp[1].HL == P.tp[2].HL &&
                 P.tp[0].stages == P.tp[1].stages && P.tp[1].stages == P.tp[2].stages &&
-                P.tp[0].bslots == P.tp[1].bslots && P.tp[1].bslots == P.tp[2].bslots)
+                P.tp[0].bslots == P.tp[1].bslots && P.tp[1].bslots == P.tp[2].bslots &&
+                P.tp[0].E == P.tp[1].E && P.tp[1].E == P.tp[2].E)
                 P.fused3 = 1;
             return st;
         }

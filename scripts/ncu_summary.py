@@ -10,6 +10,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument('--launches')
 ap.add_argument('--full')
 ap.add_argument('--out', required=True)
+ap.add_argument('--traffic-key', help="also write profiles/ncu_traffic.json[key] = per-pass DRAM bytes")
 a = ap.parse_args()
 summary = {}
 if a.launches:
@@ -80,6 +81,23 @@ if a.full:
         e['top_stalls'] = {n: round(v, 2) for v, n in sorted(stalls, reverse=True)[:6]}
         kern.append(e)
     summary['full'] = kern
+    if a.traffic_key:
+        import os, re
+        tp = os.path.join(os.path.dirname(os.path.abspath(__file__)), '..', 'profiles', 'ncu_traffic.json')
+        tj = json.load(open(tp)) if os.path.exists(tp) else {}
+        ent = {}
+        for e in kern:
+            m = re.search(r'row_pass_tlc_kernel<(\d+), (\d+)', e['kernel'])
+            if not m:
+                continue
+            kind = {'1': 'R1', '2': 'R2', '0': 'R3'}[m.group(2)]
+            def num(x):
+                v, u = x.split(' ', 1) if ' ' in x else (x, '')
+                v = float(v.replace(',', ''))
+                return v * {'byte': 1, 'Kbyte': 1e3, 'Mbyte': 1e6, 'Gbyte': 1e9}.get(u.strip(), 1)
+            ent[kind] = num(e['dram__bytes_read.sum']) + num(e['dram__bytes_write.sum'])
+        tj[a.traffic_key] = ent
+        json.dump(tj, open(tp, 'w'), indent=1)
     with open(a.out + '_ncu_full.md', 'w') as f:
         f.write('# ncu --set full (cold caches, serialized replay)\n\n')
         for e in kern:

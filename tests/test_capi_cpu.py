@@ -191,7 +191,30 @@ def test_tlc_plan_22(lib):
     p = W.random(n, 42)
     info, d, kappa, sched = export_tlc(lib, p)
     assert info["h"] == [4, 4, 4] and info["entry_bits"] == [21, 21, 21]
+    # compact entries: sigma (8 bits) + destination position in the line (11 bits)
+    info_c, _, kappa_c, sched_c = export_tlc(lib, p, sched_format=1)
+    assert info_c["entry_bits"] == [19, 19, 19]
+    res = OC.check_tlc(p, kappa_c, sched_c, r, c, (4, 4, 4))
+    assert all(res.values()), res
     res = OC.check_tlc(p, kappa, sched, r, c, (4, 4, 4))
+    assert all(res.values()), res
+
+
+@pytest.mark.parametrize("k", [15, 18, 21])
+def test_tlc_full_and_compact_formats_agree(lib, k):
+    # the two device entry formats must export the same logical (src, dst) schedule
+    n = 1 << k
+    r, c = W.view_shape(n)
+    p = W.make_perm("random", n, seed=k)
+    i_full, _, kappa_f, s_full = export_tlc(lib, p, sched_format=0)
+    i_cmp, _, kappa_c, s_cmp = export_tlc(lib, p, sched_format=1)
+    assert np.array_equal(kappa_f, kappa_c)
+    for a, b in zip(s_full, s_cmp):
+        assert np.array_equal(a, b)
+    assert all(ec <= ef for ec, ef in zip(i_cmp["entry_bits"], i_full["entry_bits"]))
+    assert i_cmp["entry_bits"][0] < i_full["entry_bits"][0]
+    assert i_cmp["sched_bytes"] < i_full["sched_bytes"]
+    res = OC.check_tlc(p, kappa_c, s_cmp, r, c, tuple(i_cmp["h"]))
     assert all(res.values()), res
 
 

@@ -347,3 +347,14 @@ def test_tlc_rings_wrap(P, k, h, stages, fuse, log2c):
         assert h[1] < 4 and "h" in str(e)      # h2 >= 4 (16-byte tensor-store rows)
         return
     assert np.array_equal(b, OA.apply_ref(p, a)), (k, h, stages, fuse, log2c)
+
+
+@pytest.mark.parametrize("fmt", [0, 1])
+@pytest.mark.parametrize("k", [15, 17, 20, 22, 23, 25])
+def test_tlc_entry_formats(P, k, fmt):
+    # full (source row << log2 tile | destination) vs compact (line index implied) entries
+    n = 1 << k
+    p = W.random(n, 500 + k)
+    a = W.make_data(n)
+    b, info = run(P, p, a, passes=3, layout=3, sched_format=fmt)
+    assert np.array_equal(b, OA.apply_ref(p, a)), (k, fmt, info["entry_bits"])
