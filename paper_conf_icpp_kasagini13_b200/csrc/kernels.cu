@@ -1154,27 +1154,36 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         const uint32_t lc = tlc_lane_const(KIND, a.dec, lane);
         const bool lead = tid == 64;
         const uint32_t* sp = a.sched + (warp - 2) * NWORDS * 32 + lane;
-        uint32_t wc[NWORDS], wn[NWORDS];
-        if (blockIdx.x < a.ntiles) {
+        // schedule words live in registers, loaded AHEAD tiles ahead (L2 latency under the
+        // load of a pass is about one tile period)
+        constexpr int AHEAD = NWORDS <= 12 ? 2 : 1;
+        uint32_t wq[AHEAD + 1][NWORDS];
 #pragma unroll
-            for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + (long long)blockIdx.x * a.tile_words + w * 32);
+        for (int k = 0; k < AHEAD; ++k) {
+            const long long tk = blockIdx.x + (long long)k * G;
+            if (tk < a.ntiles) {
+#pragma unroll
+                for (int w = 0; w < NWORDS; ++w) wq[k][w] = __ldg(sp + tk * a.tile_words + w * 32);
+            }
         }
         for (int i = 0;; ++i) {
             const long long t = blockIdx.x + (long long)i * G;
             if (t >= a.ntiles) break;
             const int s = i % NA, sb = i % NB;
-            const long long tn = t + G;
+            const long long tn = t + (long long)AHEAD * G;
             if (tn < a.ntiles) {
 #pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wn[w] = __ldg(sp + tn * a.tile_words + w * 32);
+                for (int w = 0; w < NWORDS; ++w) wq[AHEAD][w] = __ldg(sp + tn * a.tile_words + w * 32);
             }
             mbar_wait(&R.afull[s], (uint32_t)(i / NA) & 1u);
             if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
-            tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wc, a.dec, lc, &R.aempty[s],
+            tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wq[0], a.dec, lc, &R.aempty[s],
                                       i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
             mbar_arrive(&R.bfull[sb]);
 #pragma unroll
-            for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
+            for (int k = 0; k < AHEAD; ++k)
+#pragma unroll
+                for (int w = 0; w < NWORDS; ++w) wq[k][w] = wq[k + 1][w];
         }
         stamp_if(tr, lead, 3);
     }
@@ -1297,7 +1306,7 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                     fence_proxy_async_global();
                     __threadfence();
                     red_release_gpu_add(&a.sync[k], 1ull);
-                    stamp(tr, 4 + 4 * k);
+                    stamp_if(tr, true, 4 + 4 * k);
                 }
             }
             bulk_wait0();
