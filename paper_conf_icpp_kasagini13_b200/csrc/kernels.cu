@@ -28,6 +28,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstring>
+#include <cstdlib>
 
 #include "kernels.hpp"
 
@@ -968,6 +969,9 @@ struct TlcArgs {
     unsigned long long* trace;
     int prefetch_in;           // stream the whole input into L2 up front (HBM-resident input)
     TlcDecode dec;             // entry -> destination (plan.hpp)
+    int last_lsu;              // the CTA's last tile leaves through the permuters' 128-bit stores
+    int cw;                    // words per output chunk (tile-contiguous run in global memory)
+    long long cstride;         // global word stride between a tile's consecutive chunks
 };
 
 // Shared-memory word offsets of the TLC rings: A slots, then B slots, then mbarriers.
@@ -1093,23 +1097,22 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     if (warp == 0) {
         if (lane == 0) {
             // ---------------- producer
-            // every schedule chunk of this CTA (independent of the previous pass) is
-            // requested into L2 now; for HBM-resident input, so are the input tiles
-            // beyond the ring
-            for (int i = 0;; ++i) {
+            // Schedules do not depend on the previous pass. L2-resident input (passes 2, 3):
+            // every schedule chunk of this CTA is requested into L2 before griddepcontrol.wait,
+            // using HBM while the previous pass drains. HBM-resident input (pass 1): data and
+            // schedule compete for HBM, so only the first two tiles' schedules go ahead and
+            // the rest are interleaved behind the data loads (first tile lands earlier).
+            const int sched_ahead = a.prefetch_in ? 2 : (1 << 30);
+            auto prefetch_sched = [&](int i) {
                 const long long t = blockIdx.x + (long long)i * G;
-                if (t >= a.ntiles) break;
-                prefetch_l2_bulk(a.sched + t * a.tile_words, (uint32_t)(a.tile_words * 4));
+                if (t < a.ntiles) prefetch_l2_bulk(a.sched + t * a.tile_words, (uint32_t)(a.tile_words * 4));
+            };
+            for (int i = 0; i < sched_ahead; ++i) {
+                if (blockIdx.x + (long long)i * G >= a.ntiles) break;
+                prefetch_sched(i);
             }
             pdl_wait();
             stamp(tr, 1);
-            if (a.prefetch_in) {
-                for (int i = NA;; ++i) {
-                    const long long t = blockIdx.x + (long long)i * G;
-                    if (t >= a.ntiles) break;
-                    prefetch_l2_bulk(a.in + t * HL, (uint32_t)HL * 4u);
-                }
-            }
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
@@ -1119,6 +1122,15 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 mbar_arrive_expect_tx(&R.afull[s], (uint32_t)HL * 4u);
                 bulk_g2s(R.A + (size_t)s * HL, a.in + t * HL, (uint32_t)HL * 4u, &R.afull[s]);
                 if (i == 0) pdl_launch_dependents();
+                if (a.prefetch_in) {
+                    prefetch_sched(i + sched_ahead);
+                    if (i + 1 == NA)           // input tiles beyond the ring: into L2 now
+                        for (int j = NA;; ++j) {
+                            const long long tj = blockIdx.x + (long long)j * G;
+                            if (tj >= a.ntiles) break;
+                            prefetch_l2_bulk(a.in + tj * HL, (uint32_t)HL * 4u);
+                        }
+                }
             }
         }
     } else if (warp == 1) {
@@ -1129,6 +1141,7 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
+                if (a.last_lsu && t + G >= a.ntiles) break;     // the permuters store the last tile
                 const int s = i % NB;
                 mbar_wait(&R.bfull[s], (uint32_t)(i / NB) & 1u);
                 tlc_store(OUT, &tmap, a.out, R.B + (size_t)s * HL, t, HL, a.chunk, a.nbox, a.box_outer,
@@ -1179,6 +1192,21 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
             tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wq[0], a.dec, lc, &R.aempty[s],
                                       i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
+            if (a.last_lsu && t + G >= a.ntiles) {
+                // last tile: the 512 permuter threads store it (16 warps issue in parallel,
+                // shorter drain before the pass boundary than one TMA unit's 64-byte rows)
+                named_bar(1, kTlcPerm);
+                const uint4* B4 = reinterpret_cast<const uint4*>(R.B + (size_t)sb * HL);
+                const int pt = tid - 64;
+#pragma unroll
+                for (int m = 0; m < EPT / 4; ++m) {
+                    const int v = m * kTlcPerm + pt;           // 16-byte vector of the tile
+                    const int w = 4 * v;
+                    const long long g = (long long)(w / a.cw) * a.cstride + t * a.cw + (w % a.cw);
+                    st_v4(a.out + g, B4[v]);
+                }
+                break;
+            }
             mbar_arrive(&R.bfull[sb]);
 #pragma unroll
             for (int k = 0; k < AHEAD; ++k)
@@ -1721,6 +1749,13 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
     const dim3 grid((unsigned)tp.grid), block(64 + kTlcPerm);
     const size_t smem = tlc_smem(P, f);
     ta.dec = tp.dec;
+    {
+        static const char* env = std::getenv("PERM_TLC_LAST_LSU");
+        ta.last_lsu = env ? std::atoi(env) : 0;   // measured: no faster (explore_r01o)
+    }
+    if (tp.out_kind == 0) { ta.cw = tp.HL; ta.cstride = tp.HL; }
+    else if (tp.out_kind == 1) { ta.cw = (int)(h1 * h2); ta.cstride = P.r * h2; }
+    else { ta.cw = (int)(h3 * h2); ta.cstride = P.c * h3; }
     return tlc_dispatch(tp.ept, tp.E, [&](auto ept, auto E) {
         if (tp.out_kind == 0) return launch(row_pass_tlc_kernel<ept, 0, E>, grid, block, smem, s, pdl, map, ta);
         if (tp.out_kind == 1) return launch(row_pass_tlc_kernel<ept, 1, E>, grid, block, smem, s, pdl, map, ta);
