@@ -182,6 +182,18 @@ int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k);
 int     perm_plan_set_tracing(perm_plan* plan, int enable);
 int64_t perm_plan_trace(const perm_plan* plan, uint64_t* out, int64_t max_entries);
 
+/* Diagnostics (kernel roofline timing): launch ONE row pass of a 3-launch TLC plan
+ * (layout 3, not fused, not on the low-distribution shortcut), stream-ordered:
+ *   pass 0: in (n words, row-major a)      -> the plan's internal X1
+ *   pass 1: in (n words, X1 layout)        -> the plan's internal X2
+ *   pass 2: in (n words, X2 layout)        -> out (n words, row-major b)
+ * `in` need not come from the previous pass (any data times the same: the
+ * schedule, not the data, decides every address); in = NULL for passes 1 and 2
+ * reads the plan's own X1 / X2, so run_pass(0, a), (1, NULL), (2, NULL, b) is
+ * perm_apply. PERM_EUNSUPPORTED for other plans. */
+int perm_plan_run_pass(const perm_plan* plan, int32_t pass, const void* in, void* out,
+                       perm_stream_t stream);
+
 /* ------------------------------------------------- row-sharded (multi-GPU) */
 
 /* rank g of `world` GPUs owns rows [g*r/world, (g+1)*r/world) of the

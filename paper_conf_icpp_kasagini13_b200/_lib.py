@@ -78,6 +78,7 @@ _plan_create_sharded = _sig("perm_plan_create_sharded", _vp, _vp, _i64, _i32, _i
 _plan_create_sharded_host = _sig("perm_plan_create_sharded_host", _vp, _vp, _i64, _i32, _i32, _i32,
                                  ctypes.POINTER(PlanOptions))
 _sharded_step = _sig("perm_sharded_step", ctypes.c_int, _vp, _i32, _vp, _vp, _vp)
+_run_pass = _sig("perm_plan_run_pass", ctypes.c_int, _vp, _i32, _vp, _vp, _vp)
 _plan_destroy = _sig("perm_plan_destroy", None, _vp)
 _plan_get_info = _sig("perm_plan_get_info", ctypes.c_int, _vp, ctypes.POINTER(PlanInfo))
 _plan_describe = _sig("perm_plan_describe", _i64, _vp, ctypes.c_char_p, _i64)
@@ -219,6 +220,11 @@ class Plan:
         """One local step of a row-sharded apply (see include/perm.h perm_sharded_step)."""
         _check(_sharded_step(self._h, step, _ptr(inp), _ptr(out), _stream_handle(stream)))
         return out
+
+    def run_pass(self, k: int, inp, out=None, stream=None):
+        """Launch row pass k alone (TLC plans; see include/perm.h perm_plan_run_pass)."""
+        _check(_run_pass(self._h, k, _ptr(inp) if inp is not None else None,
+                         _ptr(out) if out is not None else None, _stream_handle(stream)))
 
     def set_profiling(self, on: bool = True):
         _check(_set_prof(self._h, 1 if on else 0))

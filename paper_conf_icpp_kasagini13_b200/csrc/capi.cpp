@@ -419,6 +419,29 @@ int perm_plan_pass_times(const perm_plan* plan, float* ms, int max_k) {
     return w;
 }
 
+int perm_plan_run_pass(const perm_plan* plan, int32_t pass, const void* in, void* out,
+                       perm_stream_t stream) {
+    if (!plan) return fail(PERM_EINVAL, "null plan");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
+    const HostPlan& P = plan->host;
+    if (P.layout != 3 || P.fused3 || plan->d_p) return fail(PERM_EUNSUPPORTED, "run_pass needs a 3-launch TLC plan");
+    if (pass < 0 || pass > 2) return fail(PERM_EINVAL, "pass must be 0, 1 or 2");
+    if (!in) {
+        if (pass == 0) return fail(PERM_EINVAL, "pass 0 needs an input buffer");
+        in = plan->d_scratch[pass - 1];        // the plan's own intermediate
+    }
+    if (pass == 2 && !out) return fail(PERM_EINVAL, "pass 2 needs an output buffer");
+    if ((reinterpret_cast<uintptr_t>(in) | reinterpret_cast<uintptr_t>(out)) & 15)
+        return fail(PERM_EINVAL, "buffers must be 16-byte aligned");
+    uint32_t* dst = pass == 0 ? plan->d_scratch[0] : (pass == 1 ? plan->d_scratch[1] : static_cast<uint32_t*>(out));
+    if (overlap(in, dst, P.n * P.eb)) return fail(PERM_EINVAL, "input overlaps the pass output");
+    const cudaError_t e = perm::launch_tlc_pass(P, pass, plan->tlc_maps, plan->d_phase[pass],
+                                                static_cast<const uint32_t*>(in), dst,
+                                                static_cast<cudaStream_t>(stream), true, nullptr);
+    if (e != cudaSuccess) return cuda_fail(e, "run_pass launch");
+    return PERM_OK;
+}
+
 int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t stream) {
     perm_plan* plan = const_cast<perm_plan*>(plan_c);   // only profiling bookkeeping mutates
     if (!plan || !a || !b) return fail(PERM_EINVAL, "null plan or buffer");

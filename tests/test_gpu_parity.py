@@ -358,3 +358,22 @@ def test_tlc_entry_formats(P, k, fmt):
     a = W.make_data(n)
     b, info = run(P, p, a, passes=3, layout=3, sched_format=fmt)
     assert np.array_equal(b, OA.apply_ref(p, a)), (k, fmt, info["entry_bits"])
+
+
+@pytest.mark.parametrize("k", [16, 22])
+def test_run_pass_chain_is_apply(P, k):
+    # perm_plan_run_pass (diagnostics / roofline timing): the three passes launched one by
+    # one through the plan's own intermediates give exactly b[P(i)] = a[i]
+    n = 1 << k
+    p = W.random(n, 900 + k)
+    a = W.make_data(n)
+    with P.Plan(p) as plan:
+        da = dev(a)
+        db = torch.full_like(da, -1)
+        plan.run_pass(0, da)
+        plan.run_pass(1, None)
+        plan.run_pass(2, None, db)
+        torch.cuda.synchronize()
+        assert np.array_equal(host_words(db), OA.apply_ref(p, a))
+        with pytest.raises(P.PermError):
+            plan.run_pass(3, da)
