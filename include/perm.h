@@ -73,7 +73,10 @@ typedef struct {
                             kernel with grid barriers; 0 = auto (currently three launches
                             chained with programmatic dependent launch); -1 = never */
     int32_t no_tma;      /* 1: use the plain (non-TMA) row-pass kernels of the 5-pass / sharded
-                            structures even when a TMA stage fits (testing, A/B comparisons) */
+                            structures even when a TMA stage fits (testing, A/B comparisons);
+                            -1: TMA slots hold the data only and the schedule is read from global
+                            memory (the default wherever a line + its schedule exceed a slot:
+                            L >= 16384, n >= 2^27) */
     int32_t direct;      /* low-distribution shortcut (for P with
                             D_w(P) <= 2n/w, e.g. identical and shuffle, the D-designated kernel
                             is coalesced and faster): 0 = auto (on when D_w(P) <= 2n/32),

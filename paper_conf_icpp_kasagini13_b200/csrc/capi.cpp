@@ -300,7 +300,7 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
                        std::to_string(m.strideP) + ",\"cta_stride\":" + std::to_string(m.cta_stride) + "}";
             };
             s += std::string(f ? "," : "") + "{\"phase\":" + std::to_string(rp.phase) +
-                 ",\"tma\":" + std::to_string(rp.tma) + ",\"stages\":" + std::to_string(rp.stages) +
+                 ",\"tma\":" + std::to_string(rp.tma) + ",\"sg\":" + std::to_string(rp.sg) + ",\"stages\":" + std::to_string(rp.stages) +
                  ",\"grid\":" + std::to_string(rp.grid) +
                  ",\"L\":" + std::to_string(P.ph[rp.phase].L) + ",\"E\":" +
                  std::to_string(P.ph[rp.phase].E) + ",\"h\":" + std::to_string(rp.h) +

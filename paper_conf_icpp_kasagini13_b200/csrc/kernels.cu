@@ -85,6 +85,9 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
                  "r"(smem_u32(src)), "r"(bytes)
                  : "memory");
 }
+__device__ __forceinline__ void prefetch_l2_bulk(const void* p, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() {
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
@@ -386,21 +389,30 @@ struct TmaArgs {
 // copy is issued before griddepcontrol.wait: it does not depend on the
 // previous pass. Output: CROSS gather (column chunks of h elements, 128-bit
 // stores) or, for row-major output, a TMA bulk store.
-template <int EPT, bool OUT_CROSS>
+//
+// SG (schedule from global): for long lines (L >= 16384, n >= 2^27) a slot holds
+// the data only; the tile's schedule is pulled into L2 by a bulk prefetch when
+// the slot is armed and read by the permuters straight from global memory
+// (coalesced 64-bit loads), so two or three 64 KiB lines stay in flight per SM.
+template <int EPT, bool OUT_CROSS, bool SG = false>
 __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(const TmaArgs a) {
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x;
     const int L = 1 << a.r.logL, h = 1 << a.r.logh;
-    const int stage_words = a.data_words + a.sched_words;
+    const int stage_words = a.data_words + (SG ? 0 : a.sched_words);
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + a.stages * stage_words);
     const int G = gridDim.x;
     const uint32_t line_bytes = (uint32_t)L * 4u;
     const bool dense = a.r.Ls == L;
-    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (uint32_t)a.sched_words * 4u;
+    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (SG ? 0u : (uint32_t)a.sched_words * 4u);
 
     auto issue_sched = [&](int s, long long t) {
-        bulk_g2s(smem + s * stage_words + a.data_words, a.r.sched + t * a.sched_words,
-                 (uint32_t)a.sched_words * 4u, &bars[s]);
+        if constexpr (SG) {
+            prefetch_l2_bulk(a.r.sched + t * a.sched_words, (uint32_t)a.sched_words * 4u);
+        } else {
+            bulk_g2s(smem + s * stage_words + a.data_words, a.r.sched + t * a.sched_words,
+                     (uint32_t)a.sched_words * 4u, &bars[s]);
+        }
     };
     auto issue_data = [&](int s, long long t) {
         uint32_t* dst = smem + s * stage_words;
@@ -452,8 +464,12 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
         mbar_wait(&bars[s], (uint32_t)(i / a.stages) & 1u);
         if (i < 4) stamp(tr, 2 + 3 * i);
         uint32_t* buf = smem + s * stage_words;
-        permute_lines<EPT, false, true>(buf, buf + a.data_words, a.r.logL, a.r.E, a.r.epw, a.r.w64,
-                                        a.r.Ls);
+        if constexpr (SG)
+            permute_lines<EPT, false, false>(buf, a.r.sched + t * a.sched_words, a.r.logL, a.r.E,
+                                             a.r.epw, a.r.w64, a.r.Ls);
+        else
+            permute_lines<EPT, false, true>(buf, buf + a.data_words, a.r.logL, a.r.E, a.r.epw,
+                                            a.r.w64, a.r.Ls);
         if (i < 4) stamp(tr, 3 + 3 * i);
         if constexpr (OUT_CROSS) {
             tile_store<EPT>(a.r, buf, t);
@@ -730,9 +746,6 @@ __global__ void __launch_bounds__(OUT_CROSS ? 32 + kWsPerm + kWsStore : 32 + kWs
 
 // ------------------------------------------------------------------ fused 3-pass persistent kernel
 
-__device__ __forceinline__ void prefetch_l2_bulk(const void* p, uint32_t bytes) {
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
-}
 __device__ __forceinline__ void fence_proxy_async_global() {
     asm volatile("fence.proxy.async.global;" ::: "memory");
 }
@@ -1547,7 +1560,7 @@ cudaError_t set_smem(K kernel, size_t bytes) {
 size_t tma_smem(const HostPlan& P, int f) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
-    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (size_t)rp.h * (g.L / 32) * g.w64 * 8;
+    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * (g.L / 32) * g.w64 * 8);
     return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
 }
 
@@ -1574,9 +1587,16 @@ cudaError_t prep_ws(HostPlan& P, int f) {
 }
 
 template <int EPT>
+const void* tma_kernel_ptr(bool cross, bool sg) {
+    if (sg) return cross ? (const void*)row_pass_tma_kernel<EPT, true, true>
+                         : (const void*)row_pass_tma_kernel<EPT, false, true>;
+    return cross ? (const void*)row_pass_tma_kernel<EPT, true> : (const void*)row_pass_tma_kernel<EPT, false>;
+}
+
+template <int EPT>
 cudaError_t set_tma_smem(bool cross, size_t smem) {
-    return cross ? set_smem(row_pass_tma_kernel<EPT, true>, smem)
-                 : set_smem(row_pass_tma_kernel<EPT, false>, smem);
+    cudaError_t e = set_smem(tma_kernel_ptr<EPT>(cross, false), smem);
+    return e == cudaSuccess ? set_smem(tma_kernel_ptr<EPT>(cross, true), smem) : e;
 }
 
 template <int EPT>
@@ -1584,9 +1604,8 @@ cudaError_t grid_tma(HostPlan& P, int f) {
     RowPass& rp = P.rp[f];
     const size_t smem = tma_smem(P, f);
     int nb = 0;
-    cudaError_t e = rp.out.cross
-        ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_tma_kernel<EPT, true>, rp.threads, smem)
-        : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_tma_kernel<EPT, false>, rp.threads, smem);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+        &nb, tma_kernel_ptr<EPT>(rp.out.cross != 0, rp.sg != 0), rp.threads, smem);
     if (e != cudaSuccess) return e;
     if (nb < 1) return cudaErrorInvalidConfiguration;
     const long long cap = (long long)nb * sm_count();
@@ -1963,8 +1982,11 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const dim3 grid((unsigned)rp.grid);
         const size_t smem = tma_smem(P, f);
         const bool cx = rp.out.cross != 0;
+        const bool sg = rp.sg != 0;
 #define PERM_TMA_CASE(E_)                                                                      \
     case E_:                                                                                   \
+        if (sg) return cx ? launch(row_pass_tma_kernel<E_, true, true>, grid, block, smem, s, pdl, ta)  \
+                          : launch(row_pass_tma_kernel<E_, false, true>, grid, block, smem, s, pdl, ta); \
         return cx ? launch(row_pass_tma_kernel<E_, true>, grid, block, smem, s, pdl, ta)       \
                   : launch(row_pass_tma_kernel<E_, false>, grid, block, smem, s, pdl, ta);
         switch (rp.ept) {

@@ -52,6 +52,7 @@ struct RowPass {
     int64_t seg_len = 0, seg_stride = 0;
     int32_t tma = 0;          // 1: persistent TMA-pipelined kernel (contiguous input lines)
     int32_t stages = 0;       // TMA ring depth
+    int32_t sg = 0;           // 1 (tma == 1): schedule read from global (L2-prefetched), slots hold data only
     int64_t grid = 0;         // persistent CTAs (set at upload from the occupancy query)
     int32_t h = 0;            // lines per CTA (tile)
     int32_t Ls = 0;           // shared-memory line stride (elements) = L + pad

@@ -885,9 +885,19 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.in = runs(L, 0, h * L);
             rp.out = runs(L, 0, h * L);
             // TMA pipeline when `stages` tiles (lines + schedule) fit in shared memory
-            rp.tma = (stages * stage_bytes(h, f, 0) <= kSmemBudget &&
-                      (h * (L / kW) * P.ph[f].w64 * 2) % 4 == 0 && !(opt && opt->no_tma)) ? 1 : 0;
+            const bool sched16 = (h * (L / kW) * P.ph[f].w64 * 2) % 4 == 0;
+            const bool no_tma = opt && opt->no_tma > 0;
+            const bool force_sg = opt && opt->no_tma < 0;
+            rp.tma = (stages * stage_bytes(h, f, 0) <= kSmemBudget && sched16 && !no_tma && !force_sg) ? 1 : 0;
             rp.stages = rp.tma ? stages : 0;
+            // long lines (L >= 16384): the slots hold the data only and the schedule is
+            // read from global (L2-prefetched), so 1-3 lines stay in flight per SM
+            if (!rp.tma && sched16 && !no_tma && h * L * 4 <= kSmemBudget) {
+                rp.tma = 1;
+                rp.sg = 1;
+                const int64_t fit = kSmemBudget / (h * L * 4);
+                rp.stages = (opt && opt->stages > 0) ? opt->stages : (int)std::min<int64_t>(4, fit);
+            }
         }
     }
     for (int f = 0; f < 3; ++f) {
@@ -915,7 +925,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 rp.conflicts_out = rp.out.cross ? simulate_conflicts(tmp, g, false) : 1;
             }
             if ((rp.h * (g.L / kW) * g.w64 * 2) % 4) { err = "TMA tile schedule is not 16-byte sized"; return PERM_EINVAL; }
-            if (rp.stages * stage_bytes(rp.h, rp.phase, pad) > kSmemBudget) {
+            const int64_t sb = rp.sg ? (int64_t)rp.h * (g.L + pad) * 4 : stage_bytes(rp.h, rp.phase, pad);
+            if (rp.stages * sb > kSmemBudget) {
                 err = "TMA stages exceed the shared-memory budget; lower h or stages";
                 return PERM_EINVAL;
             }

@@ -377,3 +377,18 @@ def test_run_pass_chain_is_apply(P, k):
         assert np.array_equal(host_words(db), OA.apply_ref(p, a))
         with pytest.raises(P.PermError):
             plan.run_pass(3, da)
+
+
+@pytest.mark.parametrize("fam", ["random", "bitrev", "transpose"])
+@pytest.mark.parametrize("k", [12, 16, 19, 22])
+def test_schedule_from_global(P, fam, k):
+    # 5-pass TMA row passes whose slots hold the data only; the permuters read the
+    # schedule from global memory (the default for lines of >= 16384 words, n >= 2^27)
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=11 + k)
+    a = W.make_data(n)
+    ref = OA.apply_ref(p, a)
+    for stages in (0, 1, 3):
+        b, info = run(P, p, a, passes=5, no_tma=-1, stages=stages)
+        assert info["passes"] == 5
+        assert np.array_equal(b, ref), stages
