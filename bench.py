@@ -58,6 +58,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--no-c3", action="store_true",
+                    help="skip the n = 2^26 random side measurement (BASELINE configs[2])")
     return ap.parse_args()
 
 
@@ -269,6 +271,82 @@ def run_sharded(args, rank, world, local):
     dist.destroy_process_group()
 
 
+def sched_bytes_per_elt(info: dict, desc: dict) -> list:
+    """Schedule bytes per element of each row pass, from the plan's entry format."""
+    if desc.get("layout") == 3:
+        # TLC format: each lane's ept entries are one bitstream of nwords 32-bit words
+        return [4 * t["nwords"] / t["ept"] for t in desc["tlc"]]
+    # W64 format: floor(64/E) entries per 64-bit word, ceil(32/epw) words per warp-round
+    return [8 * (-(-32 // (64 // e))) / 32 for e in info["entry_bits"]]
+
+
+def large_config(pkg, dev, stream, flush_l2, log2n: int, fam: str, steps: int, peak: float) -> dict:
+    """BASELINE configs[2]: n = 2^26 random on one GPU -- whole-apply time against the HBM
+    roofline of its passes' algorithmic bytes, the conventional kernel, plan build, and a
+    sampled bit-exact check (b[P(i)] = a[i] on 2^20 random i)."""
+    import torch
+    n = 1 << log2n
+    p = W.make_perm(fam, n)
+    a = W.make_data(n)
+    t0 = time.perf_counter()
+    plan = pkg.Plan(p)
+    build_s = time.perf_counter() - t0
+    info, desc = plan.info(), plan.describe()
+    dA = torch.from_numpy(a.view(np.int32)).to(dev)
+    dB = torch.empty_like(dA)
+    dP = torch.from_numpy(p).to(dev)
+
+    def med(fn):
+        ts = []
+        for i in range(steps + 3):
+            flush_l2()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            fn()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            if i >= 3:
+                ts.append(e0.elapsed_time(e1))
+        return statistics.median(ts)
+
+    t_conv = med(lambda: pkg.scatter_baseline(dP, dA, dB, stream))
+    t_apply = med(lambda: plan.apply(dA, dB, stream))
+    b = dB.cpu().numpy().view(np.uint32)
+    idx = np.random.default_rng(7).integers(0, n, size=1 << 20)
+    ok = bool(np.array_equal(b[p[idx]], a[idx]))
+    plan.set_profiling(True)
+    ks = []
+    for _ in range(max(3, steps // 2)):
+        flush_l2()
+        plan.apply(dA, dB, stream)
+        ks.append(plan.pass_times())
+    plan.set_profiling(False)
+    per_k = [statistics.mean(k[i] for k in ks) for i in range(len(ks[0]))]
+    sb = sched_bytes_per_elt(info, desc)
+    if info["passes"] == 5:
+        kinds = ["R1", "T", "R2", "T", "R3"]
+        alg = [8 * n + n * sb[0], 8 * n, 8 * n + n * sb[1], 8 * n, 8 * n + n * sb[2]]
+    else:
+        kinds = ["R1", "R2", "R3"][:len(per_k)]
+        alg = [8 * n + n * sb[i] for i in range(len(per_k))]
+    dom = int(np.argmax(per_k))
+    apply_alg = sum(alg)
+    plan.close()
+    return {"workload": f"n=2^{log2n} {fam} float32 (BASELINE configs[2]), cold L2",
+            "apply_us": 1e3 * t_apply, "conventional_us": 1e3 * t_conv,
+            "speedup_vs_conventional": t_conv / t_apply,
+            "effective_gbs": 2 * n * 4 / (t_apply * 1e-3) / 1e9,
+            "passes": info["passes"], "plan_build_s": build_s, "gpu_planner": info["gpu_planner"],
+            "apply_roofline": {"bound": "hbm", "algorithmic_bytes": apply_alg,
+                               "achieved": apply_alg / (t_apply * 1e-3) / 1e9, "peak": peak,
+                               "frac": apply_alg / (t_apply * 1e-3) / 1e9 / peak},
+            "kernel_roofline": {"kernel": kinds[dom], "kernel_ms": per_k[dom],
+                                "achieved": alg[dom] / (per_k[dom] * 1e-3) / 1e9,
+                                "frac": alg[dom] / (per_k[dom] * 1e-3) / 1e9 / peak},
+            "per_kernel_ms": dict(zip([f"{k}#{i}" for i, k in enumerate(kinds)], per_k)),
+            "sampled_bitexact": ok, "sample": "b[P(i)] == a[i] for 2^20 random i"}
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -424,14 +502,8 @@ def main():
                          f"random plans and inputs (all cold: {K} x (input + schedule) > L2), "
                          f"L2 flushed before each group; per-launch mean")
     dom = int(np.argmax(mean_k))
-    E = info["entry_bits"]
     desc = plans[sched_fams[0]].describe()
-    if desc.get("layout") == 3:
-        # TLC format: each lane's ept entries are one bitstream of nwords 32-bit words
-        sbpe = [4 * t["nwords"] / t["ept"] for t in desc["tlc"]]
-    else:
-        # W64 format: floor(64/E) entries per 64-bit word, ceil(32/epw) words per warp-round
-        sbpe = [8 * (-(-32 // (64 // e))) / 32 for e in E]
+    sbpe = sched_bytes_per_elt(info, desc)
     if info["direct"]:
         kinds = ["D-designated (direct)"]
         alg = [2 * n * 4 + n * 4]
@@ -505,6 +577,11 @@ def main():
         sched_only[f] = 1e3 * statistics.median(ts)
         pl.close()
 
+    c3 = None
+    if rank == 0 and not args.no_c3 and args.log2n == 22:
+        c3 = large_config(pkg, dev, stream, flush_l2, 26, "random", max(5, args.steps // 2),
+                          peaks["hbm_gbs"])
+
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
         cpu = cpu_oracle_baseline(host, n, args.cpu_seconds)
@@ -531,6 +608,7 @@ def main():
             "sched_bytes": info["sched_bytes"],
             "bitexact_check": ok,
             "roofline": roofline,
+            "c3_2pow26_random": c3,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": args.steps * sum(infos[f]["kernels_per_apply"] for f in fams),

@@ -87,7 +87,10 @@ typedef struct {
                              destination); 1 = compact (the line index inside the tile is implied
                              by the source offset: 19 instead of 21 bits at n = 2^22) wherever a
                              kernel is compiled for its width (not with fuse = 1) */
-    int32_t reserved[1];
+    int32_t gpu_planner; /* where the offline colourings run: 1 = on the
+                            current CUDA device (gplan.cu: Euler split with ruling-set cycle
+                            labelling), -1 = host threads (planner.cpp), 0 = auto (device for
+                            device plans with n >= 2^20, host otherwise) */
 } perm_plan_options;
 
 typedef struct {
@@ -109,7 +112,7 @@ typedef struct {
     int64_t block_elems;         /* n / world^2: one all-to-all block */
     int64_t distribution;        /* D_w(P), w = 32 (L389-L401): address groups the warps write */
     int32_t direct;              /* 1: perm_apply runs the D-designated kernel (low D_w) */
-    int32_t pad0;
+    int32_t gpu_planner;         /* 1: the colourings ran on the GPU (gplan.cu), 0: on the host */
 } perm_plan_info;
 
 /* ------------------------------------------------------------------ plans */

@@ -37,7 +37,7 @@ class PlanOptions(ctypes.Structure):
     _fields_ = [("passes", ctypes.c_int32), ("h1", ctypes.c_int32), ("h2", ctypes.c_int32),
                 ("h3", ctypes.c_int32), ("layout", ctypes.c_int32), ("stages", ctypes.c_int32),
                 ("fuse", ctypes.c_int32), ("no_tma", ctypes.c_int32), ("direct", ctypes.c_int32),
-                ("log2c", ctypes.c_int32), ("sched_format", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("log2c", ctypes.c_int32), ("sched_format", ctypes.c_int32), ("gpu_planner", ctypes.c_int32)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -50,7 +50,7 @@ class PlanInfo(ctypes.Structure):
                 ("build_ms_upload", ctypes.c_double), ("world", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("shard_elems", ctypes.c_int64),
                 ("block_elems", ctypes.c_int64), ("distribution", ctypes.c_int64),
-                ("direct", ctypes.c_int32), ("pad0", ctypes.c_int32)]
+                ("direct", ctypes.c_int32), ("gpu_planner", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {}
@@ -140,13 +140,13 @@ class Plan:
     def __init__(self, p, elem_bytes: int = 4, passes: int = 0, h=(0, 0, 0),
                  device: bool = True, layout: int = 0, stages: int = 0, fuse: int = 0,
                  world: int = 0, rank: int = 0, no_tma: int = 0, direct: int = 0, log2c: int = 0,
-                 sched_format: int = 0):
+                 sched_format: int = 0, gpu_planner: int = 0):
         """world > 0: row-sharded plan of rank `rank` (see perm_plan_create_sharded)."""
         p = _as_int32_host(p)
         self.n = int(p.size)
         self.elem_bytes = elem_bytes
         opt = PlanOptions(passes, h[0], h[1], h[2], layout, stages, fuse, no_tma, direct, log2c,
-                          sched_format)
+                          sched_format, gpu_planner)
         if world > 0:
             fn = _plan_create_sharded if device else _plan_create_sharded_host
             handle = fn(p.ctypes.data, self.n, elem_bytes, world, rank, ctypes.byref(opt))

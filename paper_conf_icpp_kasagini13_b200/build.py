@@ -12,8 +12,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(PKG, "csrc")
 ROOT = os.path.dirname(PKG)
 LIB = os.path.join(PKG, "libperm.so")
-SOURCES = ["planner.cpp", "capi.cpp", "kernels.cu"]
-HEADERS = ["plan.hpp", "kernels.hpp"]
+SOURCES = ["planner.cpp", "capi.cpp", "kernels.cu", "gplan.cu"]
+HEADERS = ["plan.hpp", "kernels.hpp", "gplan.hpp"]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",

@@ -139,9 +139,13 @@ perm_plan* create(const int32_t* p, int64_t n, int32_t eb, const perm_plan_optio
     if (!pl) { fail(PERM_ENOMEM, "out of host memory"); return nullptr; }
     std::string err;
     int st;
+    // where the colourings run: auto -> the device for device plans with n >= 2^20
+    perm_plan_options o{};
+    if (opt) o = *opt;
+    if (o.gpu_planner == 0) o.gpu_planner = (device && n >= (int64_t(1) << 20)) ? 1 : -1;
     try {
-        st = world > 0 ? perm::build_sharded_plan(p, n, eb, world, rank, opt, pl->host, err)
-                       : perm::build_host_plan(p, n, eb, opt, pl->host, err);
+        st = world > 0 ? perm::build_sharded_plan(p, n, eb, world, rank, &o, pl->host, err)
+                       : perm::build_host_plan(p, n, eb, &o, pl->host, err);
     } catch (const std::bad_alloc&) {
         st = PERM_ENOMEM;
         err = "out of host memory while planning";
@@ -249,6 +253,7 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->kernels_per_apply = (plan->d_p || P.fused3) ? 1 : P.passes;
     out->distribution = P.distribution;
     out->direct = P.direct;
+    out->gpu_planner = P.gpu_planner;
     for (int f = 0; f < 3; ++f) {
         out->entry_bits[f] = P.layout == 3 ? P.tp[f].E : P.ph[f].E;
         out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
@@ -300,7 +305,7 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
                        std::to_string(m.strideP) + ",\"cta_stride\":" + std::to_string(m.cta_stride) + "}";
             };
             s += std::string(f ? "," : "") + "{\"phase\":" + std::to_string(rp.phase) +
-                 ",\"tma\":" + std::to_string(rp.tma) + ",\"sg\":" + std::to_string(rp.sg) + ",\"stages\":" + std::to_string(rp.stages) +
+                 ",\"tma\":" + std::to_string(rp.tma) + ",\"sg\":" + std::to_string(rp.sg) + ",\"split\":" + std::to_string(rp.split) + ",\"stages\":" + std::to_string(rp.stages) +
                  ",\"grid\":" + std::to_string(rp.grid) +
                  ",\"L\":" + std::to_string(P.ph[rp.phase].L) + ",\"E\":" +
                  std::to_string(P.ph[rp.phase].E) + ",\"h\":" + std::to_string(rp.h) +

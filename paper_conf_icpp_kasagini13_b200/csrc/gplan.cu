@@ -1,0 +1,309 @@
+// gplan.cu — the offline colourings of the plan builder on the GPU.
+//
+// PAPER.md Thm 6 (L515) only proves that a d-regular bipartite multigraph has a
+// proper d-edge-colouring (König); the paper colours offline and never times it.
+// Both colourings of the method are of that kind and every degree here is a
+// power of two, so we use Euler splitting, as the host planner does
+// (planner.cpp), restructured for thousands of threads:
+//
+//   level l (degree d = d0 >> l, edges grouped in aligned blocks of d per
+//   vertex on each side, ordU / ordV = edge ids in block order):
+//   1. pair positions (2i, 2i+1) of every block: partner_U(e), partner_V(e);
+//   2. the pairings form disjoint cycles alternating V- and U-links; the map
+//      g = partner_U o partner_V walks every second edge of a cycle, so each
+//      cycle is two g-orbits and colouring one orbit 0 and the other 1 gives
+//      every vertex exactly half its edges of each colour;
+//   3. orbit labels by a ruling set: ~1/32 of the edges (hash-selected) are
+//      rulers; each ruler walks g to the next ruler and stamps its segment; the
+//      rulers (plus the edges of ruler-free orbits, which are short) then find
+//      the minimum ruler id of their orbit by synchronous pointer jumping over
+//      a compacted list: O(E) work per level instead of O(E log E);
+//   4. colour bit b(e) = [label(e) < label(partner_V(e))] (the two orbits of a
+//      cycle have different labels);
+//   5. stable split of every block into its b = 0 half and its b = 1 half
+//      (a pair holds one edge of each colour, so the destination of position
+//      2i + j is block*d + b*d/2 + i: no scan).
+//   After log2(d0) levels every block is one edge: colour(ordU[q]) = q mod d0.
+//
+// Row level (a1): vertices = source rows (edge x in block x >> log c, i.e.
+// ordU = identity) and destination rows (ordV[P(x)] = x), d0 = c.
+// Bank level (a3, per line or per TLC tile of B elements): vertices =
+// (block, source bank) and (block, destination bank), d0 = B / 32.
+// The result is checked like the host planner's: by the oracle's invariants.
+
+#include <cuda_runtime.h>
+
+#include <chrono>
+#include <cstdint>
+#include <vector>
+
+#include "gplan.hpp"
+
+namespace perm {
+
+namespace {
+
+constexpr int kRulerLog = 5;   // 1 in 32 edges starts a walk
+
+__device__ __forceinline__ uint32_t mix32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352du;
+    x ^= x >> 15; x *= 0x846ca68bu;
+    x ^= x >> 16;
+    return x;
+}
+__device__ __forceinline__ bool is_ruler(uint32_t e, uint32_t seed) {
+    return (mix32(e ^ seed) & ((1u << kRulerLog) - 1u)) == 0u;
+}
+
+__global__ void k_pair(const uint32_t* __restrict__ ord, uint32_t* __restrict__ partner, int64_t E) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < E; q += (int64_t)gridDim.x * blockDim.x)
+        partner[ord[q]] = ord[q ^ 1];
+}
+
+__global__ void k_compose(const uint32_t* __restrict__ pU, const uint32_t* __restrict__ pV,
+                          uint32_t* __restrict__ g, int64_t E) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x)
+        g[e] = pU[pV[e]];
+}
+
+// every ruler stamps its segment (itself and the non-rulers up to the next ruler)
+__global__ void k_walk(const uint32_t* __restrict__ g, uint32_t* __restrict__ seg,
+                       uint32_t* __restrict__ nxt, int64_t E, uint32_t seed) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x) {
+        if (!is_ruler((uint32_t)e, seed)) continue;
+        seg[e] = (uint32_t)e;
+        uint32_t x = g[e];
+        while (!is_ruler(x, seed)) {
+            seg[x] = (uint32_t)e;
+            x = g[x];
+        }
+        nxt[e] = x;
+    }
+}
+
+// nodes of the reduced graph: rulers (next = next ruler) and the edges of
+// ruler-free orbits (seg still ~0: next = g); compacted into list slots
+__global__ void k_compact(const uint32_t* __restrict__ g, uint32_t* __restrict__ seg,
+                          uint32_t* __restrict__ nxt, uint32_t* __restrict__ slotof,
+                          uint32_t* __restrict__ node, unsigned long long* __restrict__ count, int64_t E) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t s = seg[e];
+        if (s == 0xFFFFFFFFu) {
+            seg[e] = (uint32_t)e;
+            nxt[e] = g[e];
+            s = (uint32_t)e;
+        }
+        if (s == (uint32_t)e) {
+            const uint32_t slot = (uint32_t)atomicAdd(count, 1ull);
+            slotof[e] = slot;
+            node[slot] = (uint32_t)e;
+        }
+    }
+}
+
+__global__ void k_reduced_init(const uint32_t* __restrict__ node, const uint32_t* __restrict__ nxt,
+                               const uint32_t* __restrict__ slotof, uint32_t* __restrict__ lab,
+                               uint32_t* __restrict__ nx, int64_t R) {
+    for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < R; s += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t e = node[s];
+        lab[s] = e;
+        nx[s] = slotof[nxt[e]];
+    }
+}
+
+// synchronous pointer jumping (ping-pong buffers): after round j, lab = min over
+// the next 2^j nodes of the orbit; a round without a change means converged
+__global__ void k_jump(const uint32_t* __restrict__ lab, const uint32_t* __restrict__ nx,
+                       uint32_t* __restrict__ lab2, uint32_t* __restrict__ nx2, int64_t R,
+                       int* __restrict__ changed) {
+    int ch = 0;
+    for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < R; s += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t n1 = nx[s];
+        const uint32_t a = lab[s], b = lab[n1];
+        const uint32_t m = b < a ? b : a;
+        ch |= m != a;
+        lab2[s] = m;
+        nx2[s] = nx[n1];
+    }
+    if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+
+__global__ void k_label(const uint32_t* __restrict__ seg, const uint32_t* __restrict__ slotof,
+                        const uint32_t* __restrict__ rlab, uint32_t* __restrict__ lab, int64_t E) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x)
+        lab[e] = rlab[slotof[seg[e]]];
+}
+
+__global__ void k_split(const uint32_t* __restrict__ ord, uint32_t* __restrict__ ord2,
+                        const uint32_t* __restrict__ lab, const uint32_t* __restrict__ pV, int64_t E, int logd) {
+    const int64_t half = (int64_t)1 << (logd - 1);
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < E; q += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t e = ord[q];
+        const int64_t blk = q >> logd, i = (q & ((half << 1) - 1)) >> 1;
+        const int64_t b = lab[e] < lab[pV[e]] ? 0 : 1;
+        ord2[(blk << logd) + b * half + i] = e;
+    }
+}
+
+__global__ void k_final(const uint32_t* __restrict__ ord, uint16_t* __restrict__ col, int64_t E, uint32_t dmask) {
+    for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < E; q += (int64_t)gridDim.x * blockDim.x)
+        col[ord[q]] = (uint16_t)(q & dmask);
+}
+
+__global__ void k_row_orders(const int32_t* __restrict__ p, uint32_t* __restrict__ ordU,
+                             uint32_t* __restrict__ ordV, int64_t n) {
+    for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n; x += (int64_t)gridDim.x * blockDim.x) {
+        ordU[x] = (uint32_t)x;
+        ordV[p[x]] = (uint32_t)x;      // sorted by P(x): blocks of c per destination row
+    }
+}
+
+// bank level: block of B = 2^logB elements (a line or a TLC tile); vertex
+// (block, key & 31) on each side, position (key & 31) * B/32 + (key >> 5)
+__global__ void k_bank_orders(const uint16_t* __restrict__ keyU, const uint16_t* __restrict__ keyV,
+                              uint32_t* __restrict__ ordU, uint32_t* __restrict__ ordV, int64_t E, int logB) {
+    const int sh = logB - 5;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t base = (e >> logB) << logB;
+        const uint32_t ku = keyU ? (uint32_t)keyU[e] : (uint32_t)(e & ((1 << logB) - 1)), kv = keyV[e];
+        ordU[base + ((int64_t)(ku & 31) << sh) + (ku >> 5)] = (uint32_t)e;
+        ordV[base + ((int64_t)(kv & 31) << sh) + (kv >> 5)] = (uint32_t)e;
+    }
+}
+
+struct DevBuf {
+    void* p = nullptr;
+    ~DevBuf() { if (p) cudaFree(p); }
+};
+
+#define GP_TRY(x)                              \
+    do {                                       \
+        cudaError_t e_ = (x);                  \
+        if (e_ != cudaSuccess) return e_;      \
+    } while (0)
+
+unsigned grid_for(int64_t E) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t want = (E + 255) / 256;
+    const int64_t cap = (int64_t)sms * 8;
+    return (unsigned)(want < cap ? (want > 0 ? want : 1) : cap);
+}
+
+// Euler split of the blocks in ordU / ordV (device, E edges, degree 2^logd0);
+// writes colour[e] in [0, 2^logd0). ordU / ordV are clobbered.
+cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int logd0, uint16_t* colour,
+                               cudaStream_t s, GpuPlanStats* st) {
+    const unsigned G = grid_for(E), T = 256;
+    DevBuf bU2, bV2, bpU, bpV, bg, bseg, bnxt, bslot, bnode, blab, blab2, bnx, bnx2, bcnt, bch;
+    const size_t W = (size_t)E * 4;
+    GP_TRY(cudaMalloc(&bU2.p, W));
+    GP_TRY(cudaMalloc(&bV2.p, W));
+    GP_TRY(cudaMalloc(&bpU.p, W));
+    GP_TRY(cudaMalloc(&bpV.p, W));
+    GP_TRY(cudaMalloc(&bg.p, W));
+    GP_TRY(cudaMalloc(&bseg.p, W));
+    GP_TRY(cudaMalloc(&bnxt.p, W));
+    GP_TRY(cudaMalloc(&bslot.p, W));
+    GP_TRY(cudaMalloc(&bnode.p, W));
+    GP_TRY(cudaMalloc(&blab.p, W));
+    GP_TRY(cudaMalloc(&blab2.p, W));
+    GP_TRY(cudaMalloc(&bnx.p, W));
+    GP_TRY(cudaMalloc(&bnx2.p, W));
+    GP_TRY(cudaMalloc(&bcnt.p, 8));
+    GP_TRY(cudaMalloc(&bch.p, 4));
+    uint32_t *U = ordU, *V = ordV, *U2 = (uint32_t*)bU2.p, *V2 = (uint32_t*)bV2.p;
+    uint32_t *pU = (uint32_t*)bpU.p, *pV = (uint32_t*)bpV.p, *g = (uint32_t*)bg.p;
+    uint32_t *seg = (uint32_t*)bseg.p, *nxt = (uint32_t*)bnxt.p, *slotof = (uint32_t*)bslot.p;
+    uint32_t *node = (uint32_t*)bnode.p, *lab = (uint32_t*)blab.p, *lab2 = (uint32_t*)blab2.p;
+    uint32_t *nx = (uint32_t*)bnx.p, *nx2 = (uint32_t*)bnx2.p;
+    unsigned long long* cnt = (unsigned long long*)bcnt.p;
+    int* changed = (int*)bch.p;
+    for (int l = 0; l < logd0; ++l) {
+        const int logd = logd0 - l;
+        k_pair<<<G, T, 0, s>>>(U, pU, E);
+        k_pair<<<G, T, 0, s>>>(V, pV, E);
+        k_compose<<<G, T, 0, s>>>(pU, pV, g, E);
+        GP_TRY(cudaMemsetAsync(seg, 0xFF, W, s));
+        GP_TRY(cudaMemsetAsync(cnt, 0, 8, s));
+        const uint32_t seed = 0x9E3779B9u * (uint32_t)(l + 1);
+        k_walk<<<G, T, 0, s>>>(g, seg, nxt, E, seed);
+        k_compact<<<G, T, 0, s>>>(g, seg, nxt, slotof, node, cnt, E);
+        unsigned long long R = 0;
+        GP_TRY(cudaMemcpyAsync(&R, cnt, 8, cudaMemcpyDeviceToHost, s));
+        GP_TRY(cudaStreamSynchronize(s));
+        const unsigned GR = grid_for((int64_t)R);
+        k_reduced_init<<<GR, T, 0, s>>>(node, nxt, slotof, lab, nx, (int64_t)R);
+        uint32_t *la = lab, *lb = lab2, *na = nx, *nb = nx2;
+        for (int round = 0;; ++round) {
+            int h = 0;
+            GP_TRY(cudaMemsetAsync(changed, 0, 4, s));
+            k_jump<<<GR, T, 0, s>>>(la, na, lb, nb, (int64_t)R, changed);
+            GP_TRY(cudaMemcpyAsync(&h, changed, 4, cudaMemcpyDeviceToHost, s));
+            GP_TRY(cudaStreamSynchronize(s));
+            std::swap(la, lb);
+            std::swap(na, nb);
+            if (st) st->jump_rounds += 1;
+            if (!h || round > 64) break;
+        }
+        // la = final labels of the reduced nodes; spread to every edge (into lb: free)
+        k_label<<<G, T, 0, s>>>(seg, slotof, la, lb, E);
+        k_split<<<G, T, 0, s>>>(U, U2, lb, pV, E, logd);
+        k_split<<<G, T, 0, s>>>(V, V2, lb, pV, E, logd);
+        std::swap(U, U2);
+        std::swap(V, V2);
+        if (st) { st->levels += 1; st->reduced_nodes += (int64_t)R; }
+        GP_TRY(cudaGetLastError());
+    }
+    k_final<<<G, T, 0, s>>>(U, colour, E, (uint32_t)((1u << logd0) - 1u));
+    GP_TRY(cudaGetLastError());
+    return cudaStreamSynchronize(s);
+}
+
+}  // namespace
+
+cudaError_t gpu_row_colour(const int32_t* p_host, int64_t n, int logc, uint16_t* kappa_host,
+                           GpuPlanStats* st) {
+    cudaStream_t s = nullptr;
+    GP_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+    DevBuf bp, bU, bV, bc;
+    GP_TRY(cudaMalloc(&bp.p, (size_t)n * 4));
+    GP_TRY(cudaMalloc(&bU.p, (size_t)n * 4));
+    GP_TRY(cudaMalloc(&bV.p, (size_t)n * 4));
+    GP_TRY(cudaMalloc(&bc.p, (size_t)n * 2));
+    GP_TRY(cudaMemcpyAsync(bp.p, p_host, (size_t)n * 4, cudaMemcpyHostToDevice, s));
+    k_row_orders<<<grid_for(n), 256, 0, s>>>((const int32_t*)bp.p, (uint32_t*)bU.p, (uint32_t*)bV.p, n);
+    GP_TRY(cudaGetLastError());
+    cudaFree(bp.p);
+    bp.p = nullptr;
+    GP_TRY(euler_split_device((uint32_t*)bU.p, (uint32_t*)bV.p, n, logc, (uint16_t*)bc.p, s, st));
+    GP_TRY(cudaMemcpyAsync(kappa_host, bc.p, (size_t)n * 2, cudaMemcpyDeviceToHost, s));
+    return cudaStreamSynchronize(s);
+}
+
+cudaError_t gpu_bank_colour(const uint16_t* keyU_host, const uint16_t* keyV_host, int64_t E, int logB,
+                            uint16_t* col_host, GpuPlanStats* st) {
+    // B = 32 (a 32-element line): degree 1, every edge gets colour 0 (no split level)
+    if (logB < 5 || logB > 16 || (E & ((int64_t(1) << logB) - 1))) return cudaErrorInvalidValue;
+    cudaStream_t s = nullptr;
+    GP_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+    DevBuf bku, bkv, bU, bV, bc;
+    if (keyU_host) GP_TRY(cudaMalloc(&bku.p, (size_t)E * 2));
+    GP_TRY(cudaMalloc(&bkv.p, (size_t)E * 2));
+    GP_TRY(cudaMalloc(&bU.p, (size_t)E * 4));
+    GP_TRY(cudaMalloc(&bV.p, (size_t)E * 4));
+    GP_TRY(cudaMalloc(&bc.p, (size_t)E * 2));
+    if (keyU_host) GP_TRY(cudaMemcpyAsync(bku.p, keyU_host, (size_t)E * 2, cudaMemcpyHostToDevice, s));
+    GP_TRY(cudaMemcpyAsync(bkv.p, keyV_host, (size_t)E * 2, cudaMemcpyHostToDevice, s));
+    k_bank_orders<<<grid_for(E), 256, 0, s>>>((const uint16_t*)bku.p, (const uint16_t*)bkv.p,
+                                              (uint32_t*)bU.p, (uint32_t*)bV.p, E, logB);
+    GP_TRY(cudaGetLastError());
+    GP_TRY(euler_split_device((uint32_t*)bU.p, (uint32_t*)bV.p, E, logB - 5, (uint16_t*)bc.p, s, st));
+    GP_TRY(cudaMemcpyAsync(col_host, bc.p, (size_t)E * 2, cudaMemcpyDeviceToHost, s));
+    return cudaStreamSynchronize(s);
+}
+
+}  // namespace perm

@@ -504,6 +504,134 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
     stamp(tr, 14);
 }
 
+// ------------------------------------------------------------------ row pass, half-line ring
+
+// In-place permutation of ONE line whose two halves sit in shared-memory words
+// [o0, o0 + L/2) and [o1, o1 + L/2) (any two slots of the half-line ring).
+// Same warp-round structure and W64 schedule (read from global) as
+// permute_lines; slots are 64 KiB apart, so position pos keeps bank pos mod 32
+// and the rounds stay conflict-free.
+template <int EPT>
+__device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1, const uint32_t* __restrict__ sched,
+                                                   int logL, int E, int epw, int w64) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, W = blockDim.x >> 5;
+    const int lh = logL - 1;
+    const int hmask = (1 << lh) - 1;
+    const int wsel = lane / epw;
+    const int sh = E * (lane - wsel * epw);
+    const uint32_t mask = (1u << E) - 1u;
+    const uint32_t tmask = (1u << logL) - 1u;
+    const uint2* sp = reinterpret_cast<const uint2*>(sched) + warp * w64 + wsel;
+    const int step = W * w64;
+    uint32_t v[EPT];
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) {
+        const uint2 wd = __ldg(sp + m * step);
+        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
+        const uint32_t e = (uint32_t)(w >> sh) & mask;
+        const int s = (int)((e >> logL) << 5) + lane;
+        v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) {
+        const uint2 wd = __ldg(sp + m * step);
+        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
+        const int t = (int)(((uint32_t)(w >> sh) & mask) & tmask);
+        sm[((t >> lh) ? o1 : o0) + (t & hmask)] = v[m];
+    }
+    __syncthreads();
+}
+
+// Row-wise pass (Lemma 7) for lines of L = 32768 words (n = 2^29, 2^30), where one
+// line + any second buffer exceed shared memory: a ring of THREE half-line slots
+// (3 x 64 KiB). Line i occupies slots (2i mod 3, 2i+1 mod 3); while line i is
+// permuted, the first half of line i+1 is already loading into the third slot;
+// once the TMA store of line i's first half has read its slot, the second half
+// of line i+1 loads there, and once the second half's store has read its slot,
+// the first half of line i+2 loads there. So loads overlap the permute and the
+// stores instead of alternating with them (1.5 lines resident per SM).
+// Half-load j = 2i + q uses slot j mod 3 and is that slot's (j div 3)-th fill:
+// the mbarrier parity every thread waits on is (j div 3) & 1. Schedule: W64,
+// read from global, L2-prefetched one line ahead. Row-major output only.
+template <int EPT>
+__global__ void __launch_bounds__(1024, 1) row_pass_split_kernel(const TmaArgs a) {
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x;
+    const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + 3 * HALF);
+    const int G = gridDim.x;
+    const uint32_t half_bytes = (uint32_t)HALF * 4u;
+    const long long my_lines = a.ntiles > (int)blockIdx.x ? (a.ntiles - 1 - (int)blockIdx.x) / G + 1 : 0;
+
+    // half-load j of this CTA: line j >> 1, half j & 1, slot j % 3
+    auto issue_half = [&](long long j) {
+        const long long i = j >> 1;
+        if (i >= my_lines) return;
+        const int q = (int)(j & 1), slot = (int)(j % 3);
+        const long long t = blockIdx.x + i * G;
+        uint32_t* dst = smem + slot * HALF;
+        mbar_arrive_expect_tx(&bars[slot], half_bytes);
+        if (q == 0) prefetch_l2_bulk(a.r.sched + t * a.sched_words, (uint32_t)a.sched_words * 4u);
+        if (a.r.in_segs > 1) {
+            const uint32_t sb = (uint32_t)a.r.seg_len * 4u;
+            for (int g = 0; g < a.r.in_segs; ++g) {
+                const long long off = (long long)g * a.r.seg_len;
+                if ((off >> lh) != q) continue;
+                bulk_g2s(dst + (off & (HALF - 1)), a.r.in + g * a.r.seg_stride + t * a.r.seg_len, sb, &bars[slot]);
+            }
+        } else {
+            bulk_g2s(dst, a.r.in + t * (long long)L + (long long)q * HALF, half_bytes, &bars[slot]);
+        }
+    };
+
+    unsigned long long* tr = a.r.trace;
+    stamp(tr, 0);
+    if (tid == 0) {
+        for (int s = 0; s < 3; ++s) mbar_init(&bars[s], 1);
+        fence_mbar_init();
+        if (my_lines > 0) prefetch_l2_bulk(a.r.sched + (long long)blockIdx.x * a.sched_words,
+                                           (uint32_t)a.sched_words * 4u);
+    }
+    __syncthreads();
+    pdl_wait();
+    stamp(tr, 1);
+    if (tid == 0) {
+        issue_half(0);
+        issue_half(1);
+        issue_half(2);
+    }
+    pdl_launch_dependents();
+    for (long long i = 0; i < my_lines; ++i) {
+        const long long t = blockIdx.x + i * G;
+        const long long j0 = 2 * i, j1 = 2 * i + 1;
+        const int s0 = (int)(j0 % 3), s1 = (int)(j1 % 3);
+        mbar_wait(&bars[s0], (uint32_t)(j0 / 3) & 1u);
+        mbar_wait(&bars[s1], (uint32_t)(j1 / 3) & 1u);
+        if (i < 4) stamp(tr, 2 + 3 * i);
+        permute_split_line<EPT>(smem, s0 * HALF, s1 * HALF, a.r.sched + t * a.sched_words, a.r.logL, a.r.E,
+                                a.r.epw, a.r.w64);
+        if (i < 4) stamp(tr, 3 + 3 * i);
+        if (tid == 0) {
+            fence_proxy_async();     // generic-proxy smem writes -> async-proxy reads
+            uint32_t* dst = a.r.out + t * (long long)L;
+            bulk_s2g(dst, smem + s0 * HALF, half_bytes);
+            bulk_commit();
+            bulk_s2g(dst + HALF, smem + s1 * HALF, half_bytes);
+            bulk_commit();
+            bulk_wait_read1();       // first half read out of slot s0
+            fence_proxy_async();
+            issue_half(2 * i + 3);   // second half of line i+1 -> slot s0
+            bulk_wait_read0();       // second half read out of slot s1
+            fence_proxy_async();
+            issue_half(2 * i + 4);   // first half of line i+2 -> slot s1
+        }
+        if (i < 4) stamp(tr, 4 + 3 * i);
+    }
+    if (tid == 0) bulk_wait0();
+    stamp(tr, 14);
+}
+
 // ------------------------------------------------------------------ row pass, warp-specialized
 
 __device__ __forceinline__ void named_bar(int id, int count) {
@@ -1432,6 +1560,51 @@ __global__ void __launch_bounds__(256) transpose_kernel(const uint32_t* __restri
     for (int j = 0; j < 32; j += 8) out[(bx * 32 + ty + j) * rows + by * 32 + tx] = tile[tx][ty + j];
 }
 
+// 64 x 64 tiles with 128-bit global loads and stores (16 KiB per CTA, 8 CTAs per
+// SM: 128 KiB of loads in flight per SM, what HBM3e needs to stay busy). In
+// shared memory, row r keeps its 16-byte chunks XOR-swizzled: chunk c4 of row r
+// sits at chunk c4 ^ ((r >> 2) & 7). The 128-bit row writes stay conflict-free
+// (a quarter-warp covers 8 distinct chunks of one row) and so do the column
+// reads: lane (il, jl) reads row 4*(8*ih + il) + q, column 4*jh + jl, bank
+// ((jh ^ il) & 7)*4 + jl -- 32 distinct banks, the role Fig. 4's diagonal
+// arrangement plays for the paper's w x w tiles. Each lane gathers four rows of
+// one column into a uint4, so 8 lanes store 128 contiguous bytes of an output row.
+__global__ void __launch_bounds__(256) transpose64_kernel(const uint32_t* __restrict__ in,
+                                                          uint32_t* __restrict__ out, int logr,
+                                                          int logc) {
+    __shared__ __align__(16) uint32_t tile[64 * 64];
+    const long long rows = 1ll << logr, cols = 1ll << logc;
+    const int tid = threadIdx.x;
+    const long long bx = blockIdx.x, by = blockIdx.y;     // column tile, row tile
+    pdl_wait();
+    uint4 v[4];
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+        const int idx = tid + 256 * it, r = idx >> 4, c4 = idx & 15;
+        v[it] = ld_nc_v4(in + (by * 64 + r) * cols + bx * 64 + c4 * 4);
+    }
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+        const int idx = tid + 256 * it, r = idx >> 4, c4 = idx & 15;
+        *reinterpret_cast<uint4*>(tile + r * 64 + ((c4 ^ ((r >> 2) & 7)) << 2)) = v[it];
+    }
+    __syncthreads();
+    pdl_launch_dependents();
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+        const int idx = tid + 256 * it;
+        const int il = idx & 7, jl = (idx >> 3) & 3, ih = (idx >> 5) & 1, jh = idx >> 6;
+        const int i4 = ih * 8 + il, j = jh * 4 + jl;
+        const int col = (jh ^ il) * 4 + jl;   // swizzled word of column j (il < 8)
+        uint4 w;
+        w.x = tile[(4 * i4 + 0) * 64 + col];
+        w.y = tile[(4 * i4 + 1) * 64 + col];
+        w.z = tile[(4 * i4 + 2) * 64 + col];
+        w.w = tile[(4 * i4 + 3) * 64 + col];
+        st_v4(out + (bx * 64 + j) * rows + by * 64 + i4 * 4, w);
+    }
+}
+
 // ------------------------------------------------------------------ comparators
 
 // D-designated (L365): coalesced 128-bit reads of p and a, casual writes of b.
@@ -1560,6 +1733,7 @@ cudaError_t set_smem(K kernel, size_t bytes) {
 size_t tma_smem(const HostPlan& P, int f) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
+    if (rp.split) return (size_t)3 * (g.L / 2) * 4 + 3 * 8;
     const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * (g.L / 32) * g.w64 * 8);
     return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
 }
@@ -1587,7 +1761,8 @@ cudaError_t prep_ws(HostPlan& P, int f) {
 }
 
 template <int EPT>
-const void* tma_kernel_ptr(bool cross, bool sg) {
+const void* tma_kernel_ptr(bool cross, bool sg, bool split = false) {
+    if (split) return (const void*)row_pass_split_kernel<EPT>;
     if (sg) return cross ? (const void*)row_pass_tma_kernel<EPT, true, true>
                          : (const void*)row_pass_tma_kernel<EPT, false, true>;
     return cross ? (const void*)row_pass_tma_kernel<EPT, true> : (const void*)row_pass_tma_kernel<EPT, false>;
@@ -1596,7 +1771,8 @@ const void* tma_kernel_ptr(bool cross, bool sg) {
 template <int EPT>
 cudaError_t set_tma_smem(bool cross, size_t smem) {
     cudaError_t e = set_smem(tma_kernel_ptr<EPT>(cross, false), smem);
-    return e == cudaSuccess ? set_smem(tma_kernel_ptr<EPT>(cross, true), smem) : e;
+    if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true), smem);
+    return e == cudaSuccess ? set_smem(tma_kernel_ptr<EPT>(cross, true, true), smem) : e;
 }
 
 template <int EPT>
@@ -1605,7 +1781,7 @@ cudaError_t grid_tma(HostPlan& P, int f) {
     const size_t smem = tma_smem(P, f);
     int nb = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &nb, tma_kernel_ptr<EPT>(rp.out.cross != 0, rp.sg != 0), rp.threads, smem);
+        &nb, tma_kernel_ptr<EPT>(rp.out.cross != 0, rp.sg != 0, rp.split != 0), rp.threads, smem);
     if (e != cudaSuccess) return e;
     if (nb < 1) return cudaErrorInvalidConfiguration;
     const long long cap = (long long)nb * sm_count();
@@ -1983,6 +2159,16 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const size_t smem = tma_smem(P, f);
         const bool cx = rp.out.cross != 0;
         const bool sg = rp.sg != 0;
+        if (rp.split) {
+            switch (rp.ept) {
+                case 4: return launch(row_pass_split_kernel<4>, grid, block, smem, s, pdl, ta);
+                case 8: return launch(row_pass_split_kernel<8>, grid, block, smem, s, pdl, ta);
+                case 16: return launch(row_pass_split_kernel<16>, grid, block, smem, s, pdl, ta);
+                case 32: return launch(row_pass_split_kernel<32>, grid, block, smem, s, pdl, ta);
+                case 64: return launch(row_pass_split_kernel<64>, grid, block, smem, s, pdl, ta);
+            }
+            return cudaErrorInvalidValue;
+        }
 #define PERM_TMA_CASE(E_)                                                                      \
     case E_:                                                                                   \
         if (sg) return cx ? launch(row_pass_tma_kernel<E_, true, true>, grid, block, smem, s, pdl, ta)  \
@@ -2049,9 +2235,19 @@ cudaError_t launch_fused3(const HostPlan& P, const uint32_t* const sched[3], con
     return cudaErrorInvalidValue;
 }
 
+// 1 when the environment variable is set to something other than "0" (read once)
+static bool getenv_flag(const char* name) {
+    const char* e = std::getenv(name);
+    return e != nullptr && e[0] != '\0' && !(e[0] == '0' && e[1] == '\0');
+}
+
 cudaError_t launch_transpose(const uint32_t* in, uint32_t* out, int64_t rows, int64_t cols,
                              cudaStream_t s, bool pdl) {
     const dim3 grid((unsigned)(cols / 32), (unsigned)(rows / 32)), block(32, 8);
+    static const bool t32 = getenv_flag("PERM_TRANSPOSE32");   // A/B: the 32 x 32 kernel
+    if (rows >= 64 && cols >= 64 && !t32)
+        return launch(transpose64_kernel, dim3((unsigned)(cols / 64), (unsigned)(rows / 64)), dim3(256), 0,
+                      s, pdl, in, out, ilog2i(rows), ilog2i(cols));
     return launch(transpose_kernel, grid, block, 0, s, pdl, in, out, ilog2i(rows), ilog2i(cols));
 }
 

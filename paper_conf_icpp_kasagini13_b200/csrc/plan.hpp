@@ -53,6 +53,7 @@ struct RowPass {
     int32_t tma = 0;          // 1: persistent TMA-pipelined kernel (contiguous input lines)
     int32_t stages = 0;       // TMA ring depth
     int32_t sg = 0;           // 1 (tma == 1): schedule read from global (L2-prefetched), slots hold data only
+    int32_t split = 0;        // 1 (tma == 1, sg, h == 1): ring of three half-line slots (L = 32768)
     int64_t grid = 0;         // persistent CTAs (set at upload from the occupancy query)
     int32_t h = 0;            // lines per CTA (tile)
     int32_t Ls = 0;           // shared-memory line stride (elements) = L + pad
@@ -139,6 +140,7 @@ struct HostPlan {
     std::vector<uint32_t> sched[3];
     double ms_colour = 0, ms_bank = 0;
     int32_t threads_used = 1;
+    int32_t gpu_planner = 0;   // 1: colourings ran on the device (gplan.cu)
 };
 
 // Builds everything host-side. Returns PERM_OK or a perm_status, with `err` set.

@@ -20,6 +20,7 @@
 // cycles, colour each cycle 0,1,0,1,...: every node keeps exactly half its
 // edges on each side. Recurse log2(d) times. O(E log d).
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -31,6 +32,7 @@
 #endif
 
 #include "plan.hpp"
+#include "gplan.hpp"
 
 namespace perm {
 
@@ -553,14 +555,8 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
         const int E = tp.E, ept = tp.ept, nwords = tp.nwords;
         const TlcDecode dec = tp.dec;
         const bool full = dec.lt == tp.logHL && dec.s2 == 0 && dec.s3 == 0 && dec.m1 == 0;
-        int bad = 0;
-#pragma omp parallel reduction(| : bad)
-        {
-            EulerColourer ec;
-            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL),
-                tval((size_t)HL);
-#pragma omp for schedule(dynamic, 1)
-            for (int64_t T = 0; T < tp.ntiles; ++T) {
+        // element x of tile T: source offset in A, destination offset in B, entry payload
+        auto enum_tile = [&](int64_t T, uint32_t* src, uint32_t* dst, uint32_t* tval) {
                 int64_t e = 0;
                 if (f == 0) {
                     for (int64_t i_in = 0; i_in < h; ++i_in)
@@ -587,8 +583,47 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
                             tval[e] = full ? dst[e] : (uint32_t)kp;
                         }
                 }
-                for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
-                ec.run(kW, HL / kW, HL, U.data(), V.data(), col.data(), false);
+        };
+        std::vector<uint16_t> gcol;
+        if (opt && opt->gpu_planner > 0) {
+            // every tile's bank graph at once on the device (vertex (tile, offset mod 32))
+            const int64_t N = tp.ntiles * HL;
+            std::vector<uint16_t> ks((size_t)N), kd((size_t)N);
+#pragma omp parallel
+            {
+                std::vector<uint32_t> src((size_t)HL), dst((size_t)HL), tval((size_t)HL);
+#pragma omp for schedule(static)
+                for (int64_t T = 0; T < tp.ntiles; ++T) {
+                    enum_tile(T, src.data(), dst.data(), tval.data());
+                    for (int64_t x = 0; x < HL; ++x) {
+                        ks[T * HL + x] = (uint16_t)src[x];
+                        kd[T * HL + x] = (uint16_t)dst[x];
+                    }
+                }
+            }
+            gcol.resize((size_t)N);
+            GpuPlanStats gs;
+            const cudaError_t ce = gpu_bank_colour(ks.data(), kd.data(), N, tp.logHL, gcol.data(), &gs);
+            if (ce != cudaSuccess) {
+                err = std::string("GPU planner (TLC bank colouring): ") + cudaGetErrorString(ce);
+                return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
+            }
+        }
+        int bad = 0;
+#pragma omp parallel reduction(| : bad)
+        {
+            EulerColourer ec;
+            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL),
+                tval((size_t)HL);
+#pragma omp for schedule(dynamic, 1)
+            for (int64_t T = 0; T < tp.ntiles; ++T) {
+                enum_tile(T, src.data(), dst.data(), tval.data());
+                if (!gcol.empty()) {
+                    for (int64_t x = 0; x < HL; ++x) col[x] = gcol[T * HL + x];
+                } else {
+                    for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
+                    ec.run(kW, HL / kW, HL, U.data(), V.data(), col.data(), false);
+                }
                 uint32_t* Wt = W + T * tp.tile_words;
                 for (int64_t x = 0; x < HL; ++x) {
                     const int64_t q = col[x];                 // warp-round
@@ -648,8 +683,24 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         err = "n must be a power of two in [2^10, 2^30]";
         return PERM_EUNSUPPORTED;
     }
-    // 1. validate: bijection onto [0, n)
+    // 1. validate: bijection onto [0, n) -- a parallel pass over an atomic bitmap,
+    //    then (only when it fails) the serial pass that names the first bad entry
+    bool valid = true;
     {
+        std::vector<std::atomic<uint64_t>> bits((size_t)((n + 63) / 64));
+#pragma omp parallel for schedule(static)
+        for (int64_t w = 0; w < (int64_t)bits.size(); ++w) bits[w].store(0, std::memory_order_relaxed);
+        int bad = 0;
+#pragma omp parallel for schedule(static) reduction(| : bad)
+        for (int64_t i = 0; i < n; ++i) {
+            const int32_t v = p[i];
+            if (v < 0 || v >= n) { bad = 1; continue; }
+            const uint64_t m = uint64_t(1) << (v & 63);
+            if (bits[v >> 6].fetch_or(m, std::memory_order_relaxed) & m) bad = 1;
+        }
+        valid = !bad;
+    }
+    if (!valid) {
         std::vector<uint8_t> seen((size_t)n, 0);
         for (int64_t i = 0; i < n; ++i) {
             const int32_t v = p[i];
@@ -693,22 +744,31 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 
     // 2-3. row-level colouring
     auto t0 = clk::now();
-    std::vector<uint32_t> colour((size_t)n);
-    {
-        std::vector<uint32_t> U((size_t)n), V((size_t)n);
-#pragma omp parallel for schedule(static)
-        for (int64_t x = 0; x < n; ++x) {
-            U[x] = (uint32_t)(x >> logc);
-            V[x] = (uint32_t)((uint32_t)p[x] >> logc);
-        }
-        EulerColourer ec;
-        ec.run(r, c, n, U.data(), V.data(), colour.data(), true);
-    }
+    const bool gpu = opt && opt->gpu_planner > 0;
+    P.gpu_planner = gpu ? 1 : 0;
     P.kappa.resize((size_t)n);
+    if (gpu) {
+        GpuPlanStats gs;
+        const cudaError_t ce = gpu_row_colour(p, n, logc, P.kappa.data(), &gs);
+        if (ce != cudaSuccess) {
+            err = std::string("GPU planner (row colouring): ") + cudaGetErrorString(ce);
+            return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
+        }
+    } else {
+        std::vector<uint32_t> colour((size_t)n);
+        {
+            std::vector<uint32_t> U((size_t)n), V((size_t)n);
 #pragma omp parallel for schedule(static)
-    for (int64_t x = 0; x < n; ++x) P.kappa[x] = (uint16_t)colour[x];
-    colour.clear();
-    colour.shrink_to_fit();
+            for (int64_t x = 0; x < n; ++x) {
+                U[x] = (uint32_t)(x >> logc);
+                V[x] = (uint32_t)((uint32_t)p[x] >> logc);
+            }
+            EulerColourer ec;
+            ec.run(r, c, n, U.data(), V.data(), colour.data(), true);
+        }
+#pragma omp parallel for schedule(static)
+        for (int64_t x = 0; x < n; ++x) P.kappa[x] = (uint16_t)colour[x];
+    }
     P.ms_colour = ms_since(t0);
 
     // 4. phase permutations as per-line arrays (uint16: every L <= 2^15)
@@ -740,25 +800,42 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.words = g.lines * (g.L / kW) * g.w64 * 2;
     }
     // 5-6. bank-level colouring of every line, packed (W64); not needed by TLC plans
-    auto build_line_schedules = [&]() {
+    auto build_line_schedules = [&]() -> int {
+        std::vector<uint16_t> gcol;
         for (int f = 0; f < 3; ++f) {
             PhaseGeom& g = P.ph[f];
             P.sched[f].assign((size_t)g.words, 0u);
             const int64_t L = g.L;
             const uint16_t* ph = phi[f].data();
             uint32_t* W = P.sched[f].data();
+            if (gpu) {
+                // all lines' bank graphs at once on the device: vertex (line, j mod 32) ->
+                // (line, Phi(j) mod 32), keyU = position j (implicit), keyV = Phi(j)
+                gcol.resize((size_t)n);
+                GpuPlanStats gs;
+                const cudaError_t ce = gpu_bank_colour(nullptr, ph, n, g.logL, gcol.data(), &gs);
+                if (ce != cudaSuccess) {
+                    err = std::string("GPU planner (bank colouring): ") + cudaGetErrorString(ce);
+                    return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
+                }
+            }
 #pragma omp parallel
             {
                 EulerColourer ec;
-                std::vector<uint32_t> U((size_t)L), V((size_t)L), col((size_t)L);
+                std::vector<uint32_t> U((size_t)L), V((size_t)L), colv((size_t)L);
 #pragma omp for schedule(dynamic, 16)
                 for (int64_t line = 0; line < g.lines; ++line) {
                     const uint16_t* phl = ph + line * L;
-                    for (int64_t j = 0; j < L; ++j) {
-                        U[j] = (uint32_t)(j & 31);
-                        V[j] = (uint32_t)(phl[j] & 31);
+                    uint32_t* col = colv.data();
+                    if (gpu) {
+                        for (int64_t j = 0; j < L; ++j) col[j] = gcol[line * L + j];
+                    } else {
+                        for (int64_t j = 0; j < L; ++j) {
+                            U[j] = (uint32_t)(j & 31);
+                            V[j] = (uint32_t)(phl[j] & 31);
+                        }
+                        ec.run(kW, L / kW, L, U.data(), V.data(), col, false);
                     }
-                    ec.run(kW, L / kW, L, U.data(), V.data(), col.data(), false);
                     for (int64_t j = 0; j < L; ++j) {
                         const uint64_t sigma = (uint64_t)(j >> 5);
                         const uint64_t entry = (sigma << g.logL) | phl[j];
@@ -772,6 +849,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 }
             }
         }
+        return PERM_OK;
     };
 
     // pass structure
@@ -787,9 +865,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         P.fused_ept = (int32_t)(n / P.fused_threads);
         P.fused_Ls = (int32_t)(c + 1);   // odd stride: rows AND columns conflict-free (Fig. 4 idea)
         if (r * P.fused_Ls > 65535) { err = "fused tile exceeds 16-bit shared addresses"; return PERM_EUNSUPPORTED; }
-        build_line_schedules();
+        const int bst = build_line_schedules();
         P.ms_bank = ms_since(t0);
-        return PERM_OK;
+        return bst;
     }
     {
         int layout0 = opt ? opt->layout : 0;
@@ -806,7 +884,10 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             return st;
         }
     }
-    build_line_schedules();
+    {
+        const int bst = build_line_schedules();
+        if (bst != PERM_OK) return bst;
+    }
     P.ms_bank = ms_since(t0);
     const int64_t Q = std::min<int64_t>(16384, std::max<int64_t>(2048, pow2_floor(n / 296)));
     auto pick = [&](int idx, int64_t dflt) -> int64_t {
@@ -878,7 +959,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     } else {
         for (int f = 0; f < 3; ++f) {
             const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
-            int64_t h = pick(f, std::max<int64_t>(1, pow2_floor(Q / L)));
+            const bool force_split = opt && opt->no_tma == -2;
+            int64_t h = force_split ? 1 : pick(f, std::max<int64_t>(1, pow2_floor(Q / L)));
             if (h < 1 || h > lines_f || (h & (h - 1))) { err = "invalid h for the 5-pass layout"; return PERM_EINVAL; }
             RowPass& rp = P.rp[f];
             rp.phase = f; rp.h = (int32_t)h; rp.ctas = lines_f / h;
@@ -898,6 +980,11 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 const int64_t fit = kSmemBudget / (h * L * 4);
                 rp.stages = (opt && opt->stages > 0) ? opt->stages : (int)std::min<int64_t>(4, fit);
             }
+            // one line per slot only (L = 32768): ring of three half-line slots instead
+            if (rp.tma && rp.sg && h == 1 && (rp.stages == 1 || force_split) && 3 * (L / 2) * 4 <= kSmemBudget) {
+                rp.split = 1;
+                rp.stages = 3;
+            }
         }
     }
     for (int f = 0; f < 3; ++f) {
@@ -909,6 +996,12 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.threads = 32 + 512 + (rp.out.cross ? 256 : 0);
         } else {
             choose_threads(rp, g.L);
+            // half-line ring: 1024 threads (twice the warps keep twice the schedule loads
+            // in flight; the schedule is read from L2 in both hops)
+            if (rp.split && (int64_t)rp.h * g.L >= 8192) {
+                rp.threads = 1024;
+                rp.ept = (int32_t)((int64_t)rp.h * g.L / 1024);
+            }
         }
         if (rp.tma) {
             // TMA tiles: lines land at 16-byte aligned strides; a CROSS store of h = 8
@@ -925,7 +1018,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 rp.conflicts_out = rp.out.cross ? simulate_conflicts(tmp, g, false) : 1;
             }
             if ((rp.h * (g.L / kW) * g.w64 * 2) % 4) { err = "TMA tile schedule is not 16-byte sized"; return PERM_EINVAL; }
-            const int64_t sb = rp.sg ? (int64_t)rp.h * (g.L + pad) * 4 : stage_bytes(rp.h, rp.phase, pad);
+            const int64_t sb = rp.split ? (int64_t)g.L / 2 * 4
+                               : rp.sg ? (int64_t)rp.h * (g.L + pad) * 4 : stage_bytes(rp.h, rp.phase, pad);
             if (rp.stages * sb > kSmemBudget) {
                 err = "TMA stages exceed the shared-memory budget; lower h or stages";
                 return PERM_EINVAL;

@@ -392,3 +392,22 @@ def test_schedule_from_global(P, fam, k):
         b, info = run(P, p, a, passes=5, no_tma=-1, stages=stages)
         assert info["passes"] == 5
         assert np.array_equal(b, ref), stages
+
+
+@pytest.mark.parametrize("fam,k", [(f, k) for f in ("random", "bitrev", "identity") for k in (16, 20, 22, 24)]
+                         + [("random", 26)])
+def test_half_line_ring(P, fam, k):
+    # 5-pass row passes on the ring of three half-line slots (the default for lines of
+    # 32768 words, n = 2^29..2^30), forced here at small n: one line per CTA, the two
+    # halves of a line in any two slots, loads overlapping the permute and the stores
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=31 + k)
+    a = W.make_data(n)
+    with P.Plan(p, passes=5, no_tma=-2, direct=-1) as plan:
+        d = plan.describe()
+        assert all(rp["split"] == 1 and rp["h"] == 1 for rp in d["row_passes"])
+        da = dev(a)
+        db = torch.full_like(da, -1)
+        plan.apply(da, db)
+        torch.cuda.synchronize()
+        assert np.array_equal(host_words(db), OA.apply_ref(p, a))

@@ -26,7 +26,7 @@ def P():
     return pkg
 
 
-@pytest.mark.parametrize("no_tma", [0, 1])
+@pytest.mark.parametrize("no_tma", [0, 1, -1, -2])
 @pytest.mark.parametrize("G", [1, 2, 4, 8])
 @pytest.mark.parametrize("k", [16, 19, 22])
 def test_virtual_ranks(P, G, k, no_tma):
