@@ -35,6 +35,8 @@
 
 #include <chrono>
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include "gplan.hpp"
@@ -171,6 +173,41 @@ __global__ void k_bank_orders(const uint16_t* __restrict__ keyU, const uint16_t*
     }
 }
 
+using gclk = std::chrono::steady_clock;
+double gms(gclk::time_point t0) { return std::chrono::duration<double, std::milli>(gclk::now() - t0).count(); }
+bool gverbose() {
+    static const bool v = std::getenv("PERM_PLANNER_VERBOSE") != nullptr;
+    return v;
+}
+
+// W64 packing (plan.hpp entry_pos): element e = (line, j) with bank colour col[e]
+// sits at slot q = col*32 + (j mod 32) of its line; entry (sigma << logL) | t
+__global__ void k_w64_entries(const uint16_t* __restrict__ phi, const uint16_t* __restrict__ col,
+                              uint32_t* __restrict__ ent, int64_t n, int logL) {
+    const int64_t Lm = ((int64_t)1 << logL) - 1;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = e & Lm;
+        const int64_t q = (int64_t)col[e] * 32 + (j & 31);
+        ent[(e & ~Lm) + q] = ((uint32_t)(j >> 5) << logL) | phi[e];
+    }
+}
+// 64-bit word w = (line*(L/32) + round)*w64 + wsel holds lanes wsel*epw .. of the round
+__global__ void k_w64_pack(const uint32_t* __restrict__ ent, uint32_t* __restrict__ words, int64_t nw64,
+                           int E, int epw, int w64) {
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nw64; w += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t lr = w / w64;
+        const int wsel = (int)(w - lr * w64);
+        const uint32_t* src = ent + lr * 32;
+        uint64_t v = 0;
+        for (int i = 0; i < epw; ++i) {
+            const int x = wsel * epw + i;
+            if (x < 32) v |= (uint64_t)src[x] << (E * i);
+        }
+        words[2 * w] = (uint32_t)v;
+        words[2 * w + 1] = (uint32_t)(v >> 32);
+    }
+}
+
 struct DevBuf {
     void* p = nullptr;
     ~DevBuf() { if (p) cudaFree(p); }
@@ -196,6 +233,8 @@ unsigned grid_for(int64_t E) {
 cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int logd0, uint16_t* colour,
                                cudaStream_t s, GpuPlanStats* st) {
     const unsigned G = grid_for(E), T = 256;
+    const bool verbose = gverbose();
+    auto ta = gclk::now();
     DevBuf bU2, bV2, bpU, bpV, bg, bseg, bnxt, bslot, bnode, blab, blab2, bnx, bnx2, bcnt, bch;
     const size_t W = (size_t)E * 4;
     GP_TRY(cudaMalloc(&bU2.p, W));
@@ -220,8 +259,14 @@ cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int lo
     uint32_t *nx = (uint32_t*)bnx.p, *nx2 = (uint32_t*)bnx2.p;
     unsigned long long* cnt = (unsigned long long*)bcnt.p;
     int* changed = (int*)bch.p;
+    if (verbose) {
+        cudaStreamSynchronize(s);
+        std::fprintf(stderr, "[gplan] E=%lld logd0=%d alloc %.1f ms\n", (long long)E, logd0, gms(ta));
+    }
     for (int l = 0; l < logd0; ++l) {
         const int logd = logd0 - l;
+        auto tl = gclk::now();
+        int rounds = 0;
         k_pair<<<G, T, 0, s>>>(U, pU, E);
         k_pair<<<G, T, 0, s>>>(V, pV, E);
         k_compose<<<G, T, 0, s>>>(pU, pV, g, E);
@@ -245,6 +290,7 @@ cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int lo
             std::swap(la, lb);
             std::swap(na, nb);
             if (st) st->jump_rounds += 1;
+            ++rounds;
             if (!h || round > 64) break;
         }
         // la = final labels of the reduced nodes; spread to every edge (into lb: free)
@@ -255,6 +301,11 @@ cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int lo
         std::swap(V, V2);
         if (st) { st->levels += 1; st->reduced_nodes += (int64_t)R; }
         GP_TRY(cudaGetLastError());
+        if (verbose) {
+            cudaStreamSynchronize(s);
+            std::fprintf(stderr, "[gplan]  level %d: reduced %llu, %d jump rounds, %.2f ms\n", l,
+                         (unsigned long long)R, rounds, gms(tl));
+        }
     }
     k_final<<<G, T, 0, s>>>(U, colour, E, (uint32_t)((1u << logd0) - 1u));
     GP_TRY(cudaGetLastError());
@@ -265,6 +316,7 @@ cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int lo
 
 cudaError_t gpu_row_colour(const int32_t* p_host, int64_t n, int logc, uint16_t* kappa_host,
                            GpuPlanStats* st) {
+    auto t0 = gclk::now();
     cudaStream_t s = nullptr;
     GP_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
@@ -278,15 +330,23 @@ cudaError_t gpu_row_colour(const int32_t* p_host, int64_t n, int logc, uint16_t*
     GP_TRY(cudaGetLastError());
     cudaFree(bp.p);
     bp.p = nullptr;
+    if (gverbose()) {
+        cudaStreamSynchronize(s);
+        std::fprintf(stderr, "[gplan] row colour: alloc + upload p + orders %.1f ms\n", gms(t0));
+    }
     GP_TRY(euler_split_device((uint32_t*)bU.p, (uint32_t*)bV.p, n, logc, (uint16_t*)bc.p, s, st));
+    auto t1 = gclk::now();
     GP_TRY(cudaMemcpyAsync(kappa_host, bc.p, (size_t)n * 2, cudaMemcpyDeviceToHost, s));
-    return cudaStreamSynchronize(s);
+    const cudaError_t e = cudaStreamSynchronize(s);
+    if (gverbose()) std::fprintf(stderr, "[gplan] row colour: download %.1f ms, total %.1f ms\n", gms(t1), gms(t0));
+    return e;
 }
 
 cudaError_t gpu_bank_colour(const uint16_t* keyU_host, const uint16_t* keyV_host, int64_t E, int logB,
                             uint16_t* col_host, GpuPlanStats* st) {
     // B = 32 (a 32-element line): degree 1, every edge gets colour 0 (no split level)
     if (logB < 5 || logB > 16 || (E & ((int64_t(1) << logB) - 1))) return cudaErrorInvalidValue;
+    auto t0 = gclk::now();
     cudaStream_t s = nullptr;
     GP_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
@@ -301,9 +361,51 @@ cudaError_t gpu_bank_colour(const uint16_t* keyU_host, const uint16_t* keyV_host
     k_bank_orders<<<grid_for(E), 256, 0, s>>>((const uint16_t*)bku.p, (const uint16_t*)bkv.p,
                                               (uint32_t*)bU.p, (uint32_t*)bV.p, E, logB);
     GP_TRY(cudaGetLastError());
+    if (gverbose()) {
+        cudaStreamSynchronize(s);
+        std::fprintf(stderr, "[gplan] bank colour: alloc + upload keys + orders %.1f ms\n", gms(t0));
+    }
     GP_TRY(euler_split_device((uint32_t*)bU.p, (uint32_t*)bV.p, E, logB - 5, (uint16_t*)bc.p, s, st));
+    auto t1 = gclk::now();
     GP_TRY(cudaMemcpyAsync(col_host, bc.p, (size_t)E * 2, cudaMemcpyDeviceToHost, s));
-    return cudaStreamSynchronize(s);
+    const cudaError_t e = cudaStreamSynchronize(s);
+    if (gverbose()) std::fprintf(stderr, "[gplan] bank colour: download %.1f ms, total %.1f ms\n", gms(t1), gms(t0));
+    return e;
+}
+
+}  // namespace perm
+
+namespace perm {
+
+cudaError_t gpu_line_schedules(const uint16_t* phi_host, int64_t n, int logL, int E, int epw, int w64,
+                               uint32_t* words_host, GpuPlanStats* st) {
+    if (logL < 5 || logL > 16 || (n & ((int64_t(1) << logL) - 1))) return cudaErrorInvalidValue;
+    auto t0 = gclk::now();
+    cudaStream_t s = nullptr;
+    GP_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+    DevBuf bph, bU, bV, bc;
+    GP_TRY(cudaMalloc(&bph.p, (size_t)n * 2));
+    GP_TRY(cudaMalloc(&bU.p, (size_t)n * 4));
+    GP_TRY(cudaMalloc(&bV.p, (size_t)n * 4));
+    GP_TRY(cudaMalloc(&bc.p, (size_t)n * 2));
+    GP_TRY(cudaMemcpyAsync(bph.p, phi_host, (size_t)n * 2, cudaMemcpyHostToDevice, s));
+    k_bank_orders<<<grid_for(n), 256, 0, s>>>(nullptr, (const uint16_t*)bph.p, (uint32_t*)bU.p, (uint32_t*)bV.p,
+                                              n, logL);
+    GP_TRY(cudaGetLastError());
+    GP_TRY(euler_split_device((uint32_t*)bU.p, (uint32_t*)bV.p, n, logL - 5, (uint16_t*)bc.p, s, st));
+    // ordU / ordV are free now: entries into U, packed words into V (W64 words <= n)
+    const int64_t nw64 = (n / 32) * w64;
+    k_w64_entries<<<grid_for(n), 256, 0, s>>>((const uint16_t*)bph.p, (const uint16_t*)bc.p, (uint32_t*)bU.p, n,
+                                              logL);
+    k_w64_pack<<<grid_for(nw64), 256, 0, s>>>((const uint32_t*)bU.p, (uint32_t*)bV.p, nw64, E, epw, w64);
+    GP_TRY(cudaGetLastError());
+    auto t1 = gclk::now();
+    GP_TRY(cudaMemcpyAsync(words_host, bV.p, (size_t)nw64 * 8, cudaMemcpyDeviceToHost, s));
+    const cudaError_t e = cudaStreamSynchronize(s);
+    if (gverbose())
+        std::fprintf(stderr, "[gplan] line schedules: download %.1f ms, total %.1f ms\n", gms(t1), gms(t0));
+    return e;
 }
 
 }  // namespace perm

@@ -26,4 +26,10 @@ cudaError_t gpu_row_colour(const int32_t* p_host, int64_t n, int logc, uint16_t*
 cudaError_t gpu_bank_colour(const uint16_t* keyU_host, const uint16_t* keyV_host, int64_t E, int logB,
                             uint16_t* col_host, GpuPlanStats* st);
 
+// Bank colouring + W64 packing of one phase's per-line schedules (plan.hpp
+// entry_pos) on the device: phi = Phi per element in line order (n entries,
+// lines of 2^logL); words: host array of (n/32)*w64*2 u32.
+cudaError_t gpu_line_schedules(const uint16_t* phi_host, int64_t n, int logL, int E, int epw, int w64,
+                               uint32_t* words_host, GpuPlanStats* st);
+
 }  // namespace perm

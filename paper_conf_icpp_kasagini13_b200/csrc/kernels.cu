@@ -523,7 +523,10 @@ __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1,
     const uint32_t tmask = (1u << logL) - 1u;
     const uint2* sp = reinterpret_cast<const uint2*>(sched) + warp * w64 + wsel;
     const int step = W * w64;
+    // the schedule is read once: the destination word offsets (< 3 * 2^14 < 2^16) wait
+    // in registers, two per register, across the barrier
     uint32_t v[EPT];
+    uint32_t ta[(EPT + 1) / 2];
 #pragma unroll
     for (int m = 0; m < EPT; ++m) {
         const uint2 wd = __ldg(sp + m * step);
@@ -531,15 +534,14 @@ __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1,
         const uint32_t e = (uint32_t)(w >> sh) & mask;
         const int s = (int)((e >> logL) << 5) + lane;
         v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
+        const int t = (int)(e & tmask);
+        const uint32_t ad = (uint32_t)(((t >> lh) ? o1 : o0) + (t & hmask));
+        if (m & 1) ta[m >> 1] |= ad << 16;
+        else ta[m >> 1] = ad;
     }
     __syncthreads();
 #pragma unroll
-    for (int m = 0; m < EPT; ++m) {
-        const uint2 wd = __ldg(sp + m * step);
-        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
-        const int t = (int)(((uint32_t)(w >> sh) & mask) & tmask);
-        sm[((t >> lh) ? o1 : o0) + (t & hmask)] = v[m];
-    }
+    for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
     __syncthreads();
 }
 
@@ -555,7 +557,7 @@ __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1,
 // the mbarrier parity every thread waits on is (j div 3) & 1. Schedule: W64,
 // read from global, L2-prefetched one line ahead. Row-major output only.
 template <int EPT>
-__global__ void __launch_bounds__(1024, 1) row_pass_split_kernel(const TmaArgs a) {
+__global__ void __launch_bounds__(512, 1) row_pass_split_kernel(const TmaArgs a) {
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x;
     const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1;

@@ -801,23 +801,25 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     }
     // 5-6. bank-level colouring of every line, packed (W64); not needed by TLC plans
     auto build_line_schedules = [&]() -> int {
-        std::vector<uint16_t> gcol;
         for (int f = 0; f < 3; ++f) {
             PhaseGeom& g = P.ph[f];
             P.sched[f].assign((size_t)g.words, 0u);
             const int64_t L = g.L;
             const uint16_t* ph = phi[f].data();
             uint32_t* W = P.sched[f].data();
+            auto tph = clk::now();
             if (gpu) {
-                // all lines' bank graphs at once on the device: vertex (line, j mod 32) ->
-                // (line, Phi(j) mod 32), keyU = position j (implicit), keyV = Phi(j)
-                gcol.resize((size_t)n);
+                // all lines' bank graphs at once on the device (vertex (line, j mod 32) ->
+                // (line, Phi(j) mod 32)), colour + W64 packing there
                 GpuPlanStats gs;
-                const cudaError_t ce = gpu_bank_colour(nullptr, ph, n, g.logL, gcol.data(), &gs);
+                const cudaError_t ce = gpu_line_schedules(ph, n, g.logL, g.E, g.epw, g.w64, W, &gs);
                 if (ce != cudaSuccess) {
                     err = std::string("GPU planner (bank colouring): ") + cudaGetErrorString(ce);
                     return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
                 }
+                if (std::getenv("PERM_PLANNER_VERBOSE"))
+                    std::fprintf(stderr, "[planner] phase %d line schedules (GPU) %.1f ms\n", f, ms_since(tph));
+                continue;
             }
 #pragma omp parallel
             {
@@ -827,15 +829,11 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 for (int64_t line = 0; line < g.lines; ++line) {
                     const uint16_t* phl = ph + line * L;
                     uint32_t* col = colv.data();
-                    if (gpu) {
-                        for (int64_t j = 0; j < L; ++j) col[j] = gcol[line * L + j];
-                    } else {
-                        for (int64_t j = 0; j < L; ++j) {
-                            U[j] = (uint32_t)(j & 31);
-                            V[j] = (uint32_t)(phl[j] & 31);
-                        }
-                        ec.run(kW, L / kW, L, U.data(), V.data(), col, false);
+                    for (int64_t j = 0; j < L; ++j) {
+                        U[j] = (uint32_t)(j & 31);
+                        V[j] = (uint32_t)(phl[j] & 31);
                     }
+                    ec.run(kW, L / kW, L, U.data(), V.data(), col, false);
                     for (int64_t j = 0; j < L; ++j) {
                         const uint64_t sigma = (uint64_t)(j >> 5);
                         const uint64_t entry = (sigma << g.logL) | phl[j];
@@ -848,6 +846,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                     }
                 }
             }
+            if (std::getenv("PERM_PLANNER_VERBOSE"))
+                std::fprintf(stderr, "[planner] phase %d line schedules (colour + pack) %.1f ms\n", f, ms_since(tph));
         }
         return PERM_OK;
     };
@@ -996,12 +996,6 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.threads = 32 + 512 + (rp.out.cross ? 256 : 0);
         } else {
             choose_threads(rp, g.L);
-            // half-line ring: 1024 threads (twice the warps keep twice the schedule loads
-            // in flight; the schedule is read from L2 in both hops)
-            if (rp.split && (int64_t)rp.h * g.L >= 8192) {
-                rp.threads = 1024;
-                rp.ept = (int32_t)((int64_t)rp.h * g.L / 1024);
-            }
         }
         if (rp.tma) {
             // TMA tiles: lines land at 16-byte aligned strides; a CROSS store of h = 8

@@ -2,10 +2,11 @@ import sys, numpy as np, torch
 sys.path.insert(0, '.')
 import workloads as W
 import paper_conf_icpp_kasagini13_b200 as P
-from oracle import apply as OA
+sys.path.insert(0, 'scripts')
+from nphelp import scatter_np, inverse_np
 for k in (18, 20, 22):
     n = 1 << k
-    p = W.random(n, k); a = W.make_data(n); ref = OA.apply_ref(p, a)
+    p = W.random(n, k); a = W.make_data(n); ref = scatter_np(p, a)
     for cfg in ({'layout': 2, 'h': (8, 8, 8), 'stages': 2, 'fuse': 1}, {'fuse': -1}, {}, {'layout': 3, 'stages': 1}, {'layout': 3, 'stages': 1, 'fuse': -1}):
         pl = P.Plan(p, **cfg)
         d = pl.describe()

@@ -4,13 +4,14 @@ import numpy as np, torch
 sys.path.insert(0, '.')
 import workloads as W
 import paper_conf_icpp_kasagini13_b200 as P
-from oracle import apply as OA
+sys.path.insert(0, 'scripts')
+from nphelp import scatter_np, inverse_np
 cfgs = json.loads(sys.argv[1])
 for c in cfgs:
     k = c.pop("k"); n = 1 << k
     if "h" in c: c["h"] = tuple(c["h"])
     p = W.make_perm(c.pop("fam", "random"), n)
-    a = W.make_data(n); ref = OA.apply_ref(p, a)
+    a = W.make_data(n); ref = scatter_np(p, a)
     try:
         pl = P.Plan(p, passes=3, layout=3, **c)
     except Exception as e:

@@ -5,7 +5,8 @@ import numpy as np, torch
 sys.path.insert(0, '.')
 import workloads as W
 import paper_conf_icpp_kasagini13_b200 as P
-from oracle import apply as OA
+sys.path.insert(0, 'scripts')
+from nphelp import scatter_np, inverse_np
 ap = argparse.ArgumentParser()
 ap.add_argument('--k', default='22,24,25,26')
 ap.add_argument('--families', default='random')
@@ -32,7 +33,7 @@ for k in [int(x) for x in a.k.split(',')]:
         dp = torch.from_numpy(p).cuda()
         conv = timeit(lambda: P.scatter_baseline(dp, da, db), reps)
         del dp
-        ref = OA.apply_ref(p, ha) if a.check else None
+        ref = scatter_np(p, ha) if a.check else None
         for cfg in json.loads(a.configs):
             kw = dict(cfg)
             if 'h' in kw: kw['h'] = tuple(kw['h'])

@@ -4,7 +4,8 @@ import numpy as np, torch
 sys.path.insert(0, '.')
 import workloads as W
 import paper_conf_icpp_kasagini13_b200 as P
-from oracle import apply as OA
+sys.path.insert(0, 'scripts')
+from nphelp import scatter_np, inverse_np
 ap = argparse.ArgumentParser()
 ap.add_argument('--log2n', type=int, default=22)
 ap.add_argument('--family', default='random')
@@ -18,7 +19,7 @@ p = W.make_perm(a.family, n)
 host_a = W.make_data(n)
 da = torch.from_numpy(host_a.view(np.int32)).cuda(); db = torch.empty_like(da)
 flush = torch.empty(64 << 20, dtype=torch.int32, device='cuda')
-ref = OA.apply_ref(p, host_a) if a.check else None
+ref = scatter_np(p, host_a) if a.check else None
 def timeit(fn):
     ts = []
     for i in range(a.reps + 3):

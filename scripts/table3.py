@@ -7,8 +7,8 @@ import numpy as np, torch
 sys.path.insert(0, '.')
 import workloads as W
 import paper_conf_icpp_kasagini13_b200 as P
-from oracle import apply as OA
-from oracle import distribution as OD
+sys.path.insert(0, 'scripts')
+from nphelp import scatter_np, inverse_np
 ap = argparse.ArgumentParser()
 ap.add_argument('--log2n', type=int, default=22)
 ap.add_argument('--perms', type=int, default=32)
@@ -29,14 +29,15 @@ def timeit(fn):
 rows = {'D-designated': [], 'S-designated': [], 'scheduled': [], 'D_w/n': []}
 for s in range(a.perms):
     p = W.random(n, 42 + s)
-    dp = torch.from_numpy(p).cuda(); dq = torch.from_numpy(OA.inverse(p)).cuda()
+    dp = torch.from_numpy(p).cuda(); dq = torch.from_numpy(inverse_np(p)).cuda()
     rows['D-designated'].append(timeit(lambda: P.scatter_baseline(dp, da, db)))
     rows['S-designated'].append(timeit(lambda: P.gather_baseline(dq, da, db)))
     with P.Plan(p) as plan:
+        dw = plan.info()['distribution']          # D_w(P), the planner's count (L389-L401)
         rows['scheduled'].append(timeit(lambda: plan.apply(da, db)))
         if s == 0:
-            ok = bool(np.array_equal(db.cpu().numpy().view(np.uint32), OA.apply_ref(p, ha)))
-    rows['D_w/n'].append(OD.distribution(p, 32) / n)
+            ok = bool(np.array_equal(db.cpu().numpy().view(np.uint32), scatter_np(p, ha)))
+    rows['D_w/n'].append(dw / n)
 out = {k: {'min': min(v), 'avg': statistics.mean(v), 'max': max(v)} for k, v in rows.items()}
 out['n'] = n; out['perms'] = a.perms; out['unit'] = 'us (D_w/n: ratio)'; out['bitexact_first'] = ok
 print(json.dumps(out))

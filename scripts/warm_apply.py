@@ -3,14 +3,15 @@ import sys, statistics, json
 import numpy as np, torch
 sys.path.insert(0, '.')
 import workloads as W
-from oracle import apply as OA
+sys.path.insert(0, 'scripts')
+from nphelp import scatter_np, inverse_np
 import paper_conf_icpp_kasagini13_b200 as P
 flush = torch.empty(64 << 20, dtype=torch.int32, device='cuda')
 for k in [int(x) for x in (sys.argv[1] if len(sys.argv) > 1 else "22").split(",")]:
     n = 1 << k
     p = W.make_perm("random", n)
     a_host = W.make_data(n)
-    ref = OA.apply_ref(p, a_host)
+    ref = scatter_np(p, a_host)
     cfgs = json.loads(sys.argv[2]) if len(sys.argv) > 2 else [{}, {"fuse": 1}]
     for cfg in cfgs:
         kw = dict(cfg)
