@@ -289,7 +289,12 @@ def sched_bytes_per_elt(info: dict, desc: dict) -> list:
     if desc.get("layout") == 3:
         # TLC format: each lane's ept entries are one bitstream of nwords 32-bit words
         return [4 * t["nwords"] / t["ept"] for t in desc["tlc"]]
-    # W64 format: floor(64/E) entries per 64-bit word, ceil(32/epw) words per warp-round
+    # per-line formats: u32 words per line / line length (W64: floor(64/E) entries per
+    # 64-bit word; dense: one E-bit entry per element)
+    rps = desc.get("row_passes")
+    if rps:
+        by_phase = {rp["phase"]: 4 * rp["sched_words_per_line"] / rp["L"] for rp in rps}
+        return [by_phase[f] for f in range(3)]
     return [8 * (-(-32 // (64 // e))) / 32 for e in info["entry_bits"]]
 
 

@@ -308,7 +308,9 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
                  ",\"tma\":" + std::to_string(rp.tma) + ",\"sg\":" + std::to_string(rp.sg) + ",\"split\":" + std::to_string(rp.split) + ",\"stages\":" + std::to_string(rp.stages) +
                  ",\"grid\":" + std::to_string(rp.grid) +
                  ",\"L\":" + std::to_string(P.ph[rp.phase].L) + ",\"E\":" +
-                 std::to_string(P.ph[rp.phase].E) + ",\"h\":" + std::to_string(rp.h) +
+                 std::to_string(P.ph[rp.phase].E) + ",\"dense\":" + std::to_string(P.ph[rp.phase].dense) +
+                 ",\"sched_words_per_line\":" + std::to_string(P.ph[rp.phase].wpl) +
+                 ",\"h\":" + std::to_string(rp.h) +
                  ",\"ctas\":" + std::to_string(rp.ctas) + ",\"threads\":" +
                  std::to_string(rp.threads) + ",\"ept\":" + std::to_string(rp.ept) +
                  ",\"Ls\":" + std::to_string(rp.Ls) + ",\"smem_bytes\":" +

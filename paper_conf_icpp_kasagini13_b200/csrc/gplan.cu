@@ -208,6 +208,24 @@ __global__ void k_w64_pack(const uint32_t* __restrict__ ent, uint32_t* __restric
     }
 }
 
+// dense format: round lr = E u32 words, lane x's entry at bit x*E; thread per word
+__global__ void k_dense_pack(const uint32_t* __restrict__ ent, uint32_t* __restrict__ words, int64_t nwords,
+                             int E) {
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nwords; w += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t lr = w / E;
+        const int wi = (int)(w - lr * E);
+        const uint32_t* src = ent + lr * 32;
+        const int x0 = (32 * wi) / E, x1 = min(31, (32 * wi + 31) / E);
+        uint32_t v = 0;
+        for (int x = x0; x <= x1; ++x) {
+            const int pos = x * E - 32 * wi;
+            const uint64_t e = src[x];
+            v |= pos >= 0 ? (uint32_t)(e << pos) : (uint32_t)(e >> -pos);
+        }
+        words[w] = v;
+    }
+}
+
 struct DevBuf {
     void* p = nullptr;
     ~DevBuf() { if (p) cudaFree(p); }
@@ -378,7 +396,7 @@ cudaError_t gpu_bank_colour(const uint16_t* keyU_host, const uint16_t* keyV_host
 namespace perm {
 
 cudaError_t gpu_line_schedules(const uint16_t* phi_host, int64_t n, int logL, int E, int epw, int w64,
-                               uint32_t* words_host, GpuPlanStats* st) {
+                               int dense, uint32_t* words_host, GpuPlanStats* st) {
     if (logL < 5 || logL > 16 || (n & ((int64_t(1) << logL) - 1))) return cudaErrorInvalidValue;
     auto t0 = gclk::now();
     cudaStream_t s = nullptr;
@@ -396,12 +414,16 @@ cudaError_t gpu_line_schedules(const uint16_t* phi_host, int64_t n, int logL, in
     GP_TRY(euler_split_device((uint32_t*)bU.p, (uint32_t*)bV.p, n, logL - 5, (uint16_t*)bc.p, s, st));
     // ordU / ordV are free now: entries into U, packed words into V (W64 words <= n)
     const int64_t nw64 = (n / 32) * w64;
+    const int64_t nw32 = dense ? (n / 32) * E : 2 * nw64;     // <= n u32 either way
     k_w64_entries<<<grid_for(n), 256, 0, s>>>((const uint16_t*)bph.p, (const uint16_t*)bc.p, (uint32_t*)bU.p, n,
                                               logL);
-    k_w64_pack<<<grid_for(nw64), 256, 0, s>>>((const uint32_t*)bU.p, (uint32_t*)bV.p, nw64, E, epw, w64);
+    if (dense)
+        k_dense_pack<<<grid_for(nw32), 256, 0, s>>>((const uint32_t*)bU.p, (uint32_t*)bV.p, nw32, E);
+    else
+        k_w64_pack<<<grid_for(nw64), 256, 0, s>>>((const uint32_t*)bU.p, (uint32_t*)bV.p, nw64, E, epw, w64);
     GP_TRY(cudaGetLastError());
     auto t1 = gclk::now();
-    GP_TRY(cudaMemcpyAsync(words_host, bV.p, (size_t)nw64 * 8, cudaMemcpyDeviceToHost, s));
+    GP_TRY(cudaMemcpyAsync(words_host, bV.p, (size_t)nw32 * 4, cudaMemcpyDeviceToHost, s));
     const cudaError_t e = cudaStreamSynchronize(s);
     if (gverbose())
         std::fprintf(stderr, "[gplan] line schedules: download %.1f ms, total %.1f ms\n", gms(t1), gms(t0));

@@ -27,9 +27,9 @@ cudaError_t gpu_bank_colour(const uint16_t* keyU_host, const uint16_t* keyV_host
                             uint16_t* col_host, GpuPlanStats* st);
 
 // Bank colouring + W64 packing of one phase's per-line schedules (plan.hpp
-// entry_pos) on the device: phi = Phi per element in line order (n entries,
-// lines of 2^logL); words: host array of (n/32)*w64*2 u32.
+// entry_pos32: W64 or dense) on the device: phi = Phi per element in line order (n
+// entries, lines of 2^logL); words: host array of (n/32)*(dense ? E : 2*w64) u32.
 cudaError_t gpu_line_schedules(const uint16_t* phi_host, int64_t n, int logL, int E, int epw, int w64,
-                               uint32_t* words_host, GpuPlanStats* st);
+                               int dense, uint32_t* words_host, GpuPlanStats* st);
 
 }  // namespace perm

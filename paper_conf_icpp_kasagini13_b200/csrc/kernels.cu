@@ -125,6 +125,40 @@ __device__ __forceinline__ uint2 sched_load64(const uint2* p) {
     if constexpr (SMEM) return *p;
     else return __ldg(p);
 }
+template <bool SMEM>
+__device__ __forceinline__ uint32_t sched_load32(const uint32_t* p) {
+    if constexpr (SMEM) return *p;
+    else return __ldg(p);
+}
+
+// Entry of warp-round q for this lane, W64 or dense format (plan.hpp PhaseGeom).
+// W64: 64-bit word q*w64 + lane/epw, shift E*(lane % epw). Dense: round q = E
+// u32 words, lane's entry at bit lane*E (two loads + funnel shift; the second
+// load repeats the first when the entry does not straddle).
+struct SchedDec {
+    int dense, E, w64, wsel, sh, dwo, dwo2, dbo;
+    uint32_t mask;
+    __device__ __forceinline__ SchedDec(int dense_, int E_, int epw, int w64_, int lane)
+        : dense(dense_), E(E_), w64(w64_) {
+        wsel = lane / epw;
+        sh = E * (lane - wsel * epw);
+        const int bit = lane * E;
+        dwo = bit >> 5;
+        dbo = bit & 31;
+        dwo2 = dwo + ((dbo + E > 32) ? 1 : 0);
+        mask = (1u << E) - 1u;
+    }
+    template <bool SMEM>
+    __device__ __forceinline__ uint32_t get(const uint32_t* sched, int q) const {
+        if (dense) {
+            const uint32_t* p = sched + q * E;
+            const uint32_t lo = sched_load32<SMEM>(p + dwo), hi = sched_load32<SMEM>(p + dwo2);
+            return (uint32_t)((((uint64_t)hi << 32) | lo) >> dbo) & mask;
+        }
+        const uint2 wd = sched_load64<SMEM>(reinterpret_cast<const uint2*>(sched) + q * w64 + wsel);
+        return (uint32_t)((((uint64_t)wd.y << 32) | wd.x) >> sh) & mask;
+    }
+};
 
 // In-place permutation of the lines resident in shared memory. Warp-round q
 // (0 <= q < h*L/32) of this CTA is line q >> (logL-5), round q & (L/32 - 1);
@@ -136,15 +170,11 @@ __device__ __forceinline__ uint2 sched_load64(const uint2* p) {
 // per register) for the write hop, so the schedule is read once.
 template <int EPT, bool COLS, bool SCHED_SMEM = false>
 __device__ __forceinline__ void permute_lines(uint32_t* sm, const uint32_t* __restrict__ sched,
-                                              int logL, int E, int epw, int w64, int Ls) {
+                                              int logL, int E, int epw, int w64, int Ls, int dense = 0) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, W = blockDim.x >> 5;
     const int logR = logL - 5;                      // log2(rounds per line)
-    const int wsel = lane / epw;
-    const int sh = E * (lane - wsel * epw);
-    const uint32_t mask = (1u << E) - 1u;
+    const SchedDec dec(dense, E, epw, w64, lane);
     const uint32_t tmask = (1u << logL) - 1u;
-    const uint2* sp = reinterpret_cast<const uint2*>(sched) + warp * w64 + wsel;
-    const int step = W * w64;
     // Up to 32 elements per thread the decoded destinations stay in registers
     // (two 16-bit addresses per register); beyond that they are re-decoded in
     // the write hop to stay within 128 registers.
@@ -154,9 +184,7 @@ __device__ __forceinline__ void permute_lines(uint32_t* sm, const uint32_t* __re
     // read hop: v[m] = line[32*sigma + lane]   (bank = lane + const: conflict-free)
 #pragma unroll
     for (int m = 0; m < EPT; ++m) {
-        const uint2 wd = sched_load64<SCHED_SMEM>(sp + m * step);
-        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
-        const uint32_t e = (uint32_t)(w >> sh) & mask;
+        const uint32_t e = dec.get<SCHED_SMEM>(sched, warp + W * m);
         const int l = (warp + W * m) >> logR;
         const int s = (int)((e >> logL) << 5) + lane;
         v[m] = COLS ? sm[s * Ls + l] : sm[l * Ls + s];
@@ -174,12 +202,9 @@ __device__ __forceinline__ void permute_lines(uint32_t* sm, const uint32_t* __re
         for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
     } else {
         const int warp2 = __shfl_sync(kFull, warp, 0);   // not CSE-able: re-derive addresses
-        const uint2* sp2 = reinterpret_cast<const uint2*>(sched) + warp2 * w64 + wsel;
 #pragma unroll
         for (int m = 0; m < EPT; ++m) {
-            const uint2 wd = sched_load64<SCHED_SMEM>(sp2 + m * step);
-            const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
-            const uint32_t e = (uint32_t)(w >> sh) & mask;
+            const uint32_t e = dec.get<SCHED_SMEM>(sched, warp2 + W * m);
             const int l = (warp2 + W * m) >> logR;
             const int t = (int)(e & tmask);
             if (COLS) sm[t * Ls + l] = v[m];
@@ -232,7 +257,7 @@ struct RowArgs {
     const uint32_t* in;
     uint32_t* out;
     const uint32_t* sched;     // this pass's packed phase
-    int logL, logh, Ls, E, epw, w64;
+    int logL, logh, Ls, E, epw, w64, dense;
     long long sched_words_per_cta;
     Io i, o;
     unsigned long long* trace;   // optional: 16 %globaltimer stamps per CTA (tracing)
@@ -365,7 +390,7 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_kernel(cons
     __syncthreads();
     stamp(a.trace, 2);
     pdl_launch_dependents();
-    permute_lines<EPT, false>(sm, sched, a.logL, a.E, a.epw, a.w64, a.Ls);
+    permute_lines<EPT, false>(sm, sched, a.logL, a.E, a.epw, a.w64, a.Ls, a.dense);
     stamp(a.trace, 3);
     tile_store<EPT>(a, sm, cta);
     stamp(a.trace, 14);
@@ -466,10 +491,10 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
         uint32_t* buf = smem + s * stage_words;
         if constexpr (SG)
             permute_lines<EPT, false, false>(buf, a.r.sched + t * a.sched_words, a.r.logL, a.r.E,
-                                             a.r.epw, a.r.w64, a.r.Ls);
+                                             a.r.epw, a.r.w64, a.r.Ls, a.r.dense);
         else
             permute_lines<EPT, false, true>(buf, buf + a.data_words, a.r.logL, a.r.E, a.r.epw,
-                                            a.r.w64, a.r.Ls);
+                                            a.r.w64, a.r.Ls, a.r.dense);
         if (i < 4) stamp(tr, 3 + 3 * i);
         if constexpr (OUT_CROSS) {
             tile_store<EPT>(a.r, buf, t);
@@ -513,25 +538,19 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
 // and the rounds stay conflict-free.
 template <int EPT>
 __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1, const uint32_t* __restrict__ sched,
-                                                   int logL, int E, int epw, int w64) {
+                                                   int logL, int E, int epw, int w64, int dense) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, W = blockDim.x >> 5;
     const int lh = logL - 1;
     const int hmask = (1 << lh) - 1;
-    const int wsel = lane / epw;
-    const int sh = E * (lane - wsel * epw);
-    const uint32_t mask = (1u << E) - 1u;
+    const SchedDec dec(dense, E, epw, w64, lane);
     const uint32_t tmask = (1u << logL) - 1u;
-    const uint2* sp = reinterpret_cast<const uint2*>(sched) + warp * w64 + wsel;
-    const int step = W * w64;
     // the schedule is read once: the destination word offsets (< 3 * 2^14 < 2^16) wait
     // in registers, two per register, across the barrier
     uint32_t v[EPT];
     uint32_t ta[(EPT + 1) / 2];
 #pragma unroll
     for (int m = 0; m < EPT; ++m) {
-        const uint2 wd = __ldg(sp + m * step);
-        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
-        const uint32_t e = (uint32_t)(w >> sh) & mask;
+        const uint32_t e = dec.get<false>(sched, warp + W * m);
         const int s = (int)((e >> logL) << 5) + lane;
         v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
         const int t = (int)(e & tmask);
@@ -612,7 +631,7 @@ __global__ void __launch_bounds__(512, 1) row_pass_split_kernel(const TmaArgs a)
         mbar_wait(&bars[s1], (uint32_t)(j1 / 3) & 1u);
         if (i < 4) stamp(tr, 2 + 3 * i);
         permute_split_line<EPT>(smem, s0 * HALF, s1 * HALF, a.r.sched + t * a.sched_words, a.r.logL, a.r.E,
-                                a.r.epw, a.r.w64);
+                                a.r.epw, a.r.w64, a.r.dense);
         if (i < 4) stamp(tr, 3 + 3 * i);
         if (tid == 0) {
             fence_proxy_async();     // generic-proxy smem writes -> async-proxy reads
@@ -1736,7 +1755,7 @@ size_t tma_smem(const HostPlan& P, int f) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
     if (rp.split) return (size_t)3 * (g.L / 2) * 4 + 3 * 8;
-    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * (g.L / 32) * g.w64 * 8);
+    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * g.wpl * 4);
     return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
 }
 
@@ -2120,7 +2139,8 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
     ra.E = g.E;
     ra.epw = g.epw;
     ra.w64 = g.w64;
-    ra.sched_words_per_cta = (long long)rp.h * (g.L / 32) * g.w64 * 2;
+    ra.dense = g.dense;
+    ra.sched_words_per_cta = (long long)rp.h * g.wpl;
     ra.i = make_io(rp.in);
     ra.o = make_io(rp.out);
     ra.in_segs = rp.in_segs;

@@ -30,7 +30,12 @@ struct PhaseGeom {
     int32_t E = 0;        // entry bits = logL + (logL - 5)
     int32_t epw = 0;      // entries per 64-bit word
     int32_t w64 = 0;      // 64-bit words per warp-round
-    int64_t words = 0;    // 32-bit words: lines * (L/32) * w64 * 2
+    int64_t words = 0;    // 32-bit words: lines * wpl
+    // "dense" format (5-pass phases with L >= 16384, where W64 wastes 18-28 of 64
+    // bits): warp-round k's 32 entries are one bitstream of E u32 words, lane x's
+    // entry at bit x*E (two 32-bit loads + a funnel shift decode it)
+    int32_t dense = 0;
+    int64_t wpl = 0;      // 32-bit words per line: (L/32) * (dense ? E : 2*w64)
 };
 
 // Layout of one row pass of the tiled 3-pass pipeline.
@@ -164,13 +169,39 @@ inline void entry_pos(const PhaseGeom& g, int64_t line, int64_t q, int64_t& word
     bit = (int)(g.E * (lane % g.epw));
 }
 
+// 32-bit word index and bit offset (< 32) of entry (line, slot q) in either format
+inline void entry_pos32(const PhaseGeom& g, int64_t line, int64_t q, int64_t& wi, int& b) {
+    if (g.dense) {
+        const int64_t round = q >> 5, lane = q & 31;
+        const int64_t bit = lane * g.E;
+        wi = line * g.wpl + round * g.E + (bit >> 5);
+        b = (int)(bit & 31);
+    } else {
+        int64_t w64;
+        int bit;
+        entry_pos(g, line, q, w64, bit);
+        wi = 2 * w64 + (bit >> 5);
+        b = bit & 31;
+    }
+}
+
+inline void pack_entry(uint32_t* words, const PhaseGeom& g, int64_t line, int64_t q, uint64_t entry) {
+    int64_t wi;
+    int b;
+    entry_pos32(g, line, q, wi, b);
+    const uint64_t sh = entry << b;
+    words[wi] |= (uint32_t)sh;
+    if (b + g.E > 32) words[wi + 1] |= (uint32_t)(sh >> 32);
+}
+
 inline uint32_t unpack_entry(const std::vector<uint32_t>& words, const PhaseGeom& g,
                              int64_t line, int64_t q) {
-    int64_t w;
-    int bit;
-    entry_pos(g, line, q, w, bit);
-    const uint64_t v = (uint64_t)words[2 * w] | ((uint64_t)words[2 * w + 1] << 32);
-    return (uint32_t)((v >> bit) & ((1ull << g.E) - 1));
+    int64_t wi;
+    int b;
+    entry_pos32(g, line, q, wi, b);
+    uint64_t v = words[wi];
+    if (b + g.E > 32) v |= (uint64_t)words[wi + 1] << 32;
+    return (uint32_t)((v >> b) & ((1ull << g.E) - 1));
 }
 
 // Entry of (tile T, warp-round q, lane x) of a TLC pass.

@@ -785,6 +785,13 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         phi[1][(int64_t)kk * r + i] = (uint16_t)drow;           // Phi2_k(i) = P(x) div c
         phi[2][(int64_t)drow * c + kk] = (uint16_t)dcol;        // Phi3_i'(k) = P(x) mod c
     }
+    // pass structure
+    int passes = opt ? opt->passes : 0;
+    // measured on B200 (DESIGN.md §7): fused CTA to 2^14, TLC 3-pass 2^15..2^25 (LINES /
+    // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^26
+    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 25 ? 3 : 5);
+    // dense schedule bitstreams only where the 5-pass row kernels read them
+    const bool dense_phases = passes == 5 && !(opt && opt->sched_format < 0);
     // geometry of the three phases
     const int64_t lines[3] = {r, c, r};
     const int64_t Ls[3] = {c, r, c};
@@ -797,13 +804,15 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.E = 2 * g.logL - 5;
         g.epw = 64 / g.E;
         g.w64 = (kW + g.epw - 1) / g.epw;
-        g.words = g.lines * (g.L / kW) * g.w64 * 2;
+        g.dense = dense_phases && (g.logL >= 14 || (opt && opt->sched_format == 2)) ? 1 : 0;
+        g.wpl = (int64_t)(g.L / kW) * (g.dense ? g.E : g.w64 * 2);
+        g.words = g.lines * g.wpl;
     }
     // 5-6. bank-level colouring of every line, packed (W64); not needed by TLC plans
     auto build_line_schedules = [&]() -> int {
         for (int f = 0; f < 3; ++f) {
             PhaseGeom& g = P.ph[f];
-            P.sched[f].assign((size_t)g.words, 0u);
+            P.sched[f].assign((size_t)g.words + 4, 0u);    // +4: a dense decode's second load
             const int64_t L = g.L;
             const uint16_t* ph = phi[f].data();
             uint32_t* W = P.sched[f].data();
@@ -812,7 +821,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 // all lines' bank graphs at once on the device (vertex (line, j mod 32) ->
                 // (line, Phi(j) mod 32)), colour + W64 packing there
                 GpuPlanStats gs;
-                const cudaError_t ce = gpu_line_schedules(ph, n, g.logL, g.E, g.epw, g.w64, W, &gs);
+                const cudaError_t ce = gpu_line_schedules(ph, n, g.logL, g.E, g.epw, g.w64, g.dense, W, &gs);
                 if (ce != cudaSuccess) {
                     err = std::string("GPU planner (bank colouring): ") + cudaGetErrorString(ce);
                     return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
@@ -837,12 +846,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                     for (int64_t j = 0; j < L; ++j) {
                         const uint64_t sigma = (uint64_t)(j >> 5);
                         const uint64_t entry = (sigma << g.logL) | phl[j];
-                        int64_t w;
-                        int bit;
-                        entry_pos(g, line, (int64_t)col[j] * kW + (j & 31), w, bit);
-                        const uint64_t sh = entry << bit;
-                        W[2 * w] |= (uint32_t)sh;
-                        W[2 * w + 1] |= (uint32_t)(sh >> 32);
+                        pack_entry(W, g, line, (int64_t)col[j] * kW + (j & 31), entry);
                     }
                 }
             }
@@ -852,11 +856,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         return PERM_OK;
     };
 
-    // pass structure
-    int passes = opt ? opt->passes : 0;
-    // measured on B200 (DESIGN.md §7): fused CTA to 2^14, TLC 3-pass 2^15..2^25 (LINES /
-    // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^26
-    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 25 ? 3 : 5);
+    // pass structure (chosen above, with the schedule format)
     if (passes == 1 && k > 14) { err = "fused single-CTA pass needs n <= 2^14"; return PERM_EUNSUPPORTED; }
     if (passes != 1 && passes != 3 && passes != 5) { err = "passes must be 0, 1, 3 or 5"; return PERM_EINVAL; }
     P.passes = passes;
@@ -898,7 +898,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     // bytes of one TMA stage: h lines (stride L + pad) + the tile's packed schedule
     auto stage_bytes = [&](int64_t h, int f, int pad) -> int64_t {
         const PhaseGeom& g = P.ph[f];
-        return h * (g.L + pad) * 4 + h * (g.L / kW) * g.w64 * 8;
+        return h * (g.L + pad) * 4 + h * g.wpl * 4;
     };
     constexpr int64_t kSmemBudget = 220 * 1024;
     int layout = opt ? opt->layout : 0;
@@ -967,7 +967,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.in = runs(L, 0, h * L);
             rp.out = runs(L, 0, h * L);
             // TMA pipeline when `stages` tiles (lines + schedule) fit in shared memory
-            const bool sched16 = (h * (L / kW) * P.ph[f].w64 * 2) % 4 == 0;
+            const bool sched16 = (h * P.ph[f].wpl) % 4 == 0;
             const bool no_tma = opt && opt->no_tma > 0;
             const bool force_sg = opt && opt->no_tma < 0;
             rp.tma = (stages * stage_bytes(h, f, 0) <= kSmemBudget && sched16 && !no_tma && !force_sg) ? 1 : 0;
@@ -1011,7 +1011,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 tmp.threads = 256;
                 rp.conflicts_out = rp.out.cross ? simulate_conflicts(tmp, g, false) : 1;
             }
-            if ((rp.h * (g.L / kW) * g.w64 * 2) % 4) { err = "TMA tile schedule is not 16-byte sized"; return PERM_EINVAL; }
+            if ((rp.h * g.wpl) % 4) { err = "TMA tile schedule is not 16-byte sized"; return PERM_EINVAL; }
             const int64_t sb = rp.split ? (int64_t)g.L / 2 * 4
                                : rp.sg ? (int64_t)rp.h * (g.L + pad) * 4 : stage_bytes(rp.h, rp.phase, pad);
             if (rp.stages * sb > kSmemBudget) {
@@ -1071,9 +1071,10 @@ int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, i
     const int64_t count[3] = {P.r_l, P.c_l, P.r_l};
     for (int f = 0; f < 3; ++f) {
         PhaseGeom& g = P.ph[f];
-        const int64_t wpl = (int64_t)(g.L / kW) * g.w64 * 2;     // words per line
+        const int64_t wpl = g.wpl;                                // words per line
         std::vector<uint32_t> slice(P.sched[f].begin() + first[f] * wpl,
                                     P.sched[f].begin() + (first[f] + count[f]) * wpl);
+        slice.resize(slice.size() + 4, 0u);      // dense decode's second load stays in bounds
         P.sched[f].swap(slice);
         g.lines = count[f];
         g.words = count[f] * wpl;

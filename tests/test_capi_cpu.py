@@ -106,7 +106,7 @@ def test_cpp_plan_22_random(lib):
     assert info["passes"] == 3
     # W64 schedule: 17-bit entries, 3 per 64-bit word, 11 words per warp-round of 32
     assert info["entry_bits"] == [17, 17, 17]
-    assert info["sched_bytes"] == 3 * (n // 32) * 11 * 8
+    assert info["sched_bytes"] == 3 * ((n // 32) * 11 * 8 + 16)    # + 4 pad words per phase
 
 
 def test_pass_options_and_info(lib):
@@ -320,3 +320,24 @@ def test_distribution_and_direct_shortcut(lib, k):
     assert lib.Plan(W.make_perm("bitrev", n), device=False).info()["direct"] == 0
     if k >= 16:   # sharded plans never take the single-device shortcut
         assert lib.Plan(W.identity(n), device=False, world=2, rank=0).info()["direct"] == 0
+
+
+@pytest.mark.parametrize("k", [12, 14, 16, 17])
+@pytest.mark.parametrize("fam", ["random", "bitrev", "shuffle"])
+def test_dense_schedule_format_passes_oracle_checker(lib, fam, k):
+    # 5-pass per-line schedules as dense bitstreams (E bits per entry, the default for
+    # lines of >= 16384 words; forced here with sched_format = 2) decode to a valid plan
+    n = 1 << k
+    r, c = W.view_shape(n)
+    p = W.make_perm(fam, n, seed=5 + k)
+    info, kappa, sched = export_plan(lib, p, passes=5, sched_format=2)
+    OC.assert_plan(p, kappa, sched, r, c, 32)
+    with lib.Plan(p, device=False, passes=5, sched_format=2) as pl:
+        d = pl.describe()
+    for rp in d["row_passes"]:
+        assert rp["dense"] == 1 and rp["sched_words_per_line"] == rp["L"] // 32 * rp["E"]
+    # W64 (sched_format = -1) and dense give the same logical schedule
+    _, kappa2, sched2 = export_plan(lib, p, passes=5, sched_format=-1)
+    assert np.array_equal(kappa, kappa2)
+    for (s1, t1), (s2, t2) in zip(sched, sched2):
+        assert np.array_equal(s1, s2) and np.array_equal(t1, t2)

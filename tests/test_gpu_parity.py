@@ -392,6 +392,10 @@ def test_schedule_from_global(P, fam, k):
         b, info = run(P, p, a, passes=5, no_tma=-1, stages=stages)
         assert info["passes"] == 5
         assert np.array_equal(b, ref), stages
+    # dense schedule bitstreams (default for L >= 16384) in the SG, slot and plain kernels
+    for no_tma in (-1, 0, 1):
+        b, _ = run(P, p, a, passes=5, no_tma=no_tma, sched_format=2)
+        assert np.array_equal(b, ref), ("dense", no_tma)
 
 
 @pytest.mark.parametrize("fam,k", [(f, k) for f in ("random", "bitrev", "identity") for k in (16, 20, 22, 24)]
@@ -403,11 +407,13 @@ def test_half_line_ring(P, fam, k):
     n = 1 << k
     p = W.make_perm(fam, n, seed=31 + k)
     a = W.make_data(n)
-    with P.Plan(p, passes=5, no_tma=-2, direct=-1) as plan:
-        d = plan.describe()
-        assert all(rp["split"] == 1 and rp["h"] == 1 for rp in d["row_passes"])
-        da = dev(a)
-        db = torch.full_like(da, -1)
-        plan.apply(da, db)
-        torch.cuda.synchronize()
-        assert np.array_equal(host_words(db), OA.apply_ref(p, a))
+    for fmt in (-1, 2):          # W64 and dense schedule formats
+        with P.Plan(p, passes=5, no_tma=-2, direct=-1, sched_format=fmt) as plan:
+            d = plan.describe()
+            assert all(rp["split"] == 1 and rp["h"] == 1 for rp in d["row_passes"])
+            assert all(rp["dense"] == (fmt == 2) for rp in d["row_passes"])
+            da = dev(a)
+            db = torch.full_like(da, -1)
+            plan.apply(da, db)
+            torch.cuda.synchronize()
+            assert np.array_equal(host_words(db), OA.apply_ref(p, a)), fmt

@@ -45,12 +45,14 @@ def test_gpu_planner_line_schedules(P, fam, k):
     r, c = W.view_shape(n)
     p = W.make_perm(fam, n, seed=100 + k)
     passes = 1 if k <= 14 and k % 2 == 0 else 5
-    with P.Plan(p, passes=passes, gpu_planner=1, direct=-1) as plan:
-        info = plan.info()
-        assert info["gpu_planner"] == 1
-        kappa, scheds = plan.export()
-        OC.assert_plan(p, kappa.astype(np.int64), [decode(s) for s in scheds], r, c, 32)
-        assert apply_ok(P, plan, p, W.make_data(n))
+    # 5-pass: also the dense bitstream format (device-side packing of both formats)
+    for fmt in ((0,) if passes == 1 else (0, 2)):
+        with P.Plan(p, passes=passes, gpu_planner=1, direct=-1, sched_format=fmt) as plan:
+            info = plan.info()
+            assert info["gpu_planner"] == 1
+            kappa, scheds = plan.export()
+            OC.assert_plan(p, kappa.astype(np.int64), [decode(s) for s in scheds], r, c, 32)
+            assert apply_ok(P, plan, p, W.make_data(n))
 
 
 @pytest.mark.parametrize("fam", W.FAMILIES)

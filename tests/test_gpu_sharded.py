@@ -36,7 +36,9 @@ def test_virtual_ranks(P, G, k, no_tma):
     a = W.make_data(n)
     for fam in ("random", "bitrev", "transpose"):
         p = W.make_perm(fam, n, seed=G + k)
-        plans = [P.Plan(p, world=G, rank=g, no_tma=no_tma) for g in range(G)]
+        # dense schedule bitstreams with the SG kernels (no_tma = -1)
+        fmt = 2 if no_tma == -1 else 0
+        plans = [P.Plan(p, world=G, rank=g, no_tma=no_tma, sched_format=fmt) for g in range(G)]
         try:
             a_sh = [torch.from_numpy(a[g * shard:(g + 1) * shard].view(np.int32).copy()).cuda() for g in range(G)]
             b_sh = [torch.full((shard,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
