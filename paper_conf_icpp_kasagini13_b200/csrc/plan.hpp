@@ -9,6 +9,9 @@
 
 #include <cstdint>
 #include <string>
+#include <memory>
+#include <new>
+#include <utility>
 #include <vector>
 
 #include "../../include/perm.h"
@@ -16,6 +19,19 @@
 namespace perm {
 
 constexpr int kW = 32;                 // HMM width w = warp size = banks (L199-L207)
+
+// allocator that default-initialises (no zero fill): large planner arrays that are
+// written in full before they are read (zero-filling GBs at n = 2^30 costs seconds)
+template <class T>
+struct NoInitAlloc : std::allocator<T> {
+    template <class U> struct rebind { using other = NoInitAlloc<U>; };
+    NoInitAlloc() = default;
+    template <class U> NoInitAlloc(const NoInitAlloc<U>&) {}
+    template <class U> void construct(U* p) noexcept { ::new ((void*)p) U; }
+    template <class U, class... A> void construct(U* p, A&&... a) { ::new ((void*)p) U(std::forward<A>(a)...); }
+};
+using U16Buf = std::vector<uint16_t, NoInitAlloc<uint16_t>>;
+using U32Buf = std::vector<uint32_t, NoInitAlloc<uint32_t>>;
 
 // One phase of row-wise permutations: `lines` independent lines of length L.
 // Device schedule ("W64" format): entry = (sigma << logL) | t, E = 2*logL - 5
@@ -142,7 +158,7 @@ struct HostPlan {
     RowPass rp[3];
     int32_t fused_ept = 0, fused_threads = 0, fused_Ls = 0;
     std::vector<uint16_t> kappa;
-    std::vector<uint32_t> sched[3];
+    U32Buf sched[3];
     double ms_colour = 0, ms_bank = 0;
     int32_t threads_used = 1;
     int32_t gpu_planner = 0;   // 1: colourings ran on the device (gplan.cu)
@@ -194,7 +210,7 @@ inline void pack_entry(uint32_t* words, const PhaseGeom& g, int64_t line, int64_
     if (b + g.E > 32) words[wi + 1] |= (uint32_t)(sh >> 32);
 }
 
-inline uint32_t unpack_entry(const std::vector<uint32_t>& words, const PhaseGeom& g,
+inline uint32_t unpack_entry(const U32Buf& words, const PhaseGeom& g,
                              int64_t line, int64_t q) {
     int64_t wi;
     int b;
@@ -205,7 +221,7 @@ inline uint32_t unpack_entry(const std::vector<uint32_t>& words, const PhaseGeom
 }
 
 // Entry of (tile T, warp-round q, lane x) of a TLC pass.
-inline uint32_t tlc_entry(const std::vector<uint32_t>& words, const TlcPass& tp, int64_t T,
+inline uint32_t tlc_entry(const U32Buf& words, const TlcPass& tp, int64_t T,
                           int64_t q, int64_t x) {
     const int64_t pw = q / tp.ept, m = q % tp.ept;
     const int64_t bit = m * tp.E, w = bit >> 5, off = bit & 31;

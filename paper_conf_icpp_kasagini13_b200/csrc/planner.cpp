@@ -25,7 +25,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <memory>
+#include <new>
 #include <numeric>
+#include <utility>
 
 #ifdef _OPENMP
 #include <omp.h>
@@ -466,7 +469,7 @@ IoMode cross(int64_t blockP, int64_t strideP, int64_t cta_stride) {
 //   pass 1: src = i_in*c + j,                     dst = ((k/h2)*h1 + i_in)*h2 + k%h2
 //   pass 2: src = i*h2 + k_in,                    dst = i'*h2 + k_in
 //   pass 3: src = ((k/h2)*h3 + i_in)*h2 + k%h2,   dst = i_in*c + k'
-int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_options* opt,
+int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
               std::string& err) {
     const int64_t r = P.r, c = P.c;
     P.layout = 3;
@@ -588,7 +591,7 @@ int build_tlc(HostPlan& P, const std::vector<uint16_t>* phi, const perm_plan_opt
         if (opt && opt->gpu_planner > 0) {
             // every tile's bank graph at once on the device (vertex (tile, offset mod 32))
             const int64_t N = tp.ntiles * HL;
-            std::vector<uint16_t> ks((size_t)N), kd((size_t)N);
+            U16Buf ks((size_t)N), kd((size_t)N);
 #pragma omp parallel
             {
                 std::vector<uint32_t> src((size_t)HL), dst((size_t)HL), tval((size_t)HL);
@@ -773,7 +776,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
 
     // 4. phase permutations as per-line arrays (uint16: every L <= 2^15)
     t0 = clk::now();
-    std::vector<uint16_t> phi[3];
+    U16Buf phi[3];
     for (auto& v : phi) v.resize((size_t)n);
 #pragma omp parallel for schedule(static)
     for (int64_t x = 0; x < n; ++x) {
@@ -812,7 +815,14 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     auto build_line_schedules = [&]() -> int {
         for (int f = 0; f < 3; ++f) {
             PhaseGeom& g = P.ph[f];
-            P.sched[f].assign((size_t)g.words + 4, 0u);    // +4: a dense decode's second load
+            // +4: a dense decode's second load; the device path writes every word, the
+            // host path ORs entries into zeroed words
+            if (gpu) {
+                P.sched[f].resize((size_t)g.words + 4);
+                for (int i = 0; i < 4; ++i) P.sched[f][(size_t)g.words + i] = 0u;
+            } else {
+                P.sched[f].assign((size_t)g.words + 4, 0u);
+            }
             const int64_t L = g.L;
             const uint16_t* ph = phi[f].data();
             uint32_t* W = P.sched[f].data();
@@ -1072,7 +1082,7 @@ int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, i
     for (int f = 0; f < 3; ++f) {
         PhaseGeom& g = P.ph[f];
         const int64_t wpl = g.wpl;                                // words per line
-        std::vector<uint32_t> slice(P.sched[f].begin() + first[f] * wpl,
+        U32Buf slice(P.sched[f].begin() + first[f] * wpl,
                                     P.sched[f].begin() + (first[f] + count[f]) * wpl);
         slice.resize(slice.size() + 4, 0u);      // dense decode's second load stays in bounds
         P.sched[f].swap(slice);
