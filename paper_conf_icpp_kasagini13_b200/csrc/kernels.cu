@@ -536,31 +536,58 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
 // Same warp-round structure and W64 schedule (read from global) as
 // permute_lines; slots are 64 KiB apart, so position pos keeps bank pos mod 32
 // and the rounds stay conflict-free.
-template <int EPT>
+template <int EPT, bool DENSE, bool KEEP>
 __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1, const uint32_t* __restrict__ sched,
-                                                   int logL, int E, int epw, int w64, int dense) {
+                                                   int logL, int E, int epw, int w64) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, W = blockDim.x >> 5;
     const int lh = logL - 1;
     const int hmask = (1 << lh) - 1;
-    const SchedDec dec(dense, E, epw, w64, lane);
+    const SchedDec dec(DENSE ? 1 : 0, E, epw, w64, lane);
     const uint32_t tmask = (1u << logL) - 1u;
-    // the schedule is read once: the destination word offsets (< 3 * 2^14 < 2^16) wait
-    // in registers, two per register, across the barrier
+    // one decode per format (compile time): W64 = one 64-bit load, dense = two 32-bit loads
+    auto entry = [&](int q) -> uint32_t {
+        if constexpr (DENSE) {
+            const uint32_t* p = sched + q * E;
+            const uint32_t lo = __ldg(p + dec.dwo), hi = __ldg(p + dec.dwo2);
+            return (uint32_t)((((uint64_t)hi << 32) | lo) >> dec.dbo) & dec.mask;
+        } else {
+            const uint2 wd = __ldg(reinterpret_cast<const uint2*>(sched) + q * w64 + dec.wsel);
+            return (uint32_t)((((uint64_t)wd.y << 32) | wd.x) >> dec.sh) & dec.mask;
+        }
+    };
     uint32_t v[EPT];
-    uint32_t ta[(EPT + 1) / 2];
+    if constexpr (KEEP) {
+        // the schedule is read once: the destination word offsets (< 3 * 2^14 < 2^16)
+        // wait in registers, two per register, across the barrier
+        uint32_t ta[(EPT + 1) / 2];
 #pragma unroll
-    for (int m = 0; m < EPT; ++m) {
-        const uint32_t e = dec.get<false>(sched, warp + W * m);
-        const int s = (int)((e >> logL) << 5) + lane;
-        v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
-        const int t = (int)(e & tmask);
-        const uint32_t ad = (uint32_t)(((t >> lh) ? o1 : o0) + (t & hmask));
-        if (m & 1) ta[m >> 1] |= ad << 16;
-        else ta[m >> 1] = ad;
+        for (int m = 0; m < EPT; ++m) {
+            const uint32_t e = entry(warp + W * m);
+            const int s = (int)((e >> logL) << 5) + lane;
+            v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
+            const int t = (int)(e & tmask);
+            const uint32_t ad = (uint32_t)(((t >> lh) ? o1 : o0) + (t & hmask));
+            if (m & 1) ta[m >> 1] |= ad << 16;
+            else ta[m >> 1] = ad;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
+    } else {
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) {
+            const uint32_t e = entry(warp + W * m);
+            const int s = (int)((e >> logL) << 5) + lane;
+            v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
+        }
+        __syncthreads();
+        const int warp2 = __shfl_sync(kFull, warp, 0);   // not CSE-able: the loads are re-issued
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) {
+            const int t = (int)(entry(warp2 + W * m) & tmask);
+            sm[((t >> lh) ? o1 : o0) + (t & hmask)] = v[m];
+        }
     }
-    __syncthreads();
-#pragma unroll
-    for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
     __syncthreads();
 }
 
@@ -575,8 +602,8 @@ __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1,
 // Half-load j = 2i + q uses slot j mod 3 and is that slot's (j div 3)-th fill:
 // the mbarrier parity every thread waits on is (j div 3) & 1. Schedule: W64,
 // read from global, L2-prefetched one line ahead. Row-major output only.
-template <int EPT>
-__global__ void __launch_bounds__(512, 1) row_pass_split_kernel(const TmaArgs a) {
+template <int EPT, bool DENSE, bool KEEP>
+__global__ void __launch_bounds__((EPT >= 64) ? 512 : 1024, 1) row_pass_split_kernel(const TmaArgs a) {
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x;
     const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1;
@@ -630,8 +657,8 @@ __global__ void __launch_bounds__(512, 1) row_pass_split_kernel(const TmaArgs a)
         mbar_wait(&bars[s0], (uint32_t)(j0 / 3) & 1u);
         mbar_wait(&bars[s1], (uint32_t)(j1 / 3) & 1u);
         if (i < 4) stamp(tr, 2 + 3 * i);
-        permute_split_line<EPT>(smem, s0 * HALF, s1 * HALF, a.r.sched + t * a.sched_words, a.r.logL, a.r.E,
-                                a.r.epw, a.r.w64, a.r.dense);
+        permute_split_line<EPT, DENSE, KEEP>(smem, s0 * HALF, s1 * HALF, a.r.sched + t * a.sched_words, a.r.logL,
+                                             a.r.E, a.r.epw, a.r.w64);
         if (i < 4) stamp(tr, 3 + 3 * i);
         if (tid == 0) {
             fence_proxy_async();     // generic-proxy smem writes -> async-proxy reads
@@ -1782,8 +1809,20 @@ cudaError_t prep_ws(HostPlan& P, int f) {
 }
 
 template <int EPT>
-const void* tma_kernel_ptr(bool cross, bool sg, bool split = false) {
-    if (split) return (const void*)row_pass_split_kernel<EPT>;
+const void* split_kernel_ptr(bool dense, bool keep) {
+    if constexpr (EPT < 8) {
+        return nullptr;
+    } else {
+        if (dense) return keep ? (const void*)row_pass_split_kernel<EPT, true, true>
+                               : (const void*)row_pass_split_kernel<EPT, true, false>;
+        return keep ? (const void*)row_pass_split_kernel<EPT, false, true>
+                    : (const void*)row_pass_split_kernel<EPT, false, false>;
+    }
+}
+
+template <int EPT>
+const void* tma_kernel_ptr(bool cross, bool sg, bool split = false, bool dense = false, bool keep = true) {
+    if (split) return split_kernel_ptr<EPT>(dense, keep);
     if (sg) return cross ? (const void*)row_pass_tma_kernel<EPT, true, true>
                          : (const void*)row_pass_tma_kernel<EPT, false, true>;
     return cross ? (const void*)row_pass_tma_kernel<EPT, true> : (const void*)row_pass_tma_kernel<EPT, false>;
@@ -1793,7 +1832,11 @@ template <int EPT>
 cudaError_t set_tma_smem(bool cross, size_t smem) {
     cudaError_t e = set_smem(tma_kernel_ptr<EPT>(cross, false), smem);
     if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true), smem);
-    return e == cudaSuccess ? set_smem(tma_kernel_ptr<EPT>(cross, true, true), smem) : e;
+    if constexpr (EPT >= 8) {
+        for (int v = 0; v < 4 && e == cudaSuccess; ++v)
+            e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, v & 1, v >> 1), smem);
+    }
+    return e;
 }
 
 template <int EPT>
@@ -1802,7 +1845,9 @@ cudaError_t grid_tma(HostPlan& P, int f) {
     const size_t smem = tma_smem(P, f);
     int nb = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &nb, tma_kernel_ptr<EPT>(rp.out.cross != 0, rp.sg != 0, rp.split != 0), rp.threads, smem);
+        &nb, tma_kernel_ptr<EPT>(rp.out.cross != 0, rp.sg != 0, rp.split != 0, P.ph[rp.phase].dense != 0,
+                                 rp.split_keep != 0),
+        rp.threads, smem);
     if (e != cudaSuccess) return e;
     if (nb < 1) return cudaErrorInvalidConfiguration;
     const long long cap = (long long)nb * sm_count();
@@ -2182,13 +2227,20 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const bool cx = rp.out.cross != 0;
         const bool sg = rp.sg != 0;
         if (rp.split) {
+            const bool dn = g.dense != 0, kp = rp.split_keep != 0;
+#define PERM_SPLIT_CASE(E_)                                                                               \
+    case E_:                                                                                              \
+        if (dn) return kp ? launch(row_pass_split_kernel<E_, true, true>, grid, block, smem, s, pdl, ta)    \
+                          : launch(row_pass_split_kernel<E_, true, false>, grid, block, smem, s, pdl, ta);  \
+        return kp ? launch(row_pass_split_kernel<E_, false, true>, grid, block, smem, s, pdl, ta)           \
+                  : launch(row_pass_split_kernel<E_, false, false>, grid, block, smem, s, pdl, ta);
             switch (rp.ept) {
-                case 4: return launch(row_pass_split_kernel<4>, grid, block, smem, s, pdl, ta);
-                case 8: return launch(row_pass_split_kernel<8>, grid, block, smem, s, pdl, ta);
-                case 16: return launch(row_pass_split_kernel<16>, grid, block, smem, s, pdl, ta);
-                case 32: return launch(row_pass_split_kernel<32>, grid, block, smem, s, pdl, ta);
-                case 64: return launch(row_pass_split_kernel<64>, grid, block, smem, s, pdl, ta);
+                PERM_SPLIT_CASE(8)
+                PERM_SPLIT_CASE(16)
+                PERM_SPLIT_CASE(32)
+                PERM_SPLIT_CASE(64)
             }
+#undef PERM_SPLIT_CASE
             return cudaErrorInvalidValue;
         }
 #define PERM_TMA_CASE(E_)                                                                      \

@@ -1006,6 +1006,23 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             rp.threads = 32 + 512 + (rp.out.cross ? 256 : 0);
         } else {
             choose_threads(rp, g.L);
+            if (rp.split) {
+                // half-line ring variants (PERM_SPLIT): r1024 [default] = destinations
+                // re-decoded in the write hop, 1024 threads (EPT 32 at L = 32768, no
+                // spills); k1024 = destinations kept in registers; k512 / r512 = 512 threads
+                // (EPT 64: spills)
+                const char* sv = std::getenv("PERM_SPLIT");
+                const std::string v = sv ? sv : "r1024";
+                rp.split_keep = v[0] == 'k' ? 1 : 0;
+                const int64_t T = (v.find("1024") != std::string::npos) ? 1024 : 512;
+                if ((int64_t)rp.h * g.L >= 8 * T) {
+                    rp.threads = (int32_t)T;
+                    rp.ept = (int32_t)((int64_t)rp.h * g.L / T);
+                } else if (rp.ept < 8) {
+                    rp.ept = 8;
+                    rp.threads = (int32_t)std::max<int64_t>(32, (int64_t)rp.h * g.L / 8);
+                }
+            }
         }
         if (rp.tma) {
             // TMA tiles: lines land at 16-byte aligned strides; a CROSS store of h = 8
