@@ -88,8 +88,8 @@ typedef struct {
                              by the source offset: 19 instead of 21 bits at n = 2^22) wherever a
                              kernel is compiled for its width (not with fuse = 1).
                              5-pass per-line schedules: 0 = dense bitstreams (E bits per entry)
-                             for lines of >= 16384 words, W64 below; 2 = dense for every line
-                             length; -1 = W64 everywhere */
+                             for lines of 16384 words (the schedule-from-global slots), W64
+                             elsewhere; 2 = dense for every line length; -1 = W64 everywhere */
     int32_t gpu_planner; /* where the offline colourings run: 1 = on the
                             current CUDA device (gplan.cu: Euler split with ruling-set cycle
                             labelling), -1 = host threads (planner.cpp), 0 = auto (device for

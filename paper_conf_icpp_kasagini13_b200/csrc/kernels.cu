@@ -536,7 +536,7 @@ __global__ void __launch_bounds__(512, (EPT <= 16) ? 2 : 1) row_pass_tma_kernel(
 // Same warp-round structure and W64 schedule (read from global) as
 // permute_lines; slots are 64 KiB apart, so position pos keeps bank pos mod 32
 // and the rounds stay conflict-free.
-template <int EPT, bool DENSE, bool KEEP>
+template <int EPT, bool DENSE, bool KEEP, bool MERGE = false>
 __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1, const uint32_t* __restrict__ sched,
                                                    int logL, int E, int epw, int w64) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, W = blockDim.x >> 5;
@@ -581,7 +581,11 @@ __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1,
             v[m] = sm[((s >> lh) ? o1 : o0) + (s & hmask)];
         }
         __syncthreads();
-        const int warp2 = __shfl_sync(kFull, warp, 0);   // not CSE-able: the loads are re-issued
+        // MERGE: the write hop names the same addresses, so the compiler issues each
+        // schedule load once, all up front (measured fastest at L = 32768 with W64
+        // entries, although it parks part of them in local memory); otherwise the
+        // loads are re-issued after the barrier (warp index laundered through a shuffle)
+        const int warp2 = MERGE ? warp : __shfl_sync(kFull, warp, 0);
 #pragma unroll
         for (int m = 0; m < EPT; ++m) {
             const int t = (int)(entry(warp2 + W * m) & tmask);
@@ -604,6 +608,8 @@ __device__ __forceinline__ void permute_split_line(uint32_t* sm, int o0, int o1,
 // read from global, L2-prefetched one line ahead. Row-major output only.
 template <int EPT, bool DENSE, bool KEEP>
 __global__ void __launch_bounds__((EPT >= 64) ? 512 : 1024, 1) row_pass_split_kernel(const TmaArgs a) {
+    // !DENSE && !KEEP: W64 entries, loads merged across the two hops (the default)
+    constexpr bool MERGE = !DENSE && !KEEP;
     extern __shared__ __align__(128) uint32_t smem[];
     const int tid = threadIdx.x;
     const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1;
@@ -657,8 +663,8 @@ __global__ void __launch_bounds__((EPT >= 64) ? 512 : 1024, 1) row_pass_split_ke
         mbar_wait(&bars[s0], (uint32_t)(j0 / 3) & 1u);
         mbar_wait(&bars[s1], (uint32_t)(j1 / 3) & 1u);
         if (i < 4) stamp(tr, 2 + 3 * i);
-        permute_split_line<EPT, DENSE, KEEP>(smem, s0 * HALF, s1 * HALF, a.r.sched + t * a.sched_words, a.r.logL,
-                                             a.r.E, a.r.epw, a.r.w64);
+        permute_split_line<EPT, DENSE, KEEP, MERGE>(smem, s0 * HALF, s1 * HALF, a.r.sched + t * a.sched_words,
+                                                    a.r.logL, a.r.E, a.r.epw, a.r.w64);
         if (i < 4) stamp(tr, 3 + 3 * i);
         if (tid == 0) {
             fence_proxy_async();     // generic-proxy smem writes -> async-proxy reads

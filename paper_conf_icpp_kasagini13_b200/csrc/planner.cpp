@@ -736,7 +736,11 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     }
     P.n = n; P.eb = eb; P.k = k;
     // view r x c (L603: "not restricted to a square matrix"); default c = 2^ceil(k/2)
-    const int logc = (opt && opt->log2c > 0) ? opt->log2c : k - k / 2, logr = k - logc;
+    // n = 2^29 (5 passes): c = 2^14, r = 2^15, so the two row phases run on 16384-word
+    // lines (schedule-from-global slots) and only the column phase on 32768-word lines
+    // (half-line ring) -- the other way round it is two slow passes and one fast one
+    const int logc_auto = (k == 29 && !(opt && opt->passes == 3)) ? 14 : k - k / 2;
+    const int logc = (opt && opt->log2c > 0) ? opt->log2c : logc_auto, logr = k - logc;
     if (logc < 5 || logr < 5) { err = "view: log2c must leave r, c >= 32"; return PERM_EINVAL; }
     P.r = int64_t(1) << logr;
     P.c = int64_t(1) << logc;
@@ -807,7 +811,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.E = 2 * g.logL - 5;
         g.epw = 64 / g.E;
         g.w64 = (kW + g.epw - 1) / g.epw;
-        g.dense = dense_phases && (g.logL >= 14 || (opt && opt->sched_format == 2)) ? 1 : 0;
+        // dense at L = 16384 (SG slots); L = 32768 lines (half-line ring) keep W64, whose
+        // merged loads measured faster there (profiles/r01_split_variants_s5.log)
+        g.dense = dense_phases && (g.logL == 14 || (opt && opt->sched_format == 2)) ? 1 : 0;
         g.wpl = (int64_t)(g.L / kW) * (g.dense ? g.E : g.w64 * 2);
         g.words = g.lines * g.wpl;
     }
@@ -1007,12 +1013,13 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         } else {
             choose_threads(rp, g.L);
             if (rp.split) {
-                // half-line ring variants (PERM_SPLIT): r1024 [default] = destinations
-                // re-decoded in the write hop, 1024 threads (EPT 32 at L = 32768, no
-                // spills); k1024 = destinations kept in registers; k512 / r512 = 512 threads
-                // (EPT 64: spills)
+                // half-line ring variants (PERM_SPLIT): r512 [default] = 512 threads, the
+                // write hop re-reads the schedule (merged with the read hop's loads for W64
+                // entries); r1024 = 1024 threads; k512 / k1024 = destinations kept in
+                // registers. Measured at 2^30 (dense / W64 entries): r512 4.08 / 3.20 ms,
+                // r1024 3.90 / 3.33, k1024 4.77, k512 5.40 (spills)
                 const char* sv = std::getenv("PERM_SPLIT");
-                const std::string v = sv ? sv : "r1024";
+                const std::string v = sv ? sv : "r512";
                 rp.split_keep = v[0] == 'k' ? 1 : 0;
                 const int64_t T = (v.find("1024") != std::string::npos) ? 1024 : 512;
                 if ((int64_t)rp.h * g.L >= 8 * T) {

@@ -417,3 +417,30 @@ def test_half_line_ring(P, fam, k):
             plan.apply(da, db)
             torch.cuda.synchronize()
             assert np.array_equal(host_words(db), OA.apply_ref(p, a)), fmt
+
+
+@pytest.mark.parametrize("variant", ["r1024", "k1024", "r512", "k512"])
+@pytest.mark.parametrize("k", [22, 26])
+def test_half_line_ring_variants(P, variant, k, monkeypatch):
+    # register strategies of the half-line ring (PERM_SPLIT, read at plan build), both
+    # schedule formats
+    monkeypatch.setenv("PERM_SPLIT", variant)
+    n = 1 << k
+    p = W.random(n, 70 + k)
+    a = W.make_data(n)
+    ref = OA.apply_ref(p, a)
+    for fmt in (-1, 2):
+        b, _ = run(P, p, a, passes=5, no_tma=-2, sched_format=fmt)
+        assert np.array_equal(b, ref), (variant, fmt)
+
+
+@pytest.mark.parametrize("k", [19, 21])
+@pytest.mark.parametrize("fam", ["random", "transpose", "bitrev"])
+def test_tall_views_5pass(P, k, fam):
+    # r > c views (the n = 2^29 default shape, L603: the view need not be square)
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=k)
+    a = W.make_data(n)
+    b, info = run(P, p, a, passes=5, log2c=k // 2)
+    assert (info["rows"], info["cols"]) == (1 << (k - k // 2), 1 << (k // 2))
+    assert np.array_equal(b, OA.apply_ref(p, a))
