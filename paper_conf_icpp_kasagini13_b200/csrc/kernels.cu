@@ -926,6 +926,138 @@ __global__ void __launch_bounds__(OUT_CROSS ? 32 + kWsPerm + kWsStore : 32 + kWs
     }
 }
 
+// ------------------------------------------------------------------ half-line ring, staged schedule
+
+constexpr int kStgWorkers = 512;                 // 16 warps
+constexpr int kStgChunkWords = 2048;             // 8 KiB schedule chunks (64 W64 rounds)
+constexpr int kStgBufs = 4;                      // chunk ring depth
+
+// Half-line ring (row_pass_split_kernel) with the W64 schedule STREAMED THROUGH SHARED
+// MEMORY: the 35 KiB left beside the three 64 KiB half-line slots hold a ring of four
+// 8 KiB schedule chunks that a dedicated producer warp fills with TMA bulk copies (one
+// chunk = 64 warp-rounds = 4 rounds of each of the 16 permuter warps), running ahead into
+// the next line while the current one is written back. The permuters read each entry once
+// from shared memory (no long-latency global loads in the permute), keep the decoded
+// destination offsets in registers across the barrier, and release a chunk with an
+// mbarrier arrive. Permuters synchronise with named barrier 1 (the producer warp never
+// joins them).
+template <int EPT>
+__global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(const TmaArgs a) {
+    extern __shared__ __align__(128) uint32_t smem[];
+    const int tid = threadIdx.x;
+    const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1, hmask = HALF - 1;
+    uint32_t* cbuf = smem + 3 * HALF;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + kStgBufs * kStgChunkWords);
+    uint64_t* full = bars + 3;                   // chunk landed
+    uint64_t* empty = bars + 3 + kStgBufs;       // chunk consumed by all permuters
+    const int G = gridDim.x;
+    const uint32_t half_bytes = (uint32_t)HALF * 4u;
+    const long long my_lines = a.ntiles > (int)blockIdx.x ? (a.ntiles - 1 - (int)blockIdx.x) / G + 1 : 0;
+    constexpr int kW = kStgWorkers / 32;                   // permuter warps
+    const int w64 = a.r.w64;
+    const int chunks_per_line = EPT / 4;         // == (L/32) / (kStgChunkWords / (2*w64)) for w64 = 16
+
+    auto issue_half = [&](long long j) {
+        const long long i = j >> 1;
+        if (i >= my_lines) return;
+        const int q = (int)(j & 1), slot = (int)(j % 3);
+        const long long t = blockIdx.x + i * G;
+        mbar_arrive_expect_tx(&bars[slot], half_bytes);
+        if (q == 0) prefetch_l2_bulk(a.r.sched + t * a.sched_words, (uint32_t)a.sched_words * 4u);
+        bulk_g2s(smem + slot * HALF, a.r.in + t * (long long)L + (long long)q * HALF, half_bytes, &bars[slot]);
+    };
+
+    if (tid == 0) {
+        for (int s = 0; s < 3; ++s) mbar_init(&bars[s], 1);
+        for (int b = 0; b < kStgBufs; ++b) {
+            mbar_init(&full[b], 1);
+            mbar_init(&empty[b], kStgWorkers);
+        }
+        fence_mbar_init();
+        if (my_lines > 0) prefetch_l2_bulk(a.r.sched + (long long)blockIdx.x * a.sched_words,
+                                           (uint32_t)a.sched_words * 4u);
+    }
+    __syncthreads();
+    const long long total_chunks = my_lines * chunks_per_line;
+    auto issue_chunk = [&](long long g) {
+        const int b = (int)(g % kStgBufs);
+        const long long i = g / chunks_per_line, c = g - i * chunks_per_line;
+        const long long t = blockIdx.x + i * G;
+        mbar_arrive_expect_tx(&full[b], kStgChunkWords * 4u);
+        bulk_g2s(cbuf + b * kStgChunkWords, a.r.sched + t * a.sched_words + c * kStgChunkWords,
+                 kStgChunkWords * 4u, &full[b]);
+    };
+    if (tid == 0)
+        for (long long g = 0; g < kStgBufs && g < total_chunks; ++g) issue_chunk(g);
+    pdl_wait();
+    if (tid == 0) {
+        issue_half(0);
+        issue_half(1);
+        issue_half(2);
+    }
+    pdl_launch_dependents();
+    const int lane = tid & 31, warp = tid >> 5;
+    const int wsel = lane / a.r.epw;
+    const int sh = a.r.E * (lane - wsel * a.r.epw);
+    const uint32_t mask = (1u << a.r.E) - 1u, tmask = (1u << a.r.logL) - 1u;
+    const int logL = a.r.logL;
+    constexpr int MPC = 4;               // m-steps per chunk: 64 rounds = 4 x 16 warps
+    constexpr int CPL = EPT / MPC;       // chunks per line (host: w64 == 16, so 64 rounds/chunk)
+    for (long long i = 0; i < my_lines; ++i) {
+        const long long t = blockIdx.x + i * G;
+        const long long j0 = 2 * i, j1 = 2 * i + 1;
+        const int s0 = (int)(j0 % 3), s1 = (int)(j1 % 3);
+        const int o0 = s0 * HALF, o1 = s1 * HALF;
+        mbar_wait(&bars[s0], (uint32_t)(j0 / 3) & 1u);
+        mbar_wait(&bars[s1], (uint32_t)(j1 / 3) & 1u);
+        uint32_t v[EPT];
+        uint32_t ta[EPT / 2];
+#pragma unroll
+        for (int c = 0; c < CPL; ++c) {
+            const long long g = i * CPL + c;
+            const int b = (int)(g % kStgBufs);
+            mbar_wait(&full[b], (uint32_t)((g / kStgBufs) & 1));
+            const uint2* cb = reinterpret_cast<const uint2*>(cbuf + b * kStgChunkWords);
+#pragma unroll
+            for (int mm = 0; mm < MPC; ++mm) {
+                const int m = c * MPC + mm;
+                const uint2 wd = cb[(warp + kW * mm) * w64 + wsel];
+                const uint32_t e = (uint32_t)((((uint64_t)wd.y << 32) | wd.x) >> sh) & mask;
+                const int s = (int)((e >> logL) << 5) + lane;
+                v[m] = smem[((s >> lh) ? o1 : o0) + (s & hmask)];
+                const int tt = (int)(e & tmask);
+                const uint32_t ad = (uint32_t)(((tt >> lh) ? o1 : o0) + (tt & hmask));
+                if (m & 1) ta[m >> 1] |= ad << 16;
+                else ta[m >> 1] = ad;
+            }
+            mbar_arrive(&empty[b]);
+            if (tid == 0 && g + kStgBufs < total_chunks) {
+                mbar_wait(&empty[b], (uint32_t)((g / kStgBufs) & 1));   // all 512 consumed chunk g
+                issue_chunk(g + kStgBufs);
+            }
+        }
+        __syncthreads();
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) smem[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
+        __syncthreads();
+        if (tid == 0) {
+            fence_proxy_async();
+            uint32_t* dst = a.r.out + t * (long long)L;
+            bulk_s2g(dst, smem + o0, half_bytes);
+            bulk_commit();
+            bulk_s2g(dst + HALF, smem + o1, half_bytes);
+            bulk_commit();
+            bulk_wait_read1();
+            fence_proxy_async();
+            issue_half(2 * i + 3);
+            bulk_wait_read0();
+            fence_proxy_async();
+            issue_half(2 * i + 4);
+        }
+    }
+    if (tid == 0) bulk_wait0();
+}
+
 // ------------------------------------------------------------------ fused 3-pass persistent kernel
 
 __device__ __forceinline__ void fence_proxy_async_global() {
@@ -1787,6 +1919,8 @@ cudaError_t set_smem(K kernel, size_t bytes) {
 size_t tma_smem(const HostPlan& P, int f) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
+    if (rp.split && rp.split_stg)
+        return (size_t)3 * (g.L / 2) * 4 + (size_t)kStgBufs * kStgChunkWords * 4 + (3 + 2 * kStgBufs) * 8;
     if (rp.split) return (size_t)3 * (g.L / 2) * 4 + 3 * 8;
     const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * g.wpl * 4);
     return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
@@ -1827,7 +1961,11 @@ const void* split_kernel_ptr(bool dense, bool keep) {
 }
 
 template <int EPT>
-const void* tma_kernel_ptr(bool cross, bool sg, bool split = false, bool dense = false, bool keep = true) {
+const void* tma_kernel_ptr(bool cross, bool sg, bool split = false, bool dense = false, bool keep = true,
+                           bool stg = false) {
+    if constexpr (EPT == 32 || EPT == 64) {
+        if (split && stg) return (const void*)row_pass_split_stg_kernel<EPT>;
+    }
     if (split) return split_kernel_ptr<EPT>(dense, keep);
     if (sg) return cross ? (const void*)row_pass_tma_kernel<EPT, true, true>
                          : (const void*)row_pass_tma_kernel<EPT, false, true>;
@@ -1842,6 +1980,9 @@ cudaError_t set_tma_smem(bool cross, size_t smem) {
         for (int v = 0; v < 4 && e == cudaSuccess; ++v)
             e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, v & 1, v >> 1), smem);
     }
+    if constexpr (EPT == 32 || EPT == 64) {
+        if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, false, false, true), smem);
+    }
     return e;
 }
 
@@ -1852,7 +1993,7 @@ cudaError_t grid_tma(HostPlan& P, int f) {
     int nb = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
         &nb, tma_kernel_ptr<EPT>(rp.out.cross != 0, rp.sg != 0, rp.split != 0, P.ph[rp.phase].dense != 0,
-                                 rp.split_keep != 0),
+                                 rp.split_keep != 0, rp.split_stg != 0),
         rp.threads, smem);
     if (e != cudaSuccess) return e;
     if (nb < 1) return cudaErrorInvalidConfiguration;
@@ -2232,6 +2373,11 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const size_t smem = tma_smem(P, f);
         const bool cx = rp.out.cross != 0;
         const bool sg = rp.sg != 0;
+        if (rp.split && rp.split_stg) {
+            if (rp.ept == 32) return launch(row_pass_split_stg_kernel<32>, grid, block, smem, s, pdl, ta);
+            if (rp.ept == 64) return launch(row_pass_split_stg_kernel<64>, grid, block, smem, s, pdl, ta);
+            return cudaErrorInvalidValue;
+        }
         if (rp.split) {
             const bool dn = g.dense != 0, kp = rp.split_keep != 0;
 #define PERM_SPLIT_CASE(E_)                                                                               \

@@ -76,6 +76,7 @@ struct RowPass {
     int32_t sg = 0;           // 1 (tma == 1): schedule read from global (L2-prefetched), slots hold data only
     int32_t split = 0;        // 1 (tma == 1, sg, h == 1): ring of three half-line slots (L = 32768)
     int32_t split_keep = 1;   // split: 1 = destinations kept in registers (512 threads), 0 = re-decoded
+    int32_t split_stg = 0;    // split: 1 = W64 schedule streamed through smem chunks by a producer warp
     int64_t grid = 0;         // persistent CTAs (set at upload from the occupancy query)
     int32_t h = 0;            // lines per CTA (tile)
     int32_t Ls = 0;           // shared-memory line stride (elements) = L + pad

@@ -1021,6 +1021,16 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 const char* sv = std::getenv("PERM_SPLIT");
                 const std::string v = sv ? sv : "r512";
                 rp.split_keep = v[0] == 'k' ? 1 : 0;
+                // s512: the W64 schedule streamed through shared-memory chunks by TMA
+                // (needs 64-bit words holding 2 entries: w64 = 16)
+                const int64_t ept512 = (int64_t)rp.h * g.L / 512;
+                if (v == "s512" && g.w64 == 16 && !g.dense && (ept512 == 32 || ept512 == 64)) {
+                    rp.split_stg = 1;
+                    rp.threads = 512;
+                    rp.ept = (int32_t)ept512;
+                    goto split_done;
+                }
+                {
                 const int64_t T = (v.find("1024") != std::string::npos) ? 1024 : 512;
                 if ((int64_t)rp.h * g.L >= 8 * T) {
                     rp.threads = (int32_t)T;
@@ -1029,6 +1039,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                     rp.ept = 8;
                     rp.threads = (int32_t)std::max<int64_t>(32, (int64_t)rp.h * g.L / 8);
                 }
+                }
+            split_done:;
             }
         }
         if (rp.tma) {

@@ -444,3 +444,23 @@ def test_tall_views_5pass(P, k, fam):
     b, info = run(P, p, a, passes=5, log2c=k // 2)
     assert (info["rows"], info["cols"]) == (1 << (k - k // 2), 1 << (k // 2))
     assert np.array_equal(b, OA.apply_ref(p, a))
+
+
+@pytest.mark.parametrize("k,log2c", [(19, 14), (20, 15), (21, 15)])
+@pytest.mark.parametrize("fam", ["random", "bitrev"])
+def test_half_line_ring_staged_schedule(P, k, log2c, fam, monkeypatch):
+    # PERM_SPLIT=s512: the half-line ring with the W64 schedule streamed through shared
+    # memory in TMA chunks (lines of 16384 / 32768 words via wide views, L603)
+    monkeypatch.setenv("PERM_SPLIT", "s512")
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=k + log2c)
+    a = W.make_data(n)
+    with P.Plan(p, passes=5, no_tma=-2, direct=-1, log2c=log2c, sched_format=-1) as plan:
+        d = plan.describe()
+        long_lines = [rp for rp in d["row_passes"] if rp["L"] >= 16384]
+        assert long_lines and all(rp["threads"] == 512 for rp in long_lines)
+        da = dev(a)
+        db = torch.full_like(da, -1)
+        plan.apply(da, db)
+        torch.cuda.synchronize()
+        assert np.array_equal(host_words(db), OA.apply_ref(p, a))
