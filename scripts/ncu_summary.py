@@ -10,6 +10,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument('--launches')
 ap.add_argument('--full')
 ap.add_argument('--out', required=True)
+ap.add_argument('--only', help="regex: keep only matching kernels in the launch table (e.g. the apply's kernels)")
 ap.add_argument('--traffic-key', help="also write profiles/ncu_traffic.json[key] = per-pass DRAM bytes")
 a = ap.parse_args()
 summary = {}
@@ -38,6 +39,8 @@ if a.launches:
     agg = defaultdict(lambda: defaultdict(list))
     for d in per.values():
         nm = d['name'].split('(')[0].replace('void ', '')[:90]
+        if a.only and not __import__('re').search(a.only, nm):
+            continue
         for k, v in d.items():
             if k != 'name' and isinstance(v, float):
                 agg[nm][k].append(v)
