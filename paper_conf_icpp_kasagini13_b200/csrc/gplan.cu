@@ -95,8 +95,17 @@ __global__ void k_compact(const uint32_t* __restrict__ g, uint32_t* __restrict__
             nxt[e] = g[e];
             s = (uint32_t)e;
         }
-        if (s == (uint32_t)e) {
-            const uint32_t slot = (uint32_t)atomicAdd(count, 1ull);
+        // warp-aggregated slot allocation: one atomic per warp (for short-orbit inputs,
+        // e.g. identity, nearly every edge is a node)
+        const bool is_node = s == (uint32_t)e;
+        const unsigned act = __activemask();
+        const unsigned bal = __ballot_sync(act, is_node);
+        const int leader = __ffs(act) - 1, lane = threadIdx.x & 31;
+        unsigned long long base = 0;
+        if (lane == leader && bal) base = atomicAdd(count, (unsigned long long)__popc(bal));
+        base = __shfl_sync(act, base, leader);
+        if (is_node) {
+            const uint32_t slot = (uint32_t)(base + __popc(bal & ((1u << lane) - 1u)));
             slotof[e] = slot;
             node[slot] = (uint32_t)e;
         }
@@ -136,14 +145,20 @@ __global__ void k_label(const uint32_t* __restrict__ seg, const uint32_t* __rest
         lab[e] = rlab[slotof[seg[e]]];
 }
 
+// colour bit of every edge: b(e) = [label(e) >= label(partner_V(e))]
+__global__ void k_bit(const uint32_t* __restrict__ lab, const uint32_t* __restrict__ pV,
+                      uint8_t* __restrict__ bit, int64_t E) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < E; e += (int64_t)gridDim.x * blockDim.x)
+        bit[e] = lab[e] < lab[pV[e]] ? 0 : 1;
+}
+
 __global__ void k_split(const uint32_t* __restrict__ ord, uint32_t* __restrict__ ord2,
-                        const uint32_t* __restrict__ lab, const uint32_t* __restrict__ pV, int64_t E, int logd) {
+                        const uint8_t* __restrict__ bit, int64_t E, int logd) {
     const int64_t half = (int64_t)1 << (logd - 1);
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < E; q += (int64_t)gridDim.x * blockDim.x) {
         const uint32_t e = ord[q];
         const int64_t blk = q >> logd, i = (q & ((half << 1) - 1)) >> 1;
-        const int64_t b = lab[e] < lab[pV[e]] ? 0 : 1;
-        ord2[(blk << logd) + b * half + i] = e;
+        ord2[(blk << logd) + (int64_t)bit[e] * half + i] = e;
     }
 }
 
@@ -313,8 +328,10 @@ cudaError_t euler_split_device(uint32_t* ordU, uint32_t* ordV, int64_t E, int lo
         }
         // la = final labels of the reduced nodes; spread to every edge (into lb: free)
         k_label<<<G, T, 0, s>>>(seg, slotof, la, lb, E);
-        k_split<<<G, T, 0, s>>>(U, U2, lb, pV, E, logd);
-        k_split<<<G, T, 0, s>>>(V, V2, lb, pV, E, logd);
+        uint8_t* bit = reinterpret_cast<uint8_t*>(g);      // g is dead after the walk
+        k_bit<<<G, T, 0, s>>>(lb, pV, bit, E);
+        k_split<<<G, T, 0, s>>>(U, U2, bit, E, logd);
+        k_split<<<G, T, 0, s>>>(V, V2, bit, E, logd);
         std::swap(U, U2);
         std::swap(V, V2);
         if (st) { st->levels += 1; st->reduced_nodes += (int64_t)R; }

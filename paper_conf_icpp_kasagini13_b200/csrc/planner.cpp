@@ -975,7 +975,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     } else {
         for (int f = 0; f < 3; ++f) {
             const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
-            const bool force_split = opt && opt->no_tma == -2;
+            // (forced half-line ring: lines of >= 256 words, one line per CTA; a 32-word
+            // line would leave a CTA less than one warp)
+            const bool force_split = opt && opt->no_tma == -2 && L >= 256;
             int64_t h = force_split ? 1 : pick(f, std::max<int64_t>(1, pow2_floor(Q / L)));
             if (h < 1 || h > lines_f || (h & (h - 1))) { err = "invalid h for the 5-pass layout"; return PERM_EINVAL; }
             RowPass& rp = P.rp[f];
@@ -997,7 +999,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 rp.stages = (opt && opt->stages > 0) ? opt->stages : (int)std::min<int64_t>(4, fit);
             }
             // one line per slot only (L = 32768): ring of three half-line slots instead
-            if (rp.tma && rp.sg && h == 1 && (rp.stages == 1 || force_split) && 3 * (L / 2) * 4 <= kSmemBudget) {
+            if (rp.tma && rp.sg && h == 1 && (rp.stages == 1 || force_split) && L >= 256 &&
+                3 * (L / 2) * 4 <= kSmemBudget) {
                 rp.split = 1;
                 rp.stages = 3;
             }
@@ -1013,13 +1016,14 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         } else {
             choose_threads(rp, g.L);
             if (rp.split) {
-                // half-line ring variants (PERM_SPLIT): r512 [default] = 512 threads, the
-                // write hop re-reads the schedule (merged with the read hop's loads for W64
-                // entries); r1024 = 1024 threads; k512 / k1024 = destinations kept in
-                // registers. Measured at 2^30 (dense / W64 entries): r512 4.08 / 3.20 ms,
-                // r1024 3.90 / 3.33, k1024 4.77, k512 5.40 (spills)
+                // half-line ring variants (PERM_SPLIT): s512 [default] = W64 schedule streamed
+                // through shared-memory chunks (3.14 ms per pass at 2^30); r512 = 512 threads,
+                // the write hop re-reads the schedule (merged with the read hop's loads for
+                // W64 entries: 3.20 ms); r1024 = 1024 threads; k512 / k1024 = destinations
+                // kept in registers (spill: 4.8-5.4 ms). s512 falls back to r512 where the
+                // schedule words do not hold 2 entries (w64 != 16) or the format is dense.
                 const char* sv = std::getenv("PERM_SPLIT");
-                const std::string v = sv ? sv : "r512";
+                const std::string v = sv ? sv : "s512";
                 rp.split_keep = v[0] == 'k' ? 1 : 0;
                 // s512: the W64 schedule streamed through shared-memory chunks by TMA
                 // (needs 64-bit words holding 2 entries: w64 = 16)
