@@ -990,6 +990,8 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
         bulk_g2s(smem + slot * HALF, a.r.in + t * (long long)L + (long long)q * HALF, half_bytes, &bars[slot]);
     };
 
+    unsigned long long* tr = a.r.trace;
+    stamp(tr, 0);
     if (tid == 0) {
         for (int s = 0; s < 3; ++s) mbar_init(&bars[s], 1);
         for (int b = 0; b < kStgBufs; ++b) {
@@ -1013,6 +1015,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
     if (tid == 0)
         for (long long g = 0; g < kStgBufs && g < total_chunks; ++g) issue_chunk(g);
     pdl_wait();
+    stamp(tr, 1);
     if (tid == 0) {
         issue_half(0);
         issue_half(1);
@@ -1033,6 +1036,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
         const int o0 = s0 * HALF, o1 = s1 * HALF;
         mbar_wait(&bars[s0], (uint32_t)(j0 / 3) & 1u);
         mbar_wait(&bars[s1], (uint32_t)(j1 / 3) & 1u);
+        if (i < 4) stamp(tr, 2 + 3 * (int)i);
         uint32_t v[EPT];
         uint32_t ta[EPT / 2];
 #pragma unroll
@@ -1063,6 +1067,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
 #pragma unroll
         for (int m = 0; m < EPT; ++m) smem[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
         __syncthreads();
+        if (i < 4) stamp(tr, 3 + 3 * (int)i);
         if (tid == 0) {
             fence_proxy_async();
             uint32_t* dst = a.r.out + t * (long long)L;
@@ -1077,8 +1082,10 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
             fence_proxy_async();
             issue_half(2 * i + 4);
         }
+        if (i < 4) stamp(tr, 4 + 3 * (int)i);
     }
     if (tid == 0) bulk_wait0();
+    stamp(tr, 14);
 }
 
 // ------------------------------------------------------------------ fused 3-pass persistent kernel
