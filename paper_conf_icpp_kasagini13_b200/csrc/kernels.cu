@@ -952,33 +952,37 @@ __global__ void __launch_bounds__(OUT_CROSS ? 32 + kWsPerm + kWsStore : 32 + kWs
 // ------------------------------------------------------------------ half-line ring, staged schedule
 
 constexpr int kStgWorkers = 512;                 // 16 warps
-constexpr int kStgChunkWords = 2048;             // 8 KiB schedule chunks (64 W64 rounds)
-constexpr int kStgBufs = 4;                      // chunk ring depth
+constexpr int kStgChunkWords = 2048;             // W64: 8 KiB schedule chunks (64 rounds of 16 words)
+constexpr int kStgDenseWords = 64 * 25;          // dense: 64 rounds of E <= 25 words (6.25 KiB)
 
-// Half-line ring (row_pass_split_kernel) with the W64 schedule STREAMED THROUGH SHARED
-// MEMORY: the 35 KiB left beside the three 64 KiB half-line slots hold a ring of four
-// 8 KiB schedule chunks that a dedicated producer warp fills with TMA bulk copies (one
-// chunk = 64 warp-rounds = 4 rounds of each of the 16 permuter warps), running ahead into
-// the next line while the current one is written back. The permuters read each entry once
-// from shared memory (no long-latency global loads in the permute), keep the decoded
-// destination offsets in registers across the barrier, and release a chunk with an
-// mbarrier arrive. Permuters synchronise with named barrier 1 (the producer warp never
-// joins them).
-template <int EPT>
+// Half-line ring (row_pass_split_kernel) with the schedule STREAMED THROUGH SHARED MEMORY:
+// the 35 KiB left beside the three 64 KiB half-line slots hold a ring of schedule chunks
+// (W64: four of 8 KiB; dense: five of 64*E words) filled with TMA bulk copies. One chunk =
+// 64 warp-rounds = 4 rounds of each of the 16 warps; the ring runs ahead into the next line
+// while the current one is written back. Thread 0 refills a buffer once all 512 threads have
+// arrived on its `empty` mbarrier (16 warps = 4 per SM quadrant keep 128 registers per
+// thread). Each entry is read once from shared memory and the decoded destination offsets
+// stay in registers across the barrier. The permute is bound by the chunk latency (per-CTA
+// traces, profiles/r01_trace_ring_s8.log), hence the dense format's smaller, deeper ring.
+template <int EPT, bool DENSE>
 __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(const TmaArgs a) {
     extern __shared__ __align__(128) uint32_t smem[];
+    constexpr int NB = DENSE ? 5 : 4;            // chunk ring depth
+    constexpr int CWS = DENSE ? kStgDenseWords : kStgChunkWords;   // buffer stride (words)
     const int tid = threadIdx.x;
     const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1, hmask = HALF - 1;
+    const int E = a.r.E;
+    const int CW = DENSE ? 64 * E : kStgChunkWords;                 // words per chunk
     uint32_t* cbuf = smem + 3 * HALF;
-    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + kStgBufs * kStgChunkWords);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + NB * CWS);
     uint64_t* full = bars + 3;                   // chunk landed
-    uint64_t* empty = bars + 3 + kStgBufs;       // chunk consumed by all permuters
+    uint64_t* empty = bars + 3 + NB;             // chunk consumed by all 512 threads
     const int G = gridDim.x;
     const uint32_t half_bytes = (uint32_t)HALF * 4u;
     const long long my_lines = a.ntiles > (int)blockIdx.x ? (a.ntiles - 1 - (int)blockIdx.x) / G + 1 : 0;
-    constexpr int kW = kStgWorkers / 32;                   // permuter warps
+    constexpr int kW = kStgWorkers / 32;                   // warps
     const int w64 = a.r.w64;
-    const int chunks_per_line = EPT / 4;         // == (L/32) / (kStgChunkWords / (2*w64)) for w64 = 16
+    const int chunks_per_line = EPT / 4;         // (L/32 rounds) / 64 rounds per chunk
 
     auto issue_half = [&](long long j) {
         const long long i = j >> 1;
@@ -994,7 +998,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
     stamp(tr, 0);
     if (tid == 0) {
         for (int s = 0; s < 3; ++s) mbar_init(&bars[s], 1);
-        for (int b = 0; b < kStgBufs; ++b) {
+        for (int b = 0; b < NB; ++b) {
             mbar_init(&full[b], 1);
             mbar_init(&empty[b], kStgWorkers);
         }
@@ -1005,15 +1009,14 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
     __syncthreads();
     const long long total_chunks = my_lines * chunks_per_line;
     auto issue_chunk = [&](long long g) {
-        const int b = (int)(g % kStgBufs);
+        const int b = (int)(g % NB);
         const long long i = g / chunks_per_line, c = g - i * chunks_per_line;
         const long long t = blockIdx.x + i * G;
-        mbar_arrive_expect_tx(&full[b], kStgChunkWords * 4u);
-        bulk_g2s(cbuf + b * kStgChunkWords, a.r.sched + t * a.sched_words + c * kStgChunkWords,
-                 kStgChunkWords * 4u, &full[b]);
+        mbar_arrive_expect_tx(&full[b], (uint32_t)CW * 4u);
+        bulk_g2s(cbuf + b * CWS, a.r.sched + t * a.sched_words + c * CW, (uint32_t)CW * 4u, &full[b]);
     };
     if (tid == 0)
-        for (long long g = 0; g < kStgBufs && g < total_chunks; ++g) issue_chunk(g);
+        for (long long g = 0; g < NB && g < total_chunks; ++g) issue_chunk(g);
     pdl_wait();
     stamp(tr, 1);
     if (tid == 0) {
@@ -1023,12 +1026,11 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
     }
     pdl_launch_dependents();
     const int lane = tid & 31, warp = tid >> 5;
-    const int wsel = lane / a.r.epw;
-    const int sh = a.r.E * (lane - wsel * a.r.epw);
-    const uint32_t mask = (1u << a.r.E) - 1u, tmask = (1u << a.r.logL) - 1u;
+    const SchedDec dec(DENSE ? 1 : 0, E, a.r.epw, w64, lane);
+    const uint32_t tmask = (1u << a.r.logL) - 1u;
     const int logL = a.r.logL;
     constexpr int MPC = 4;               // m-steps per chunk: 64 rounds = 4 x 16 warps
-    constexpr int CPL = EPT / MPC;       // chunks per line (host: w64 == 16, so 64 rounds/chunk)
+    constexpr int CPL = EPT / MPC;       // chunks per line
     for (long long i = 0; i < my_lines; ++i) {
         const long long t = blockIdx.x + i * G;
         const long long j0 = 2 * i, j1 = 2 * i + 1;
@@ -1042,14 +1044,13 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
 #pragma unroll
         for (int c = 0; c < CPL; ++c) {
             const long long g = i * CPL + c;
-            const int b = (int)(g % kStgBufs);
-            mbar_wait(&full[b], (uint32_t)((g / kStgBufs) & 1));
-            const uint2* cb = reinterpret_cast<const uint2*>(cbuf + b * kStgChunkWords);
+            const int b = (int)(g % NB);
+            mbar_wait(&full[b], (uint32_t)((g / NB) & 1));
+            const uint32_t* cb = cbuf + b * CWS;
 #pragma unroll
             for (int mm = 0; mm < MPC; ++mm) {
                 const int m = c * MPC + mm;
-                const uint2 wd = cb[(warp + kW * mm) * w64 + wsel];
-                const uint32_t e = (uint32_t)((((uint64_t)wd.y << 32) | wd.x) >> sh) & mask;
+                const uint32_t e = dec.get<true>(cb, warp + kW * mm);
                 const int s = (int)((e >> logL) << 5) + lane;
                 v[m] = smem[((s >> lh) ? o1 : o0) + (s & hmask)];
                 const int tt = (int)(e & tmask);
@@ -1058,9 +1059,9 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
                 else ta[m >> 1] = ad;
             }
             mbar_arrive(&empty[b]);
-            if (tid == 0 && g + kStgBufs < total_chunks) {
-                mbar_wait(&empty[b], (uint32_t)((g / kStgBufs) & 1));   // all 512 consumed chunk g
-                issue_chunk(g + kStgBufs);
+            if (tid == 0 && g + NB < total_chunks) {
+                mbar_wait(&empty[b], (uint32_t)((g / NB) & 1));   // all 512 consumed chunk g
+                issue_chunk(g + NB);
             }
         }
         __syncthreads();
@@ -1950,7 +1951,8 @@ size_t tma_smem(const HostPlan& P, int f) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
     if (rp.split && rp.split_stg)
-        return (size_t)3 * (g.L / 2) * 4 + (size_t)kStgBufs * kStgChunkWords * 4 + (3 + 2 * kStgBufs) * 8;
+        return g.dense ? (size_t)3 * (g.L / 2) * 4 + (size_t)5 * kStgDenseWords * 4 + (3 + 2 * 5) * 8
+                       : (size_t)3 * (g.L / 2) * 4 + (size_t)4 * kStgChunkWords * 4 + (3 + 2 * 4) * 8;
     if (rp.split) return (size_t)3 * (g.L / 2) * 4 + 3 * 8;
     const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * g.wpl * 4);
     return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
@@ -1994,7 +1996,8 @@ template <int EPT>
 const void* tma_kernel_ptr(bool cross, bool sg, bool split = false, bool dense = false, bool keep = true,
                            bool stg = false) {
     if constexpr (EPT == 32 || EPT == 64) {
-        if (split && stg) return (const void*)row_pass_split_stg_kernel<EPT>;
+        if (split && stg) return dense ? (const void*)row_pass_split_stg_kernel<EPT, true>
+                                       : (const void*)row_pass_split_stg_kernel<EPT, false>;
     }
     if (split) return split_kernel_ptr<EPT>(dense, keep);
     if (sg) return cross ? (const void*)row_pass_tma_kernel<EPT, true, true>
@@ -2012,6 +2015,7 @@ cudaError_t set_tma_smem(bool cross, size_t smem) {
     }
     if constexpr (EPT == 32 || EPT == 64) {
         if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, false, false, true), smem);
+        if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, true, false, true), smem);
     }
     return e;
 }
@@ -2404,8 +2408,11 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const bool cx = rp.out.cross != 0;
         const bool sg = rp.sg != 0;
         if (rp.split && rp.split_stg) {
-            if (rp.ept == 32) return launch(row_pass_split_stg_kernel<32>, grid, block, smem, s, pdl, ta);
-            if (rp.ept == 64) return launch(row_pass_split_stg_kernel<64>, grid, block, smem, s, pdl, ta);
+            const bool dn = g.dense != 0;
+            if (rp.ept == 32) return dn ? launch(row_pass_split_stg_kernel<32, true>, grid, block, smem, s, pdl, ta)
+                                        : launch(row_pass_split_stg_kernel<32, false>, grid, block, smem, s, pdl, ta);
+            if (rp.ept == 64) return dn ? launch(row_pass_split_stg_kernel<64, true>, grid, block, smem, s, pdl, ta)
+                                        : launch(row_pass_split_stg_kernel<64, false>, grid, block, smem, s, pdl, ta);
             return cudaErrorInvalidValue;
         }
         if (rp.split) {

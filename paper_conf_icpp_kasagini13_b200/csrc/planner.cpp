@@ -811,9 +811,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.E = 2 * g.logL - 5;
         g.epw = 64 / g.E;
         g.w64 = (kW + g.epw - 1) / g.epw;
-        // dense at L = 16384 (SG slots); L = 32768 lines (half-line ring) keep W64, whose
-        // merged loads measured faster there (profiles/r01_split_variants_s5.log)
-        g.dense = dense_phases && (g.logL == 14 || (opt && opt->sched_format == 2)) ? 1 : 0;
+        // dense for L >= 16384: the schedule-from-global slots (L = 16384) and the half-line
+        // ring's staged chunks (L = 32768: five 6.25 KiB chunks in flight instead of four 8 KiB)
+        g.dense = dense_phases && (g.logL >= 14 || (opt && opt->sched_format == 2)) ? 1 : 0;
         g.wpl = (int64_t)(g.L / kW) * (g.dense ? g.E : g.w64 * 2);
         g.words = g.lines * g.wpl;
     }
@@ -1028,7 +1028,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
                 // s512: the W64 schedule streamed through shared-memory chunks by TMA
                 // (needs 64-bit words holding 2 entries: w64 = 16)
                 const int64_t ept512 = (int64_t)rp.h * g.L / 512;
-                if (v == "s512" && g.w64 == 16 && !g.dense && (ept512 == 32 || ept512 == 64)) {
+                if (v == "s512" && (g.dense || g.w64 == 16) && (ept512 == 32 || ept512 == 64)) {
                     rp.split_stg = 1;
                     rp.threads = 512;
                     rp.ept = (int32_t)ept512;

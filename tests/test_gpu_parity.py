@@ -455,12 +455,15 @@ def test_half_line_ring_staged_schedule(P, k, log2c, fam, monkeypatch):
     n = 1 << k
     p = W.make_perm(fam, n, seed=k + log2c)
     a = W.make_data(n)
-    with P.Plan(p, passes=5, no_tma=-2, direct=-1, log2c=log2c, sched_format=-1) as plan:
-        d = plan.describe()
-        long_lines = [rp for rp in d["row_passes"] if rp["L"] >= 16384]
-        assert long_lines and all(rp["threads"] == 512 for rp in long_lines)
-        da = dev(a)
-        db = torch.full_like(da, -1)
-        plan.apply(da, db)
-        torch.cuda.synchronize()
-        assert np.array_equal(host_words(db), OA.apply_ref(p, a))
+    ref = OA.apply_ref(p, a)
+    for fmt in (-1, 0):           # W64 chunks (4 x 8 KiB) and dense chunks (5 x 64*E words)
+        with P.Plan(p, passes=5, no_tma=-2, direct=-1, log2c=log2c, sched_format=fmt) as plan:
+            d = plan.describe()
+            long_lines = [rp for rp in d["row_passes"] if rp["L"] >= 16384]
+            assert long_lines and all(rp["threads"] == 512 for rp in long_lines)
+            assert all(rp["dense"] == (fmt == 0) for rp in long_lines)
+            da = dev(a)
+            db = torch.full_like(da, -1)
+            plan.apply(da, db)
+            torch.cuda.synchronize()
+            assert np.array_equal(host_words(db), ref), fmt
