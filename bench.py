@@ -522,7 +522,7 @@ def main():
     desc = plans[sched_fams[0]].describe()
     sbpe = sched_bytes_per_elt(info, desc)
     if info["direct"]:
-        kinds = ["D-designated (direct)"]
+        kinds = ["S-designated on P^-1 (direct)" if info["direct"] == 1 else "D-designated (direct)"]
         alg = [2 * n * 4 + n * 4]
     elif info["kernels_per_apply"] == 1 and info["passes"] == 3:
         kinds = ["fused R1+R2+R3"]

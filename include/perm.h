@@ -78,9 +78,12 @@ typedef struct {
                             memory (the default wherever a line + its schedule exceed a slot:
                             L >= 16384, n >= 2^27) */
     int32_t direct;      /* low-distribution shortcut (for P with
-                            D_w(P) <= 2n/w, e.g. identical and shuffle, the D-designated kernel
+                            D_w(P) <= 2n/w, e.g. identical and shuffle, a one-kernel copy
                             is coalesced and faster): 0 = auto (on when D_w(P) <= 2n/32),
-                            -1 = never (always run the scheduled passes), 1 = always */
+                            -1 = never (always run the scheduled passes), 1 = always, with
+                            the S-designated kernel b[i] = a[q[i]], q = P^-1 (L373; writes
+                            whole sectors, reads D_w(P^-1) = D_w(P) groups), 2 = always,
+                            with the D-designated kernel b[p[i]] = a[i] (L365) */
     int32_t log2c;       /* view r x c with c = 2^log2c (the view "is not
                             restricted to a square matrix"); 0 = c = 2^ceil(k/2) */
     int32_t sched_format; /* TLC layout entry format: 0 = full (source row << log2(tile) |
@@ -114,7 +117,8 @@ typedef struct {
     int64_t shard_elems;         /* n / world */
     int64_t block_elems;         /* n / world^2: one all-to-all block */
     int64_t distribution;        /* D_w(P), w = 32 (L389-L401): address groups the warps write */
-    int32_t direct;              /* 1: perm_apply runs the D-designated kernel (low D_w) */
+    int32_t direct;              /* 1: perm_apply runs the S-designated kernel on q = P^-1,
+                                    2: the D-designated kernel on p (low D_w); 0: passes */
     int32_t gpu_planner;         /* 1: the colourings ran on the GPU (gplan.cu), 0: on the host */
 } perm_plan_info;
 

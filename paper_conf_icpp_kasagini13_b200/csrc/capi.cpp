@@ -35,7 +35,7 @@ struct perm_plan {
     unsigned long long* d_trace = nullptr;
     int64_t trace_stride = 0;          // CTAs per pass slot
     unsigned long long* d_sync = nullptr;   // fused 3-pass grid-barrier counters
-    int32_t* d_p = nullptr;                 // direct (D-designated) shortcut
+    int32_t* d_p = nullptr;                 // low-distribution shortcut: q = P^-1 (or p)
     alignas(64) CUtensorMap tlc_maps[3];   // TLC layout: TMA tensor maps of X1, X2
 };
 
@@ -472,8 +472,10 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
     int k = 0;   // index of the kernel being launched (for the error message)
     mark();
     if (plan->d_p) {
-        // low distribution (D_w(P) <= 2n/w, L699-L701): the D-designated kernel is coalesced
-        e = perm::launch_scatter(plan->d_p, in, out, P.n, 4, s);
+        // low distribution (D_w(P) <= 2n/w, L699-L701): one coalesced kernel; d_p holds
+        // q = P^-1 for the S-designated kernel (direct 1) or p for the D-designated (2)
+        e = P.direct == 2 ? perm::launch_scatter(plan->d_p, in, out, P.n, 4, s)
+                          : perm::launch_gather(plan->d_p, in, out, P.n, 4, s);
         mark();
     } else if (P.passes == 1) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};

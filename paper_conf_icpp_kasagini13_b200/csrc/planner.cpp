@@ -730,8 +730,21 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         P.distribution = dw;
         const int dopt = opt ? opt->direct : 0;
         if (dopt > 0 || (dopt == 0 && dw <= 2 * n / kW)) {
-            P.direct = 1;
-            P.p_copy.assign(p, p + n);
+            // D_w(P^-1) = D_w(P): both count the distinct (warp block of sources, address
+            // group of destinations) pairs, so the S-designated kernel b[i] = a[q[i]]
+            // (L373) reads as few groups as the D-designated one writes, and its writes
+            // are whole sectors (the scatter's partial-sector writes cost 21 vs 12 us for
+            // the shuffle at n = 2^22, profiles/bench_r01r.json s_designated_us).
+            // direct = 2 keeps the D-designated kernel (A/B).
+            P.direct = dopt == 2 ? 2 : 1;
+            P.p_copy.resize((size_t)n);
+            if (P.direct == 2) {
+                P.p_copy.assign(p, p + n);
+            } else {
+                int32_t* q = P.p_copy.data();
+#pragma omp parallel for schedule(static)
+                for (int64_t i = 0; i < n; ++i) q[p[i]] = (int32_t)i;
+            }
         }
     }
     P.n = n; P.eb = eb; P.k = k;

@@ -314,6 +314,13 @@ def test_distribution_and_direct_shortcut(lib, k):
             assert pl.info()["direct"] == 0
         with lib.Plan(p, device=False, direct=1) as pl:
             assert pl.info()["direct"] == 1
+        with lib.Plan(p, device=False, direct=2) as pl:
+            assert pl.info()["direct"] == 2
+        # the S-designated shortcut on q = P^-1 relies on D_w(P^-1) = D_w(P): both
+        # count the distinct (source warp block, destination group) pairs
+        q = np.empty_like(p)
+        q[p] = np.arange(n, dtype=p.dtype)
+        assert OD.distribution(q, 32) == dw, fam
     # identity and shuffle are the paper's low-distribution cases
     assert lib.Plan(W.identity(n), device=False).info()["direct"] == 1
     assert lib.Plan(W.make_perm("shuffle", n), device=False).info()["direct"] == 1

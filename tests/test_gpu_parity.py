@@ -303,13 +303,15 @@ def test_fp64_elements(P, k):
 @pytest.mark.parametrize("k", [10, 14, 16, 22])
 @pytest.mark.parametrize("eb", [4, 8])
 def test_direct_shortcut(P, k, eb):
-    # for D_w(P) <= 2n/w (identical, shuffle) the D-designated
-    # kernel is the faster choice; the plan takes it by default and stays bit-exact
+    # for D_w(P) <= 2n/w (identical, shuffle) one coalesced kernel
+    # is the faster choice; the plan takes it by default (S-designated on q = P^-1,
+    # direct 1; D-designated on p with direct 2) and stays bit-exact
     n = 1 << k
     a = W.make_data(n, eb)
     view = np.int32 if eb == 4 else np.int64
     for fam, direct, want in (("identity", 0, 1), ("shuffle", 0, 1), ("random", 0, 0),
-                              ("random", 1, 1), ("bitrev", 1, 1), ("identity", -1, 0)):
+                              ("random", 1, 1), ("bitrev", 1, 1), ("identity", -1, 0),
+                              ("shuffle", 2, 2), ("random", 2, 2)):
         p = W.make_perm(fam, n, seed=k)
         with P.Plan(p, elem_bytes=eb, direct=direct) as plan:
             info = plan.info()
