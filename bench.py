@@ -522,7 +522,8 @@ def main():
     desc = plans[sched_fams[0]].describe()
     sbpe = sched_bytes_per_elt(info, desc)
     if info["direct"]:
-        kinds = ["S-designated on P^-1 (direct)" if info["direct"] == 1 else "D-designated (direct)"]
+        kinds = [{1: "S-designated on P^-1 (direct)", 2: "D-designated (direct)",
+                  3: "block gather (direct)"}[info["direct"]]]
         alg = [2 * n * 4 + n * 4]
     elif info["kernels_per_apply"] == 1 and info["passes"] == 3:
         kinds = ["fused R1+R2+R3"]

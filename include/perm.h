@@ -83,7 +83,10 @@ typedef struct {
                             -1 = never (always run the scheduled passes), 1 = always, with
                             the S-designated kernel b[i] = a[q[i]], q = P^-1 (L373; writes
                             whole sectors, reads D_w(P^-1) = D_w(P) groups), 2 = always,
-                            with the D-designated kernel b[p[i]] = a[i] (L365) */
+                            with the D-designated kernel b[p[i]] = a[i] (L365). Auto (0) runs
+                            a block gather instead (info.direct = 3) when P moves whole aligned
+                            32-word blocks in order (p[32j + x] = 32g + x: the identical
+                            permutation, block permutations), reading n/32 block indices */
     int32_t log2c;       /* view r x c with c = 2^log2c (the view "is not
                             restricted to a square matrix"); 0 = c = 2^ceil(k/2) */
     int32_t sched_format; /* TLC layout entry format: 0 = full (source row << log2(tile) |
@@ -118,7 +121,8 @@ typedef struct {
     int64_t block_elems;         /* n / world^2: one all-to-all block */
     int64_t distribution;        /* D_w(P), w = 32 (L389-L401): address groups the warps write */
     int32_t direct;              /* 1: perm_apply runs the S-designated kernel on q = P^-1,
-                                    2: the D-designated kernel on p (low D_w); 0: passes */
+                                    2: the D-designated kernel on p (low D_w), 3: the block
+                                    gather on P^-1's block map; 0: the scheduled passes */
     int32_t gpu_planner;         /* 1: the colourings ran on the GPU (gplan.cu), 0: on the host */
 } perm_plan_info;
 

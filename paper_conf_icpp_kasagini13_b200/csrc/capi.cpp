@@ -474,8 +474,10 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
     if (plan->d_p) {
         // low distribution (D_w(P) <= 2n/w, L699-L701): one coalesced kernel; d_p holds
         // q = P^-1 for the S-designated kernel (direct 1) or p for the D-designated (2)
-        e = P.direct == 2 ? perm::launch_scatter(plan->d_p, in, out, P.n, 4, s)
-                          : perm::launch_gather(plan->d_p, in, out, P.n, 4, s);
+        // or, for whole aligned blocks moved in order (direct 3), qb = block map of P^-1
+        e = P.direct == 3   ? perm::launch_block_gather(plan->d_p, in, out, P.n, s)
+            : P.direct == 2 ? perm::launch_scatter(plan->d_p, in, out, P.n, 4, s)
+                            : perm::launch_gather(plan->d_p, in, out, P.n, 4, s);
         mark();
     } else if (P.passes == 1) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};

@@ -1883,6 +1883,19 @@ __global__ void __launch_bounds__(256) gather64_kernel(const int32_t* __restrict
     }
 }
 
+// Block gather for P that moves whole aligned 32-word blocks in order (D_w(P) = n/w with
+// p[32j + x] = 32 g + x): qb[g] = j, one index per 32 words; each thread moves 16 bytes,
+// 8 consecutive threads one 128-byte block (full-line reads and writes).
+__global__ void __launch_bounds__(256) block_gather_kernel(const int32_t* __restrict__ qb,
+                                                           const uint32_t* __restrict__ a,
+                                                           uint32_t* __restrict__ b, long long nv) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nv;
+         v += (long long)gridDim.x * blockDim.x) {
+        const long long src = (long long)__ldg(qb + (v >> 3)) * 8 + (v & 7);
+        st_v4(b + 4 * v, ld_nc_v4(a + 4 * src));
+    }
+}
+
 __global__ void __launch_bounds__(256) copy_kernel(const uint32_t* __restrict__ a,
                                                    uint32_t* __restrict__ b, long long nv) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nv;
@@ -2537,6 +2550,13 @@ cudaError_t launch_gather(const int32_t* q, const void* a, void* b, int64_t n, i
         return launch(gather64_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, q,
                       static_cast<const uint2*>(a), static_cast<uint2*>(b), nv);
     return launch(gather_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, q,
+                  static_cast<const uint32_t*>(a), static_cast<uint32_t*>(b), nv);
+}
+
+cudaError_t launch_block_gather(const int32_t* qb, const void* a, void* b, int64_t n_words,
+                                cudaStream_t s) {
+    const long long nv = n_words / 4;
+    return launch(block_gather_kernel, dim3(stream_grid(nv)), dim3(256), 0, s, false, qb,
                   static_cast<const uint32_t*>(a), static_cast<uint32_t*>(b), nv);
 }
 

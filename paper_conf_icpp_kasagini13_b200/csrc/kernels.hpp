@@ -51,6 +51,8 @@ cudaError_t launch_scatter(const int32_t* p, const void* a, void* b, int64_t n, 
                            cudaStream_t s);
 cudaError_t launch_gather(const int32_t* q, const void* a, void* b, int64_t n, int eb,
                           cudaStream_t s);
+cudaError_t launch_block_gather(const int32_t* qb, const void* a, void* b, int64_t n_words,
+                                cudaStream_t s);
 cudaError_t launch_copy(const uint32_t* a, uint32_t* b, int64_t n, cudaStream_t s);
 
 }  // namespace perm

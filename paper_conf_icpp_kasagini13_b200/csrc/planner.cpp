@@ -736,9 +736,24 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             // are whole sectors (the scatter's partial-sector writes cost 21 vs 12 us for
             // the shuffle at n = 2^22, profiles/bench_r01r.json s_designated_us).
             // direct = 2 keeps the D-designated kernel (A/B).
-            P.direct = dopt == 2 ? 2 : 1;
-            P.p_copy.resize((size_t)n);
-            if (P.direct == 2) {
+            // direct = 3 when P moves whole aligned 32-word blocks in order (identity,
+            // block permutations): only the n/32-entry block map of P^-1 is read
+            bool blocks = dopt <= 0;
+            if (blocks) {
+                int bad = 0;
+#pragma omp parallel for schedule(static) reduction(| : bad)
+                for (int64_t i = 0; i < n; ++i)
+                    bad |= ((p[i] & (kW - 1)) != (i & (kW - 1))) |
+                           ((p[i] - (i & (kW - 1))) != p[i & ~int64_t(kW - 1)]);
+                blocks = !bad;
+            }
+            P.direct = blocks ? 3 : dopt == 2 ? 2 : 1;
+            P.p_copy.resize((size_t)(blocks ? n / kW : n));
+            if (P.direct == 3) {
+                int32_t* qb = P.p_copy.data();
+#pragma omp parallel for schedule(static)
+                for (int64_t j = 0; j < n / kW; ++j) qb[p[j * kW] / kW] = (int32_t)j;
+            } else if (P.direct == 2) {
                 P.p_copy.assign(p, p + n);
             } else {
                 int32_t* q = P.p_copy.data();

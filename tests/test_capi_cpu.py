@@ -308,7 +308,11 @@ def test_distribution_and_direct_shortcut(lib, k):
             with lib.Plan(p, elem_bytes=eb, device=False) as pl:
                 inf = pl.info()
                 assert inf["distribution"] == want_dw, (fam, eb)
-                assert inf["direct"] == int(want_dw <= 2 * pp.size // 32), (fam, eb)
+                m = pp.size // 32
+                blk = pp.reshape(m, 32)
+                in_order = bool(np.all(blk == blk[:, :1] + np.arange(32)) and np.all(blk[:, 0] % 32 == 0))
+                low = want_dw <= 2 * pp.size // 32
+                assert inf["direct"] == (3 if low and in_order else int(low)), (fam, eb)
                 assert pl.describe()["direct"] == inf["direct"]
         with lib.Plan(p, device=False, direct=-1) as pl:
             assert pl.info()["direct"] == 0
@@ -322,7 +326,11 @@ def test_distribution_and_direct_shortcut(lib, k):
         q[p] = np.arange(n, dtype=p.dtype)
         assert OD.distribution(q, 32) == dw, fam
     # identity and shuffle are the paper's low-distribution cases
-    assert lib.Plan(W.identity(n), device=False).info()["direct"] == 1
+    assert lib.Plan(W.identity(n), device=False).info()["direct"] == 3
+    blocks = np.random.default_rng(k).permutation(n // 32).astype(np.int32)
+    pb = (blocks[:, None] * 32 + np.arange(32, dtype=np.int32)).reshape(-1)
+    assert lib.Plan(pb, device=False).info()["direct"] == 3
+    assert lib.Plan(W.identity(n), device=False, direct=1).info()["direct"] == 1
     assert lib.Plan(W.make_perm("shuffle", n), device=False).info()["direct"] == 1
     assert lib.Plan(W.make_perm("bitrev", n), device=False).info()["direct"] == 0
     if k >= 16:   # sharded plans never take the single-device shortcut

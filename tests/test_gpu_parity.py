@@ -309,10 +309,15 @@ def test_direct_shortcut(P, k, eb):
     n = 1 << k
     a = W.make_data(n, eb)
     view = np.int32 if eb == 4 else np.int64
-    for fam, direct, want in (("identity", 0, 1), ("shuffle", 0, 1), ("random", 0, 0),
+    for fam, direct, want in (("identity", 0, 3), ("shuffle", 0, 1), ("random", 0, 0),
                               ("random", 1, 1), ("bitrev", 1, 1), ("identity", -1, 0),
-                              ("shuffle", 2, 2), ("random", 2, 2)):
-        p = W.make_perm(fam, n, seed=k)
+                              ("shuffle", 2, 2), ("random", 2, 2), ("identity", 1, 1),
+                              ("blocks", 0, 3)):
+        if fam == "blocks":   # whole aligned 32-word blocks moved in order (direct 3)
+            blocks = np.random.default_rng(k).permutation(n // 32).astype(np.int32)
+            p = (blocks[:, None] * 32 + np.arange(32, dtype=np.int32)).reshape(-1)
+        else:
+            p = W.make_perm(fam, n, seed=k)
         with P.Plan(p, elem_bytes=eb, direct=direct) as plan:
             info = plan.info()
             assert info["direct"] == want, (fam, direct)
