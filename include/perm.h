@@ -44,7 +44,7 @@ enum perm_status {
                                 elements), or elem_bytes not 4 or 8 */
     PERM_ENOMEM       = -4,  /* host or device allocation failed */
     PERM_ECUDA        = -5,  /* a CUDA runtime call failed (message has the CUDA error) */
-    PERM_ENCCL        = -6,  /* reserved for the row-sharded multi-GPU path */
+    PERM_ENCCL        = -6,  /* NCCL missing or an NCCL call failed (row-sharded path) */
     PERM_ENODEVICE    = -7   /* the call needs a device but the plan is host-only / no GPU */
 };
 
@@ -108,7 +108,8 @@ typedef struct {
     int64_t sched_bytes;         /* device bytes of the three packed bank schedules */
     int64_t scratch_bytes;       /* device bytes of intermediate buffers */
     int32_t elem_bytes;
-    int32_t passes;              /* 1, 3 or 5 */
+    int32_t passes;              /* 1, 3 or 5; 0 for a low-distribution shortcut plan
+                                    (direct != 0: one kernel, no schedule) */
     int32_t kernels_per_apply;   /* kernel launches one perm_apply issues */
     int32_t entry_bits[3];       /* bits per schedule entry, phase 1..3 (2*log2(L) - 5) */
     int32_t h[3];                /* lines per CTA of the three row passes */
@@ -216,15 +217,47 @@ int perm_plan_run_pass(const perm_plan* plan, int32_t pass, const void* in, void
 /* rank g of `world` GPUs owns rows [g*r/world, (g+1)*r/world) of the
  * r x c view, i.e. the contiguous shard a[g*n/world : (g+1)*n/world] (and the
  * same shard of b). Phases 1 and 3 (row-wise, L537-L539) are local; the
- * column-wise phase (Lemma 8: transpose, row-wise, transpose) becomes two
- * all-to-all exchanges. p is the FULL permutation (every rank passes the same p;
- * every rank colours it identically and keeps its own lines' schedules).
+ * column-wise phase (Lemma 8 L533: transpose, row-wise, transpose) becomes two
+ * uniform, P-independent all-to-all exchanges of n/world^2-element blocks over
+ * NCCL (NVLink / NVSwitch). p is the FULL permutation (every rank passes the
+ * same p; every rank colours it identically and keeps its own lines' schedules).
  * world must be a power of two with r/world >= 32 and c/world >= 32. */
+
+#define PERM_NCCL_UID_BYTES 128
+
+/* Writes a fresh ncclUniqueId (PERM_NCCL_UID_BYTES bytes, host memory) to uid_out.
+ * Rank 0 calls it and broadcasts the bytes to the other ranks out of band (e.g.
+ * torch.distributed). NCCL is loaded at run time (the process's libnccl.so.2);
+ * PERM_ENCCL when it cannot be loaded. */
+int perm_nccl_unique_id(void* uid_out);
+
+/* Sharded plan of rank `rank` on the CURRENT device. nccl_uid (PERM_NCCL_UID_BYTES
+ * bytes, the same on every rank; borrowed for the call) != NULL: the call also
+ * joins an NCCL communicator of `world` ranks (collective: every rank must call
+ * it concurrently; it blocks until all have joined) and allocates the plan's two
+ * exchange shards (2 * n/world * elem_bytes device bytes), so perm_apply_sharded
+ * works. nccl_uid == NULL: no communicator; only perm_sharded_step is available
+ * (the caller runs the exchanges, e.g. virtual ranks on one GPU).
+ * NULL on error: PERM_EINVAL / PERM_EUNSUPPORTED as perm_plan_create, or
+ * PERM_ENCCL when NCCL cannot be loaded or the communicator fails. */
 perm_plan* perm_plan_create_sharded(const int32_t* p, int64_t n, int32_t elem_bytes,
-                                    int32_t world, int32_t rank, const perm_plan_options* opt);
+                                    int32_t world, int32_t rank, const void* nccl_uid);
+perm_plan* perm_plan_create_sharded_ex(const int32_t* p, int64_t n, int32_t elem_bytes,
+                                       int32_t world, int32_t rank, const void* nccl_uid,
+                                       const perm_plan_options* opt);
+/* Planner only (no CUDA, no NCCL): for perm_plan_export / perm_plan_get_info. */
 perm_plan* perm_plan_create_sharded_host(const int32_t* p, int64_t n, int32_t elem_bytes,
                                          int32_t world, int32_t rank,
                                          const perm_plan_options* opt);
+
+/* The whole sharded apply on this rank: b_shard = rows [rank*r/world, ...) of b,
+ * b[P(i)] = a[i]. a_shard, b_shard: DEVICE buffers of n/world elements on the
+ * plan's device, 16-byte aligned, not overlapping. Stream-ordered, no host sync:
+ *   step 0 -> all-to-all -> step 1 -> all-to-all -> step 2
+ * with the plan's own exchange shards; every rank must call it (NCCL collective).
+ * PERM_ENCCL if the plan has no communicator; at most one in flight per plan. */
+int perm_apply_sharded(const perm_plan* plan, const void* a_shard, void* b_shard,
+                       perm_stream_t stream);
 
 /* One local step of a sharded apply (device buffers, stream-ordered):
  *   step 0: in = a shard (n/world elems)  -> out = send buffer (n/world)  [R1, T]
@@ -232,9 +265,15 @@ perm_plan* perm_plan_create_sharded_host(const int32_t* p, int64_t n, int32_t el
  *   step 2: in = recv buffer              -> out = b shard                [R3]
  * Between steps 0->1 and 1->2 the caller performs the all-to-all: with
  * B = n/world^2, for every pair (g, q): recv_q[g*B : (g+1)*B] = send_g[q*B : (q+1)*B]
- * (NCCL all_to_all over NVLink, or device copies for ranks sharing one GPU). */
+ * (perm_sharded_exchange, or device copies for ranks sharing one GPU). */
 int perm_sharded_step(const perm_plan* plan, int32_t step, const void* in, void* out,
                       perm_stream_t stream);
+
+/* The all-to-all of the step contract above on the plan's NCCL communicator
+ * (grouped ncclSend / ncclRecv, one pair per peer), stream-ordered. send, recv:
+ * DEVICE buffers of n/world elements. PERM_ENCCL without a communicator. */
+int perm_sharded_exchange(const perm_plan* plan, const void* send, void* recv,
+                          perm_stream_t stream);
 
 /* ------------------------------------------------------- comparators */
 

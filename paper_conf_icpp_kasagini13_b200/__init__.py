@@ -9,7 +9,7 @@ The binding is loaded on first use (so `python -m ....build` can run before the
 library exists); using any name below without a built libperm.so raises.
 """
 _EXPORTS = ("Plan", "PermError", "scatter_baseline", "gather_baseline", "copy_kernel",
-            "last_error", "version", "LIB_PATH")
+            "last_error", "version", "LIB_PATH", "nccl_unique_id")
 
 __all__ = list(_EXPORTS)
 

@@ -73,8 +73,11 @@ def _sig(name, res, *args):
 _plan_create = _sig("perm_plan_create", _vp, _vp, _i64, _i32)
 _plan_create_ex = _sig("perm_plan_create_ex", _vp, _vp, _i64, _i32, ctypes.POINTER(PlanOptions))
 _plan_create_host = _sig("perm_plan_create_host", _vp, _vp, _i64, _i32, ctypes.POINTER(PlanOptions))
-_plan_create_sharded = _sig("perm_plan_create_sharded", _vp, _vp, _i64, _i32, _i32, _i32,
+_plan_create_sharded = _sig("perm_plan_create_sharded_ex", _vp, _vp, _i64, _i32, _i32, _i32, _vp,
                             ctypes.POINTER(PlanOptions))
+_nccl_uid = _sig("perm_nccl_unique_id", ctypes.c_int, _vp)
+_apply_sharded = _sig("perm_apply_sharded", ctypes.c_int, _vp, _vp, _vp, _vp)
+_sharded_exchange = _sig("perm_sharded_exchange", ctypes.c_int, _vp, _vp, _vp, _vp)
 _plan_create_sharded_host = _sig("perm_plan_create_sharded_host", _vp, _vp, _i64, _i32, _i32, _i32,
                                  ctypes.POINTER(PlanOptions))
 _sharded_step = _sig("perm_sharded_step", ctypes.c_int, _vp, _i32, _vp, _vp, _vp)
@@ -128,6 +131,28 @@ def _ptr(x) -> int:
     return int(x)
 
 
+def _check_buf(x, nbytes: int, what: str):
+    """Device buffers handed to libperm: CUDA, contiguous, exactly nbytes (torch tensors);
+    raw integers are passed through as pointers (the caller vouches for them)."""
+    if not hasattr(x, "data_ptr"):
+        return
+    if not getattr(x, "is_cuda", False):
+        raise PermError(-1, f"{what} must be a CUDA tensor")
+    if not x.is_contiguous():
+        raise PermError(-1, f"{what} must be contiguous")
+    got = x.numel() * x.element_size()
+    if got != nbytes:
+        raise PermError(-1, f"{what} holds {got} bytes, the plan needs {nbytes}")
+
+
+def nccl_unique_id() -> bytes:
+    """A fresh ncclUniqueId (128 bytes) for perm_plan_create_sharded (rank 0 makes it,
+    every rank passes the same bytes)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(_nccl_uid(buf))
+    return buf.raw
+
+
 def _as_int32_host(p) -> np.ndarray:
     if hasattr(p, "detach"):       # torch tensor
         p = p.detach().cpu().numpy()
@@ -140,16 +165,27 @@ class Plan:
     def __init__(self, p, elem_bytes: int = 4, passes: int = 0, h=(0, 0, 0),
                  device: bool = True, layout: int = 0, stages: int = 0, fuse: int = 0,
                  world: int = 0, rank: int = 0, no_tma: int = 0, direct: int = 0, log2c: int = 0,
-                 sched_format: int = 0, gpu_planner: int = 0):
-        """world > 0: row-sharded plan of rank `rank` (see perm_plan_create_sharded)."""
+                 sched_format: int = 0, gpu_planner: int = 0, nccl_uid: bytes | None = None):
+        """world > 0: row-sharded plan of rank `rank` (see perm_plan_create_sharded);
+        nccl_uid (128 bytes, the same on every rank) also joins the plan's NCCL
+        communicator, so apply_sharded() runs the whole sharded apply in libperm."""
         p = _as_int32_host(p)
         self.n = int(p.size)
         self.elem_bytes = elem_bytes
         opt = PlanOptions(passes, h[0], h[1], h[2], layout, stages, fuse, no_tma, direct, log2c,
                           sched_format, gpu_planner)
         if world > 0:
-            fn = _plan_create_sharded if device else _plan_create_sharded_host
-            handle = fn(p.ctypes.data, self.n, elem_bytes, world, rank, ctypes.byref(opt))
+            if device:
+                uid = None
+                if nccl_uid is not None:
+                    if len(nccl_uid) != 128:
+                        raise ValueError("nccl_uid must be 128 bytes")
+                    uid = ctypes.create_string_buffer(bytes(nccl_uid), 128)
+                handle = _plan_create_sharded(p.ctypes.data, self.n, elem_bytes, world, rank, uid,
+                                              ctypes.byref(opt))
+            else:
+                handle = _plan_create_sharded_host(p.ctypes.data, self.n, elem_bytes, world, rank,
+                                                   ctypes.byref(opt))
         elif device:
             handle = _plan_create_ex(p.ctypes.data, self.n, elem_bytes, ctypes.byref(opt))
         else:
@@ -158,6 +194,9 @@ class Plan:
             _raise()
         self._h = handle
         self.on_device = device
+        self.world = world if world > 0 else 1
+        self.nbytes = self.n * elem_bytes
+        self.shard_bytes = self.nbytes // self.world
 
     # -- lifecycle
     def close(self):
@@ -207,17 +246,41 @@ class Plan:
 
     # -- hot path
     def apply(self, a, b, stream=None):
-        """b[p[i]] = a[i]; a, b CUDA tensors of n elements (4-byte dtype), stream-ordered."""
+        """b[p[i]] = a[i]; a, b CUDA tensors of n * elem_bytes bytes, stream-ordered."""
+        _check_buf(a, self.nbytes, "a")
+        _check_buf(b, self.nbytes, "b")
         _check(_apply(self._h, _ptr(a), _ptr(b), _stream_handle(stream)))
         return b
 
+    def apply_sharded(self, a_shard, b_shard, stream=None):
+        """This rank's b shard of a sharded plan created with nccl_uid (NCCL collective:
+        every rank calls it); a_shard / b_shard: n/world elements on the plan's device."""
+        _check_buf(a_shard, self.shard_bytes, "a_shard")
+        _check_buf(b_shard, self.shard_bytes, "b_shard")
+        _check(_apply_sharded(self._h, _ptr(a_shard), _ptr(b_shard), _stream_handle(stream)))
+        return b_shard
+
+    def sharded_exchange(self, send, recv, stream=None):
+        """The plan communicator's all-to-all of the perm_sharded_step block contract."""
+        _check_buf(send, self.shard_bytes, "send")
+        _check_buf(recv, self.shard_bytes, "recv")
+        _check(_sharded_exchange(self._h, _ptr(send), _ptr(recv), _stream_handle(stream)))
+        return recv
+
     def apply_host(self, a_host, b_host, stream=None):
         """End-to-end: host a -> device -> apply -> host b (synchronises the stream)."""
+        for x, what in ((a_host, "a_host"), (b_host, "b_host")):
+            nb = x.nbytes if isinstance(x, np.ndarray) else (
+                x.numel() * x.element_size() if hasattr(x, "numel") else self.nbytes)
+            if nb != self.nbytes or getattr(x, "is_cuda", False):
+                raise PermError(-1, f"{what}: host buffer of {self.nbytes} bytes expected")
         _check(_apply_host(self._h, _ptr(a_host), _ptr(b_host), _stream_handle(stream)))
         return b_host
 
     def sharded_step(self, step: int, inp, out, stream=None):
         """One local step of a row-sharded apply (see include/perm.h perm_sharded_step)."""
+        _check_buf(inp, self.shard_bytes, "in")
+        _check_buf(out, self.shard_bytes, "out")
         _check(_sharded_step(self._h, step, _ptr(inp), _ptr(out), _stream_handle(stream)))
         return out
 

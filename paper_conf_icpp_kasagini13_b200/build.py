@@ -12,8 +12,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(PKG, "csrc")
 ROOT = os.path.dirname(PKG)
 LIB = os.path.join(PKG, "libperm.so")
-SOURCES = ["planner.cpp", "capi.cpp", "kernels.cu", "gplan.cu"]
-HEADERS = ["plan.hpp", "kernels.hpp", "gplan.hpp"]
+SOURCES = ["planner.cpp", "capi.cpp", "nccl_dl.cpp", "kernels.cu", "gplan.cu"]
+HEADERS = ["plan.hpp", "kernels.hpp", "gplan.hpp", "nccl_dl.hpp"]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
@@ -41,7 +41,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     nvcc = os.environ.get("NVCC", "nvcc")
     cmd = [nvcc, *NVCC_FLAGS, *(["-Xptxas", "-v"] if verbose else []), "-o", LIB + ".tmp",
-           *[os.path.join(CSRC, s) for s in SOURCES], "-lgomp"]
+           *[os.path.join(CSRC, s) for s in SOURCES], "-lgomp", "-ldl"]
     res = subprocess.run(cmd, capture_output=True, text=True)
     if res.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + " ".join(cmd) + "\n" + res.stdout + res.stderr)

@@ -11,6 +11,7 @@
 
 #include "../../include/perm.h"
 #include "kernels.hpp"
+#include "nccl_dl.hpp"
 #include "plan.hpp"
 
 using perm::HostPlan;
@@ -37,6 +38,11 @@ struct perm_plan {
     unsigned long long* d_sync = nullptr;   // fused 3-pass grid-barrier counters
     int32_t* d_p = nullptr;                 // low-distribution shortcut: q = P^-1 (or p)
     alignas(64) CUtensorMap tlc_maps[3];   // TLC layout: TMA tensor maps of X1, X2
+    // row-sharded plans created with an NCCL unique id: the communicator of the
+    // column phase's two all-to-alls and the plan-owned send / receive shards
+    ncclComm_t comm = nullptr;
+    uint32_t* d_send = nullptr;
+    uint32_t* d_recv = nullptr;
 };
 
 namespace {
@@ -67,6 +73,13 @@ void free_device(perm_plan* pl) {
     cudaFree(pl->d_trace);
     cudaFree(pl->d_sync);
     cudaFree(pl->d_p);
+    cudaFree(pl->d_send);
+    cudaFree(pl->d_recv);
+    if (pl->comm) {
+        std::string err;
+        if (const perm::NcclApi* api = perm::nccl_api(err)) api->CommDestroy(pl->comm);
+        pl->comm = nullptr;
+    }
     for (int i = 0; i < pl->n_events; ++i) cudaEventDestroy(pl->ev[i]);
     pl->n_events = 0;
     if (cur >= 0) cudaSetDevice(cur);
@@ -95,7 +108,7 @@ int upload(perm_plan* pl) {
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemset");
         off += padded(wf);
     }
-    if (P.passes != 1) {
+    if (P.passes > 1) {
         const size_t bytes = (size_t)(P.r_l ? P.n / P.world : P.n) * P.eb;
         for (int i = 0; i < 2; ++i) {
             e = cudaMalloc(&pl->d_scratch[i], bytes);
@@ -168,6 +181,32 @@ perm_plan* create(const int32_t* p, int64_t n, int32_t eb, const perm_plan_optio
     return pl;
 }
 
+int nccl_fail(const perm::NcclApi* api, ncclResult_t r, const char* what) {
+    return fail(PERM_ENCCL, std::string(what) + ": " + (api ? api->GetErrorString(r) : "NCCL unavailable"));
+}
+
+// NCCL communicator + exchange buffers of a sharded device plan (collective over the ranks)
+int attach_comm(perm_plan* pl, const void* uid) {
+    std::string err;
+    const perm::NcclApi* api = perm::nccl_api(err);
+    if (!api) return fail(PERM_ENCCL, err);
+    const HostPlan& P = pl->host;
+    ncclUniqueId id;
+    std::memcpy(&id, uid, sizeof(id));
+    cudaError_t e = cudaSetDevice(pl->device);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+    const ncclResult_t r = api->CommInitRank(&pl->comm, P.world, id, P.rank);
+    if (r != ncclSuccess) {
+        pl->comm = nullptr;
+        return nccl_fail(api, r, "ncclCommInitRank");
+    }
+    const size_t bytes = (size_t)(P.n / P.world) * P.eb;
+    e = cudaMalloc(&pl->d_send, bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&pl->d_recv, bytes);
+    if (e != cudaSuccess) return fail(PERM_ENOMEM, std::string("cudaMalloc exchange buffers: ") + cudaGetErrorString(e));
+    return PERM_OK;
+}
+
 bool overlap(const void* a, const void* b, int64_t bytes) {
     const char* x = static_cast<const char*>(a);
     const char* y = static_cast<const char*>(b);
@@ -192,9 +231,70 @@ perm_plan* perm_plan_create_host(const int32_t* p, int64_t n, int32_t elem_bytes
     return create(p, n, elem_bytes, opt, false);
 }
 
+int perm_nccl_unique_id(void* uid_out) {
+    if (!uid_out) return fail(PERM_EINVAL, "null uid buffer");
+    std::string err;
+    const perm::NcclApi* api = perm::nccl_api(err);
+    if (!api) return fail(PERM_ENCCL, err);
+    ncclUniqueId id;
+    const ncclResult_t r = api->GetUniqueId(&id);
+    if (r != ncclSuccess) return nccl_fail(api, r, "ncclGetUniqueId");
+    std::memcpy(uid_out, &id, sizeof(id));
+    return PERM_OK;
+}
+
+perm_plan* perm_plan_create_sharded_ex(const int32_t* p, int64_t n, int32_t elem_bytes, int32_t world,
+                                       int32_t rank, const void* nccl_uid, const perm_plan_options* opt) {
+    if (world < 1) { fail(PERM_EINVAL, "world must be >= 1"); return nullptr; }
+    perm_plan* pl = create(p, n, elem_bytes, opt, true, world, rank);
+    if (!pl || !nccl_uid) return pl;
+    if (attach_comm(pl, nccl_uid) != PERM_OK) {
+        const int st = g_status;
+        const std::string msg = g_msg;
+        free_device(pl);
+        delete pl;
+        fail(st, msg);
+        return nullptr;
+    }
+    return pl;
+}
+
 perm_plan* perm_plan_create_sharded(const int32_t* p, int64_t n, int32_t elem_bytes, int32_t world,
-                                    int32_t rank, const perm_plan_options* opt) {
-    return create(p, n, elem_bytes, opt, true, world, rank);
+                                    int32_t rank, const void* nccl_uid) {
+    return perm_plan_create_sharded_ex(p, n, elem_bytes, world, rank, nccl_uid, nullptr);
+}
+
+int perm_sharded_exchange(const perm_plan* plan, const void* send, void* recv, perm_stream_t stream) {
+    if (!plan || !send || !recv) return fail(PERM_EINVAL, "null plan or buffer");
+    const HostPlan& P = plan->host;
+    if (!P.r_l) return fail(PERM_EINVAL, "not a row-sharded plan");
+    if (!plan->comm) return fail(PERM_ENCCL, "plan has no NCCL communicator (created without nccl_uid)");
+    if (overlap(send, recv, P.n / P.world * P.eb)) return fail(PERM_EINVAL, "send and recv overlap");
+    std::string err;
+    const perm::NcclApi* api = perm::nccl_api(err);
+    if (!api) return fail(PERM_ENCCL, err);
+    const int64_t block = P.n / ((int64_t)P.world * P.world);
+    const ncclResult_t r = perm::nccl_alltoall(*api, static_cast<const uint32_t*>(send), static_cast<uint32_t*>(recv),
+                                               block, P.world, plan->comm, static_cast<cudaStream_t>(stream));
+    if (r != ncclSuccess) return nccl_fail(api, r, "all-to-all");
+    return PERM_OK;
+}
+
+int perm_apply_sharded(const perm_plan* plan, const void* a_shard, void* b_shard, perm_stream_t stream) {
+    if (!plan || !a_shard || !b_shard) return fail(PERM_EINVAL, "null plan or buffer");
+    if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
+    const HostPlan& P = plan->host;
+    if (!P.r_l) return fail(PERM_EINVAL, "not a row-sharded plan (use perm_apply)");
+    if (!plan->comm) return fail(PERM_ENCCL, "plan has no NCCL communicator (created without nccl_uid)");
+    if (overlap(a_shard, b_shard, P.n / P.world * P.eb)) return fail(PERM_EINVAL, "a and b shards overlap");
+    // R1 + T-pack -> all-to-all -> R2 + T-pack -> all-to-all -> R3 (Lemma 8: the column
+    // phase's two transposes become the two uniform, P-independent exchanges)
+    int st = perm_sharded_step(plan, 0, a_shard, plan->d_send, stream);
+    if (st == PERM_OK) st = perm_sharded_exchange(plan, plan->d_send, plan->d_recv, stream);
+    if (st == PERM_OK) st = perm_sharded_step(plan, 1, plan->d_recv, plan->d_send, stream);
+    if (st == PERM_OK) st = perm_sharded_exchange(plan, plan->d_send, plan->d_recv, stream);
+    if (st == PERM_OK) st = perm_sharded_step(plan, 2, plan->d_recv, b_shard, stream);
+    return st;
 }
 
 perm_plan* perm_plan_create_sharded_host(const int32_t* p, int64_t n, int32_t elem_bytes,
@@ -247,7 +347,7 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     int64_t words = 0;
     for (int f = 0; f < 3; ++f) words += (int64_t)P.sched[f].size();
     out->sched_bytes = plan->on_device ? plan->sched_bytes : words * 4;
-    out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes == 1 ? 0 : 2 * P.n * P.eb);
+    out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes > 1 ? 2 * P.n * P.eb : 0);
     out->elem_bytes = P.user_eb;
     out->passes = P.passes;
     out->kernels_per_apply = (plan->d_p || P.fused3) ? 1 : P.passes;
@@ -334,6 +434,7 @@ int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint3
                      uint32_t* s3) {
     if (!plan) return fail(PERM_EINVAL, "null plan");
     const HostPlan& P = plan->host;
+    if (P.direct) return fail(PERM_EUNSUPPORTED, "low-distribution shortcut plan: no schedule to export");
     if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));   // words
     uint32_t* outs[3] = {s1, s2, s3};
     if (P.layout == 3) {
@@ -454,6 +555,7 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
     if (!plan || !a || !b) return fail(PERM_EINVAL, "null plan or buffer");
     if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
     const HostPlan& P = plan->host;
+    if (P.r_l) return fail(PERM_EINVAL, "row-sharded plan: use perm_apply_sharded or perm_sharded_step");
     if (overlap(a, b, P.n * P.eb)) return fail(PERM_EINVAL, "a and b overlap (out-of-place only)");
     if ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15)
         return fail(PERM_EINVAL, "a and b must be 16-byte aligned");
@@ -531,6 +633,7 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
 int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream) {
     if (!plan || !a_host || !b_host) return fail(PERM_EINVAL, "null plan or buffer");
     if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
+    if (plan->host.r_l) return fail(PERM_EINVAL, "row-sharded plan: use perm_apply_sharded or perm_sharded_step");
     const size_t bytes = (size_t)plan->host.n * plan->host.eb;
     cudaError_t e;
     if (!plan->d_stage[0]) {

@@ -2261,6 +2261,7 @@ cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const u
 }
 
 cudaError_t prepare_kernels(HostPlan& P) {
+    if (P.direct) return cudaSuccess;     // one stream kernel, no attributes to set
     if (P.layout == 3) return prep_tlc(P);
     cudaError_t e = cudaSuccess;
     auto set = [&](const void* k, size_t bytes) {

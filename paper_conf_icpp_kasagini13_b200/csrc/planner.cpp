@@ -175,13 +175,10 @@ struct EulerColourer {
             return __atomic_compare_exchange_n(&own[e], &expect, sid, false, __ATOMIC_RELAXED,
                                                __ATOMIC_RELAXED);
         };
-#pragma omp parallel num_threads(T)
-        {
-#ifdef _OPENMP
-            const int t = omp_get_thread_num();
-#else
-            const int t = 0;
-#endif
+        // one iteration per range t (not per OpenMP thread): correct whatever team size the
+        // runtime grants (OMP_DYNAMIC, nested regions, thread limits)
+#pragma omp parallel for schedule(static, 1)
+        for (int t = 0; t < T; ++t) {
             const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
             std::vector<Bound>& bd = bounds[t];
             std::vector<uint32_t>& mins = segmin[t];
@@ -269,20 +266,17 @@ struct EulerColourer {
         const double ms_flip = ms_since(t0);
         // parallel stable partition (zeros first)
         std::vector<int64_t> zc(T + 1, 0);
-#pragma omp parallel num_threads(T)
-        {
-#ifdef _OPENMP
-            const int t = omp_get_thread_num();
-#else
-            const int t = 0;
-#endif
+#pragma omp parallel for schedule(static, 1)
+        for (int t = 0; t < T; ++t) {
             const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
             int64_t z = 0;
             for (int64_t i = lo; i < hi; ++i) z += bit[i] == 0;
             zc[t + 1] = z;
-#pragma omp barrier
-#pragma omp single
-            for (int u = 0; u < T; ++u) zc[u + 1] += zc[u];
+        }
+        for (int u = 0; u < T; ++u) zc[u + 1] += zc[u];
+#pragma omp parallel for schedule(static, 1)
+        for (int t = 0; t < T; ++t) {
+            const int64_t lo = base + S * t / T, hi = base + S * (t + 1) / T;
             int64_t zp = base + zc[t], op = base + S / 2 + ((lo - base) - zc[t]);
             for (int64_t i = lo; i < hi; ++i) {
                 const int64_t dst = bit[i] ? op++ : zp++;
@@ -763,6 +757,15 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         }
     }
     P.n = n; P.eb = eb; P.k = k;
+    if (P.direct) {
+        // low-distribution shortcut: perm_apply runs one kernel on p_copy, so no colouring,
+        // schedule or scratch is built (direct = -1 keeps the scheduled passes for A/B runs)
+        const int lc = k - k / 2;
+        P.r = int64_t(1) << (k - lc);
+        P.c = int64_t(1) << lc;
+        P.passes = 0;
+        return PERM_OK;
+    }
     // view r x c (L603: "not restricted to a square matrix"); default c = 2^ceil(k/2)
     // n = 2^29 (5 passes): c = 2^14, r = 2^15, so the two row phases run on 16384-word
     // lines (schedule-from-global slots) and only the column phase on 32768-word lines
@@ -1132,6 +1135,7 @@ int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, i
     if (opt) o = *opt;
     o.passes = 5;
     o.layout = 0;
+    o.direct = -1;                      // the shortcut is a single-device kernel
     int st = build_host_plan(p, n, eb, &o, P, err);
     if (st != PERM_OK) return st;
     const int64_t r = P.r, c = P.c;

@@ -52,6 +52,7 @@ def decode(sched):
 
 
 def export_plan(lib, p, **kw):
+    kw.setdefault("direct", -1)     # shortcut plans (identity, shuffle) have no schedule
     with lib.Plan(p, device=False, **kw) as pl:
         info = pl.info()
         kappa, scheds = pl.export()
@@ -165,6 +166,7 @@ def test_bruteforce_tiny_via_cpp_euler_split(lib):
 # ---------------------------------------------------------------- TLC plans (layout 3)
 
 def export_tlc(lib, p, **kw):
+    kw.setdefault("direct", -1)
     with lib.Plan(p, device=False, passes=3, layout=3, **kw) as pl:
         info = pl.info()
         d = pl.describe()
@@ -347,7 +349,7 @@ def test_dense_schedule_format_passes_oracle_checker(lib, fam, k):
     p = W.make_perm(fam, n, seed=5 + k)
     info, kappa, sched = export_plan(lib, p, passes=5, sched_format=2)
     OC.assert_plan(p, kappa, sched, r, c, 32)
-    with lib.Plan(p, device=False, passes=5, sched_format=2) as pl:
+    with lib.Plan(p, device=False, passes=5, sched_format=2, direct=-1) as pl:
         d = pl.describe()
     for rp in d["row_passes"]:
         assert rp["dense"] == 1 and rp["sched_words_per_line"] == rp["L"] // 32 * rp["E"]

@@ -1,0 +1,65 @@
+"""GPU parity at BASELINE.json's full sizes: the default plans (the launch configuration
+bench.py and the C5 sweep time) for n = 2^26 .. 2^30, every element compared with the
+oracle's definition b[P(i)] = a[i], tolerance 0.
+
+Default structures covered: 2^26 / 2^27 five passes with the schedule in
+the TMA slot (W64) / read from global (SG); 2^28 SG with dense per-round bitstreams;
+2^29 the tall view (r = 2^15, c = 2^14: R1/R3 on 16384-word lines, R2 on the half-line
+ring); 2^30 the half-line ring with staged dense schedule chunks on every phase.
+Host RAM: up to ~60 GB at 2^30 (p, a, the oracle's b, the GPU's b, the planner).
+"""
+import gc
+
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import apply as OA
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_kasagini13_b200 import build
+    build.build()
+    import paper_conf_icpp_kasagini13_b200 as pkg
+    return pkg
+
+
+CASES = [(26, "bitrev"), (26, "transpose"),
+         (27, "random"), (27, "bitrev"), (27, "transpose"),
+         (28, "random"), (28, "bitrev"), (28, "transpose"),
+         (29, "random"),
+         (30, "random"), (30, "bitrev")]
+
+
+@pytest.mark.parametrize("k,fam", CASES)
+def test_default_plan_full_size(P, k, fam):
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=42)
+    a = W.make_data(n)
+    with P.Plan(p) as plan:
+        info = plan.info()
+        assert info["direct"] == 0 and info["passes"] == 5, info
+        if k == 29:
+            assert (info["rows"], info["cols"]) == (1 << 15, 1 << 14)     # tall view
+        da = torch.from_numpy(a.view(np.int32)).cuda()
+        db = torch.full_like(da, -1)
+        plan.apply(da, db)
+        torch.cuda.synchronize()
+        del da
+        b = db.cpu().numpy().view(np.uint32)
+        del db
+    torch.cuda.empty_cache()
+    ref = OA.apply_ref(p, a)
+    del p, a
+    ok = bool(np.array_equal(b, ref))
+    if not ok:
+        bad = np.flatnonzero(b != ref)
+        pytest.fail(f"2^{k} {fam}: {bad.size} mismatching words, first at {bad[:8].tolist()}")
+    del b, ref
+    gc.collect()

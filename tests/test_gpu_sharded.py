@@ -1,4 +1,5 @@
-"""GPU: the row-sharded path with G virtual ranks on one device.
+"""GPU: the row-sharded path with G virtual ranks on one device, and the whole
+sharded apply through libperm's C ABI (perm_apply_sharded: kernels + NCCL).
 
 Every rank's perm_sharded_step kernels run for real (R1+T-pack, R2 over G segments
 per column + T-pack, R3 over G segments per row); the all-to-all between steps is
@@ -66,3 +67,69 @@ def test_sharded_step_errors(P):
         y = torch.zeros(n, dtype=torch.int32, device="cuda")
         with pytest.raises(P.PermError):
             pl.sharded_step(0, x, y)
+
+
+@pytest.mark.parametrize("fam", ["random", "bitrev"])
+def test_virtual_ranks_g8_2pow26(P, fam):
+    # C3 size with the widest sharding the bench uses (G = 8): default kernels per step
+    from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
+    G, n = 8, 1 << 26
+    shard = n // G
+    a = W.make_data(n)
+    p = W.make_perm(fam, n, seed=5)
+    plans = [P.Plan(p, world=G, rank=g) for g in range(G)]
+    try:
+        a_sh = [torch.from_numpy(a[g * shard:(g + 1) * shard].view(np.int32).copy()).cuda() for g in range(G)]
+        b_sh = [torch.full((shard,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
+        send = [torch.empty(shard, dtype=torch.int32, device="cuda") for _ in range(G)]
+        recv = [torch.empty(shard, dtype=torch.int32, device="cuda") for _ in range(G)]
+        apply_virtual(plans, a_sh, b_sh, send, recv)
+        torch.cuda.synchronize()
+        b = np.concatenate([x.cpu().numpy().view(np.uint32) for x in b_sh])
+        assert np.array_equal(b, OA.apply_ref(p, a)), fam
+    finally:
+        for pl in plans:
+            pl.close()
+
+
+@pytest.mark.parametrize("k", [16, 22])
+def test_apply_sharded_through_nccl_world1(P, k):
+    # perm_apply_sharded: R1+T-pack, NCCL all-to-all (grouped send/recv on the caller's
+    # stream), R2+T-pack, all-to-all, R3 -- all inside libperm. One GPU in this test, so
+    # the communicator has one rank (the exchange is NCCL's self send/recv).
+    n = 1 << k
+    uid = P.nccl_unique_id()
+    assert len(uid) == 128
+    a = W.make_data(n)
+    for fam in ("random", "bitrev", "transpose"):
+        p = W.make_perm(fam, n, seed=k)
+        with P.Plan(p, world=1, rank=0, nccl_uid=uid if fam == "random" else P.nccl_unique_id()) as pl:
+            da = torch.from_numpy(a.view(np.int32).copy()).cuda()
+            db = torch.full_like(da, -1)
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                pl.apply_sharded(da, db, s)
+            s.synchronize()
+            assert np.array_equal(db.cpu().numpy().view(np.uint32), OA.apply_ref(p, a)), fam
+            # the exchange alone is the block contract (world 1: a copy)
+            x = torch.arange(n, dtype=torch.int32, device="cuda")
+            y = torch.zeros_like(x)
+            pl.sharded_exchange(x, y)
+            torch.cuda.synchronize()
+            assert torch.equal(x, y)
+
+
+def test_apply_sharded_errors(P):
+    n = 1 << 16
+    p = W.random(n, 3)
+    x = torch.zeros(n, dtype=torch.int32, device="cuda")
+    y = torch.zeros(n, dtype=torch.int32, device="cuda")
+    with P.Plan(p, world=1, rank=0) as pl:                 # no communicator
+        with pytest.raises(P.PermError) as ei:
+            pl.apply_sharded(x, y)
+        assert ei.value.status == -6
+        with pytest.raises(P.PermError):
+            pl.apply(x, y)                                  # sharded plans: not perm_apply
+    with P.Plan(p) as pl:                                   # unsharded plan
+        with pytest.raises(P.PermError):
+            pl.apply_sharded(x, y)

@@ -75,13 +75,21 @@ def shuffle(n: int) -> np.ndarray:
     return (((i << 1) | (i >> (m - 1))) & (n - 1)).astype(np.int32)
 
 
+_REV8 = np.array([int(f"{v:08b}"[::-1], 2) for v in range(256)], dtype=np.uint32)
+
+
 def bitrev(n: int) -> np.ndarray:
+    """Reverse all m bits of i: the 32-bit reversal of i (bytes reversed, each byte
+    through a 256-entry table), shifted right by 32 - m."""
     m = log2_exact(n)
-    i = np.arange(n, dtype=np.int64)
-    out = np.zeros(n, dtype=np.int64)
-    for b in range(m):
-        out |= ((i >> b) & 1) << (m - 1 - b)
-    return out.astype(np.int32)
+    if m == 0:
+        return np.zeros(1, dtype=np.int32)
+    i = np.arange(n, dtype=np.uint32)
+    out = _REV8[i & 0xFF] << 24
+    out |= _REV8[(i >> 8) & 0xFF] << 16
+    out |= _REV8[(i >> 16) & 0xFF] << 8
+    out |= _REV8[i >> 24]
+    return (out >> np.uint32(32 - m)).astype(np.int32)
 
 
 def transpose(n: int) -> np.ndarray:
