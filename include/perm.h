@@ -52,6 +52,10 @@ enum perm_status {
 enum perm_passes {
     PERM_PASSES_AUTO  = 0,
     PERM_PASSES_FUSED = 1,   /* n <= 2^14: all three phases inside one CTA's shared memory */
+    PERM_PASSES_CLUSTER = 2, /* n = 2^15..2^18: ONE launch; the array lives in the shared memory
+                                of one thread-block cluster (2..16 blocks); the column phase's
+                                two transposes become block exchanges over distributed shared
+                                memory (DSMEM bulk copies); a and b cross HBM once each */
     PERM_PASSES_3     = 3,   /* R1, R2, R3; both transposes absorbed into tiled layouts */
     PERM_PASSES_5     = 5    /* R, T, R, T, R: the paper's five kernel calls (L699) */
 };
@@ -100,6 +104,9 @@ typedef struct {
                             current CUDA device (gplan.cu: Euler split with ruling-set cycle
                             labelling), -1 = host threads (planner.cpp), 0 = auto (device for
                             device plans with n >= 2^20, host otherwise) */
+    int32_t cluster;     /* cluster path (passes = 2): thread blocks per cluster, a power of two
+                            in 2..16; 0 = 16 for n >= 2^16, else 8 (raised until a block holds
+                            <= 16384 words) */
 } perm_plan_options;
 
 typedef struct {
@@ -108,7 +115,7 @@ typedef struct {
     int64_t sched_bytes;         /* device bytes of the three packed bank schedules */
     int64_t scratch_bytes;       /* device bytes of intermediate buffers */
     int32_t elem_bytes;
-    int32_t passes;              /* 1, 3 or 5; 0 for a low-distribution shortcut plan
+    int32_t passes;              /* 1, 2 (cluster), 3 or 5; 0 for a low-distribution shortcut plan
                                     (direct != 0: one kernel, no schedule) */
     int32_t kernels_per_apply;   /* kernel launches one perm_apply issues */
     int32_t entry_bits[3];       /* bits per schedule entry, phase 1..3 (2*log2(L) - 5) */

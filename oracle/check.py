@@ -179,3 +179,64 @@ def check_tlc(p, kappa, sched, rows: int, cols: int, h, w: int = 32) -> dict:
     res["vii_sources_and_dests_cover_tile"] = ok_cover
     res["viii_lane_is_source_bank"] = ok_lane
     return res
+
+
+# ---------------------------------------------------------------- cluster plans
+#
+# DESIGN.md §5 "cluster path" (restated, not imported): C thread blocks of one cluster
+# hold the whole array; r_l = r/C, c_l = c/C, Bw = r_l*c_l. Block g's phase-1 input is
+# rows [g*r_l, ...) of a (row-major); its phase-1 output is C send blocks, element
+# (i, k) in block k div c_l at [k mod c_l][i mod r_l]; the exchange delivers send block
+# q of block g to block q at [g*Bw, (g+1)*Bw). Phase 2 output: send block i' div r_l at
+# [i' mod r_l][k mod c_l]; phase 3 output: block m's rows of b, row-major. The checker
+# derives every element from its SOURCE offset (the input side of each phase), routes
+# it with the Phi it recomputes, and compares with the destination offset.
+
+def check_cluster(p, kappa, sched, rows: int, cols: int, C: int, w: int = 32) -> dict:
+    p = np.asarray(p, dtype=np.int64)
+    kappa = np.asarray(kappa, dtype=np.int64)
+    r, c = rows, cols
+    n = r * c
+    rl, cl, S = r // C, c // C, n // C
+    Bw = rl * cl
+    res = {}
+    res["i_row_colours_bijective"] = _rows_are_perms(kappa.reshape(r, c))
+    res["ii_colour_dest_rows_distinct"] = bool(np.unique(kappa * r + p // c).size == n)
+    if not (res["i_row_colours_bijective"] and res["ii_colour_dest_rows_distinct"]):
+        return res
+    phi1, phi2, phi3 = phases_from_kappa(p, kappa, r, c)
+    ok_map = ok_cover = ok_banks = ok_lane = True
+    g = np.arange(C, dtype=np.int64)[:, None]
+    for f in range(3):
+        e = np.asarray(sched[f], dtype=np.int64).reshape(C, S)
+        src, dst = e >> 16, e & 0xFFFF
+        lane = (np.arange(S, dtype=np.int64) % w)[None, :]
+        ok_lane &= bool(np.all(src % w == lane))
+        ok_cover &= _rows_are_perms(src) and _rows_are_perms(dst)
+        ok_banks &= _rounds_distinct(src, w) and _rounds_distinct(dst, w)
+        if f == 0:
+            i = g * rl + src // c
+            k = phi1[i, src % c]
+            want = (k // cl) * Bw + (k % cl) * rl + i % rl
+        elif f == 1:
+            sender, rem = src // Bw, src % Bw
+            k_in, i_l = rem // rl, rem % rl
+            ip = phi2[g * cl + k_in, sender * rl + i_l]
+            want = (ip // rl) * Bw + (ip % rl) * cl + k_in
+        else:
+            sender, rem = src // Bw, src % Bw
+            i_l, k_in = rem // cl, rem % cl
+            kp = phi3[g * rl + i_l, sender * cl + k_in]
+            want = i_l * c + kp
+        ok_map &= bool(np.all(dst == want))
+    x = np.arange(n, dtype=np.int64)
+    i, j = x // c, x % c
+    k = phi1[i, j]
+    row2 = phi2[k, i]
+    res["iii_phases_bijective"] = all(_rows_are_perms(ph) for ph in (phi1, phi2, phi3))
+    res["iv_composition_is_P"] = bool(np.all(row2 * c + phi3[row2, k] == p))
+    res["v_blocks_implement_phi"] = ok_map
+    res["vi_rounds_conflict_free_A_and_B"] = ok_banks
+    res["vii_sources_and_dests_cover_block"] = ok_cover
+    res["viii_lane_is_source_bank"] = ok_lane
+    return res

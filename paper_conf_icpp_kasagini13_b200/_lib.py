@@ -37,7 +37,8 @@ class PlanOptions(ctypes.Structure):
     _fields_ = [("passes", ctypes.c_int32), ("h1", ctypes.c_int32), ("h2", ctypes.c_int32),
                 ("h3", ctypes.c_int32), ("layout", ctypes.c_int32), ("stages", ctypes.c_int32),
                 ("fuse", ctypes.c_int32), ("no_tma", ctypes.c_int32), ("direct", ctypes.c_int32),
-                ("log2c", ctypes.c_int32), ("sched_format", ctypes.c_int32), ("gpu_planner", ctypes.c_int32)]
+                ("log2c", ctypes.c_int32), ("sched_format", ctypes.c_int32), ("gpu_planner", ctypes.c_int32),
+                ("cluster", ctypes.c_int32)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -165,7 +166,8 @@ class Plan:
     def __init__(self, p, elem_bytes: int = 4, passes: int = 0, h=(0, 0, 0),
                  device: bool = True, layout: int = 0, stages: int = 0, fuse: int = 0,
                  world: int = 0, rank: int = 0, no_tma: int = 0, direct: int = 0, log2c: int = 0,
-                 sched_format: int = 0, gpu_planner: int = 0, nccl_uid: bytes | None = None):
+                 sched_format: int = 0, gpu_planner: int = 0, nccl_uid: bytes | None = None,
+                 cluster: int = 0):
         """world > 0: row-sharded plan of rank `rank` (see perm_plan_create_sharded);
         nccl_uid (128 bytes, the same on every rank) also joins the plan's NCCL
         communicator, so apply_sharded() runs the whole sharded apply in libperm."""
@@ -173,7 +175,7 @@ class Plan:
         self.n = int(p.size)
         self.elem_bytes = elem_bytes
         opt = PlanOptions(passes, h[0], h[1], h[2], layout, stages, fuse, no_tma, direct, log2c,
-                          sched_format, gpu_planner)
+                          sched_format, gpu_planner, cluster)
         if world > 0:
             if device:
                 uid = None

@@ -108,7 +108,7 @@ int upload(perm_plan* pl) {
         if (e != cudaSuccess) return cuda_fail(e, "cudaMemset");
         off += padded(wf);
     }
-    if (P.passes > 1) {
+    if (P.passes > 2) {
         const size_t bytes = (size_t)(P.r_l ? P.n / P.world : P.n) * P.eb;
         for (int i = 0; i < 2; ++i) {
             e = cudaMalloc(&pl->d_scratch[i], bytes);
@@ -347,15 +347,15 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     int64_t words = 0;
     for (int f = 0; f < 3; ++f) words += (int64_t)P.sched[f].size();
     out->sched_bytes = plan->on_device ? plan->sched_bytes : words * 4;
-    out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes > 1 ? 2 * P.n * P.eb : 0);
+    out->scratch_bytes = plan->on_device ? plan->scratch_bytes : (P.passes > 2 ? 2 * P.n * P.eb : 0);
     out->elem_bytes = P.user_eb;
     out->passes = P.passes;
-    out->kernels_per_apply = (plan->d_p || P.fused3) ? 1 : P.passes;
+    out->kernels_per_apply = (plan->d_p || P.fused3 || P.passes == 2) ? 1 : P.passes;
     out->distribution = P.distribution;
     out->direct = P.direct;
     out->gpu_planner = P.gpu_planner;
     for (int f = 0; f < 3; ++f) {
-        out->entry_bits[f] = P.layout == 3 ? P.tp[f].E : P.ph[f].E;
+        out->entry_bits[f] = P.layout >= 3 ? P.tp[f].E : P.ph[f].E;
         out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
     }
     out->planner_threads = P.threads_used;
@@ -378,7 +378,8 @@ int64_t perm_plan_describe(const perm_plan* plan, char* buf, int64_t len) {
                     ",\"layout\":" + std::to_string(P.layout) + ",\"fused3\":" + std::to_string(P.fused3) +
                     ",\"distribution\":" + std::to_string(P.distribution) +
                     ",\"direct\":" + std::to_string(P.direct);
-    if (P.layout == 3) {
+    if (P.passes == 2) s += ",\"cluster\":" + std::to_string(P.cluster);
+    if (P.layout >= 3) {
         s += ",\"tlc\":[";
         for (int f = 0; f < 3; ++f) {
             const perm::TlcPass& tp = P.tp[f];
@@ -437,8 +438,8 @@ int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint3
     if (P.direct) return fail(PERM_EUNSUPPORTED, "low-distribution shortcut plan: no schedule to export");
     if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));   // words
     uint32_t* outs[3] = {s1, s2, s3};
-    if (P.layout == 3) {
-        // TLC: entry (tile T, round q, lane x) -> (src word offset in A << 16) | dst offset in B
+    if (P.layout >= 3) {
+        // TLC / cluster path: entry (tile T, round q, lane x) -> (src word offset in A << 16) | dst offset in B
         for (int f = 0; f < 3; ++f) {
             if (!outs[f]) continue;
             const perm::TlcPass& tp = P.tp[f];
@@ -585,6 +586,10 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
         e = perm::launch_fused(P, sc, in, out, s);
         mark();
+    } else if (P.passes == 2) {
+        const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
+        e = perm::launch_cluster(P, sc, in, out, s);
+        mark();
     } else if (P.layout == 3 && P.fused3) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
         e = perm::launch_tlc_fused(P, plan->tlc_maps, sc, in, plan->d_scratch[0], plan->d_scratch[1], out,
@@ -597,11 +602,6 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
         mark();
         if (e == cudaSuccess) { ++k; e = perm::launch_tlc_pass(P, 1, plan->tlc_maps, plan->d_phase[1], x1, x2, s, !prof, tr(1)); mark(); }
         if (e == cudaSuccess) { ++k; e = perm::launch_tlc_pass(P, 2, plan->tlc_maps, plan->d_phase[2], x2, out, s, !prof, tr(2)); mark(); }
-    } else if (P.fused3) {
-        const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
-        e = perm::launch_fused3(P, sc, in, plan->d_scratch[0], plan->d_scratch[1], out, plan->d_sync,
-                                s, tr(0));
-        mark();
     } else if (P.passes == 3) {
         uint32_t* x1 = plan->d_scratch[0];
         uint32_t* x2 = plan->d_scratch[1];

@@ -709,7 +709,7 @@ __global__ void __launch_bounds__((EPT >= 64) ? 512 : 1024, 1) row_pass_split_ke
     stamp(tr, 14);
 }
 
-// ------------------------------------------------------------------ row pass, warp-specialized
+// ------------------------------------------------------------------ named barriers, mbarrier arrive, trace stamps
 
 __device__ __forceinline__ void named_bar(int id, int count) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
@@ -719,234 +719,6 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 }
 __device__ __forceinline__ void stamp_if(unsigned long long* tr, bool who, int slot) {
     if (tr != nullptr && who) tr[blockIdx.x * 16 + slot] = gtimer();
-}
-
-constexpr int kWsPerm = 512;    // permuter threads (16 warps)
-constexpr int kWsStore = 256;   // storer threads (8 warps), CROSS output only
-
-struct WsArgs {
-    RowArgs r;                  // geometry, output layout (r.o), trace
-    int ntiles, stages;
-    int data_words;             // h * Ls
-    int sched_words;            // h * (L/32) * w64 * 2
-};
-
-// In-place permute of one tile by the permuter warps: permuter warp pw owns the
-// EPT consecutive warp-rounds q = pw*EPT + m (one line when EPT <= L/32), so the
-// line base is computed once; schedule entries are decoded once (W64 format)
-// and the destination addresses wait in registers across the named barrier.
-template <int EPT>
-__device__ __forceinline__ void permute_tile_ws(uint32_t* sm, const uint32_t* sched, int logL,
-                                                int E, int epw, int w64, int Ls, int pw, int lane) {
-    const int logR = logL - 5;
-    const int wsel = lane / epw;
-    const int sh = E * (lane - wsel * epw);
-    const uint32_t mask = (1u << E) - 1u;
-    const uint32_t tmask = (1u << logL) - 1u;
-    const int q0 = pw * EPT;
-    const uint2* sp = reinterpret_cast<const uint2*>(sched) + q0 * w64 + wsel;
-    constexpr bool KEEP = EPT <= 32;
-    uint32_t v[EPT];
-    uint32_t ta[KEEP ? (EPT + 1) / 2 : 1];
-    const bool one_line = EPT <= (1 << logR);
-    const int lb0 = (q0 >> logR) * Ls + lane;
-#pragma unroll
-    for (int m = 0; m < EPT; ++m) {
-        const uint2 wd = sp[m * w64];
-        const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
-        const uint32_t e = (uint32_t)(w >> sh) & mask;
-        const int lb = one_line ? lb0 : ((q0 + m) >> logR) * Ls + lane;
-        v[m] = sm[lb + (int)((e >> logL) << 5)];
-        if constexpr (KEEP) {
-            const uint32_t ad = (uint32_t)(lb - lane) + (e & tmask);
-            if (m & 1) ta[m >> 1] |= ad << 16;
-            else ta[m >> 1] = ad;
-        }
-    }
-    named_bar(1, kWsPerm);
-    if constexpr (KEEP) {
-#pragma unroll
-        for (int m = 0; m < EPT; ++m) sm[(ta[m >> 1] >> ((m & 1) * 16)) & 0xFFFFu] = v[m];
-    } else {
-        const int q1 = __shfl_sync(kFull, q0, 0);
-        const uint2* sp2 = reinterpret_cast<const uint2*>(sched) + q1 * w64 + wsel;
-#pragma unroll
-        for (int m = 0; m < EPT; ++m) {
-            const uint2 wd = sp2[m * w64];
-            const uint64_t w = ((uint64_t)wd.y << 32) | wd.x;
-            const uint32_t e = (uint32_t)(w >> sh) & mask;
-            sm[((q1 + m) >> logR) * Ls + (int)(e & tmask)] = v[m];
-        }
-    }
-}
-
-// Persistent warp-specialized row-wise permutation pass (Lemma 7) over
-// contiguous input lines. Ring of `stages` shared-memory slots [h lines | the
-// tile's packed schedule]; three mbarriers per slot:
-//   full[s]  TMA bytes landed          (producer thread arms, TMA completes)
-//   perm[s]  tile permuted in place    (512 permuter threads arrive)
-//   empty[s] slot read by the storers  (256 storer threads arrive; CROSS only)
-// warp 0 lane 0: TMA producer (and, for row-major output, the TMA bulk storer);
-// warps 1..16: permuters; warps 17..24: storers (CROSS output gather + 128-bit
-// stores). Loading tile i+1, permuting tile i and storing tile i-1 overlap.
-template <int EPT, bool OUT_CROSS>
-__global__ void __launch_bounds__(OUT_CROSS ? 32 + kWsPerm + kWsStore : 32 + kWsPerm, 1)
-    row_pass_ws_kernel(const WsArgs a) {
-    extern __shared__ __align__(128) uint32_t smem[];
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int L = 1 << a.r.logL, h = 1 << a.r.logh;
-    const int NS = a.stages;
-    const int stage_words = a.data_words + a.sched_words;
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * stage_words);
-    uint64_t* permd = full + NS;
-    uint64_t* empty = permd + NS;
-    const int G = gridDim.x;
-    const uint32_t line_bytes = (uint32_t)L * 4u;
-    const bool dense = a.r.Ls == L;
-    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (uint32_t)a.sched_words * 4u;
-    unsigned long long* tr = a.r.trace;
-    stamp(tr, 0);
-    if (tid == 0) {
-        for (int s = 0; s < NS; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&permd[s], kWsPerm);
-            mbar_init(&empty[s], OUT_CROSS ? kWsStore : 1);
-        }
-        fence_mbar_init();
-    }
-    __syncthreads();
-
-    auto issue = [&](int s, long long t, bool sched_part, bool data_part) {
-        uint32_t* dst = smem + s * stage_words;
-        if (sched_part)
-            bulk_g2s(dst + a.data_words, a.r.sched + t * a.sched_words, (uint32_t)a.sched_words * 4u,
-                     &full[s]);
-        if (data_part) {
-            const uint32_t* src = a.r.in + t * h * (long long)L;
-            if (dense) {
-                bulk_g2s(dst, src, (uint32_t)h * line_bytes, &full[s]);
-            } else {
-                for (int l = 0; l < h; ++l)
-                    bulk_g2s(dst + l * a.r.Ls, src + (long long)l * L, line_bytes, &full[s]);
-            }
-        }
-    };
-
-    if (warp == 0) {
-        // ---------------- producer (and bulk storer for row-major output)
-        if (lane == 0) {
-            for (int s = 0; s < NS; ++s) {
-                const long long t = blockIdx.x + (long long)s * G;
-                if (t < a.ntiles) {
-                    mbar_arrive_expect_tx(&full[s], tile_bytes);
-                    issue(s, t, true, false);     // schedule does not depend on the previous pass
-                }
-            }
-            pdl_wait();
-            stamp(tr, 1);
-            for (int s = 0; s < NS; ++s) {
-                const long long t = blockIdx.x + (long long)s * G;
-                if (t < a.ntiles) issue(s, t, false, true);
-            }
-            pdl_launch_dependents();
-            if constexpr (OUT_CROSS) {
-                for (int i = NS;; ++i) {
-                    const long long t = blockIdx.x + (long long)i * G;
-                    if (t >= a.ntiles) break;
-                    const int s = i % NS;
-                    mbar_wait(&empty[s], (uint32_t)(i / NS - 1) & 1u);
-                    fence_proxy_async();
-                    mbar_arrive_expect_tx(&full[s], tile_bytes);
-                    issue(s, t, true, true);
-                }
-            } else {
-                for (int i = 0;; ++i) {
-                    const long long t = blockIdx.x + (long long)i * G;
-                    if (t >= a.ntiles) break;
-                    const int s = i % NS;
-                    mbar_wait(&permd[s], (uint32_t)(i / NS) & 1u);
-                    fence_proxy_async();          // permuters' smem writes -> async-proxy reads
-                    const uint32_t* buf = smem + s * stage_words;
-                    uint32_t* dst = a.r.out + t * h * (long long)L;
-                    if (dense) {
-                        bulk_s2g(dst, buf, (uint32_t)h * line_bytes);
-                    } else {
-                        for (int l = 0; l < h; ++l)
-                            bulk_s2g(dst + (long long)l * L, buf + l * a.r.Ls, line_bytes);
-                    }
-                    bulk_commit();
-                    if (i < 4) stamp_if(tr, true, 4 + 3 * i);
-                    const long long tn = t + (long long)NS * G;
-                    if (tn < a.ntiles) {
-                        bulk_wait_read0();
-                        fence_proxy_async();
-                        mbar_arrive_expect_tx(&full[s], tile_bytes);
-                        issue(s, tn, true, true);
-                    }
-                }
-                bulk_wait0();
-            }
-            stamp(tr, 14);
-        }
-    } else if (warp <= kWsPerm / 32) {
-        // ---------------- permuters
-        const int pw = warp - 1;
-        const bool lead = tid == 32;
-        for (int i = 0;; ++i) {
-            const long long t = blockIdx.x + (long long)i * G;
-            if (t >= a.ntiles) break;
-            const int s = i % NS;
-            mbar_wait(&full[s], (uint32_t)(i / NS) & 1u);
-            if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
-            uint32_t* buf = smem + s * stage_words;
-            permute_tile_ws<EPT>(buf, buf + a.data_words, a.r.logL, a.r.E, a.r.epw, a.r.w64, a.r.Ls,
-                                 pw, lane);
-            mbar_arrive(&permd[s]);
-            if (i < 4) stamp_if(tr, lead, 3 + 3 * i);
-        }
-    } else if constexpr (OUT_CROSS) {
-        // ---------------- storers: gather column chunks, 128-bit stores
-        pdl_wait();
-        const int sj = tid - 32 - kWsPerm;
-        const bool lead = sj == 0;
-        const int logh = a.r.logh;
-        const Io& m = a.r.o;
-        const int logBPh = m.logBP + logh;
-        constexpr int NV = (kWsPerm * EPT) / (4 * kWsStore);   // vectors per storer thread
-        for (int i = 0;; ++i) {
-            const long long t = blockIdx.x + (long long)i * G;
-            if (t >= a.ntiles) break;
-            const int s = i % NS;
-            mbar_wait(&permd[s], (uint32_t)(i / NS) & 1u);
-            const uint32_t* buf = smem + s * stage_words;
-            uint32_t* base = a.r.out + t * m.cta_stride;
-            constexpr int CH = NV < 8 ? NV : 8;
-#pragma unroll
-            for (int c0 = 0; c0 < NV; c0 += CH) {
-                uint4 vv[CH];
-#pragma unroll
-                for (int u = 0; u < CH; ++u) {
-                    const int f = 4 * (sj + kWsStore * (c0 + u));
-                    const int pos = f >> logh, l = f & ((1 << logh) - 1);
-                    const uint32_t* src = buf + l * a.r.Ls + pos;
-                    vv[u].x = src[0];
-                    vv[u].y = src[a.r.Ls];
-                    vv[u].z = src[2 * a.r.Ls];
-                    vv[u].w = src[3 * a.r.Ls];
-                }
-                if (c0 + CH >= NV) mbar_arrive(&empty[s]);   // slot may be refilled
-#pragma unroll
-                for (int u = 0; u < CH; ++u) {
-                    const int f = 4 * (sj + kWsStore * (c0 + u));
-                    const int pos = f >> logh;
-                    st_v4(base + (long long)(pos >> m.logBP) * m.strideP + (f & ((1 << logBPh) - 1)),
-                          vv[u]);
-                }
-            }
-            if (i < 4) stamp_if(tr, lead, 4 + 3 * i);
-        }
-        stamp_if(tr, lead, 15);
-    }
 }
 
 // ------------------------------------------------------------------ half-line ring, staged schedule
@@ -1103,207 +875,6 @@ __device__ __forceinline__ void red_release_gpu_add(unsigned long long* p, unsig
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-struct PassCfg {
-    const uint32_t* in;
-    uint32_t* out;
-    const uint32_t* sched;     // this phase's packed schedule
-    int ntiles;                // lines / h
-    int cross;                 // 1: out[t*h + pos*strideP + l] (column chunks); 0: row-major lines
-    long long strideP;
-};
-
-struct Fused3Args {
-    PassCfg p[3];
-    int logL, logh, Ls, E, epw, w64;
-    int stages, data_words, sched_words;
-    unsigned long long* sync;  // [0], [1]: arrivals at the barriers after pass 0 / pass 1,
-                               // [2]: exits (the last CTA out resets all three)
-    unsigned long long* trace;
-};
-
-// The whole scheduled permutation (Thm 9: row-wise, column-wise, row-wise) in
-// ONE persistent launch, for square views (every phase has lines of length L).
-// Same warp roles and slot ring as row_pass_ws_kernel, continued across the
-// three passes (global tile sequence j). Between pass k and k+1 every element
-// of the intermediate must be written before any is read, so: the storers of a
-// CTA fence and publish their last pass-k store (red.release.gpu on sync[k]);
-// the producer may already arm a slot and TMA the NEXT pass's schedule, but
-// issues the next pass's data copies only after sync[k] reaches the grid size.
-// All CTAs are co-resident (grid = one CTA per SM). The last CTA to exit
-// resets the counters, so the kernel is replayable (e.g. inside a CUDA graph).
-template <int EPT>
-__global__ void __launch_bounds__(32 + kWsPerm + kWsStore, 1) fused3_ws_kernel(const Fused3Args a) {
-    extern __shared__ __align__(128) uint32_t smem[];
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int L = 1 << a.logL, h = 1 << a.logh;
-    const int NS = a.stages;
-    const int stage_words = a.data_words + a.sched_words;
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * stage_words);
-    uint64_t* permd = full + NS;
-    uint64_t* empty = permd + NS;
-    const int G = gridDim.x;
-    const uint32_t line_bytes = (uint32_t)L * 4u;
-    const bool dense = a.Ls == L;
-    const uint32_t tile_bytes = (uint32_t)h * line_bytes + (uint32_t)a.sched_words * 4u;
-    unsigned long long* tr = a.trace;
-    stamp(tr, 0);
-    if (tid == 0) {
-        for (int s = 0; s < NS; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&permd[s], kWsPerm);
-            mbar_init(&empty[s], kWsStore);
-        }
-        fence_mbar_init();
-    }
-    __syncthreads();
-    // tiles of pass k owned by this CTA: t = blockIdx.x + i*G < ntiles_k
-    auto my_tiles = [&](int k) -> int {
-        const int n = a.p[k].ntiles - (int)blockIdx.x;
-        return n > 0 ? (n + G - 1) / G : 0;
-    };
-
-    if (warp == 0) {
-        if (lane == 0) {
-            // ---------------- producer
-            int j = 0;
-            for (int k = 0; k < 3; ++k) {
-                const PassCfg& pc = a.p[k];
-                const int nt = my_tiles(k);
-                bool data_ok = (k == 0);
-                for (int i = 0; i < nt; ++i, ++j) {
-                    const long long t = blockIdx.x + (long long)i * G;
-                    const int s = j % NS;
-                    if (j >= NS) mbar_wait(&empty[s], (uint32_t)(j / NS - 1) & 1u);
-                    fence_proxy_async();
-                    mbar_arrive_expect_tx(&full[s], tile_bytes);
-                    uint32_t* dst = smem + s * stage_words;
-                    bulk_g2s(dst + a.data_words, pc.sched + t * a.sched_words,
-                             (uint32_t)a.sched_words * 4u, &full[s]);
-                    if (!data_ok) {
-                        // grid barrier: every CTA has published its pass k-1 stores. One
-                        // counter per barrier: a CTA that runs ahead (e.g. owns no tiles)
-                        // must not count toward an earlier barrier.
-                        while (ld_acquire_gpu(&a.sync[k - 1]) < (unsigned long long)G) __nanosleep(64);
-                        fence_proxy_async_global();
-                        data_ok = true;
-                        stamp(tr, 1 + 4 * k);
-                    }
-                    const uint32_t* src = pc.in + t * h * (long long)L;
-                    if (dense) {
-                        bulk_g2s(dst, src, (uint32_t)h * line_bytes, &full[s]);
-                    } else {
-                        for (int l = 0; l < h; ++l)
-                            bulk_g2s(dst + l * a.Ls, src + (long long)l * L, line_bytes, &full[s]);
-                    }
-                }
-                if (k == 0) {
-                    // pass 0's loads are out: the later passes' schedules do not depend on
-                    // the data, so stream them into L2 while pass 0 permutes and stores
-                    for (int k2 = 1; k2 < 3; ++k2)
-                        for (int i = 0; i < my_tiles(k2); ++i) {
-                            const long long t = blockIdx.x + (long long)i * G;
-                            prefetch_l2_bulk(a.p[k2].sched + t * a.sched_words,
-                                             (uint32_t)a.sched_words * 4u);
-                        }
-                }
-            }
-        }
-    } else if (warp <= kWsPerm / 32) {
-        // ---------------- permuters
-        const int pw = warp - 1;
-        const bool lead = tid == 32;
-        int j = 0;
-        for (int k = 0; k < 3; ++k) {
-            const int nt = my_tiles(k);
-            for (int i = 0; i < nt; ++i, ++j) {
-                const int s = j % NS;
-                mbar_wait(&full[s], (uint32_t)(j / NS) & 1u);
-                if (i == 0) stamp_if(tr, lead, 2 + 4 * k);
-                uint32_t* buf = smem + s * stage_words;
-                permute_tile_ws<EPT>(buf, buf + a.data_words, a.logL, a.E, a.epw, a.w64, a.Ls, pw, lane);
-                mbar_arrive(&permd[s]);
-            }
-            stamp_if(tr, lead, 3 + 4 * k);
-        }
-    } else {
-        // ---------------- storers
-        const int sj = tid - 32 - kWsPerm;
-        const bool lead = sj == 0;
-        const int logh = a.logh;
-        constexpr int NV = (kWsPerm * EPT) / (4 * kWsStore);
-        constexpr int CH = NV < 8 ? NV : 8;
-        int j = 0;
-        for (int k = 0; k < 3; ++k) {
-            const PassCfg& pc = a.p[k];
-            const int nt = my_tiles(k);
-            for (int i = 0; i < nt; ++i, ++j) {
-                const long long t = blockIdx.x + (long long)i * G;
-                const int s = j % NS;
-                mbar_wait(&permd[s], (uint32_t)(j / NS) & 1u);
-                const uint32_t* buf = smem + s * stage_words;
-                if (pc.cross) {
-                    uint32_t* base = pc.out + t * h;
-#pragma unroll
-                    for (int c0 = 0; c0 < NV; c0 += CH) {
-                        uint4 vv[CH];
-#pragma unroll
-                        for (int u = 0; u < CH; ++u) {
-                            const int f = 4 * (sj + kWsStore * (c0 + u));
-                            const int pos = f >> logh, l = f & (h - 1);
-                            const uint32_t* src = buf + l * a.Ls + pos;
-                            vv[u].x = src[0];
-                            vv[u].y = src[a.Ls];
-                            vv[u].z = src[2 * a.Ls];
-                            vv[u].w = src[3 * a.Ls];
-                        }
-                        if (c0 + CH >= NV) mbar_arrive(&empty[s]);
-#pragma unroll
-                        for (int u = 0; u < CH; ++u) {
-                            const int f = 4 * (sj + kWsStore * (c0 + u));
-                            const int pos = f >> logh, l = f & (h - 1);
-                            st_v4(base + (long long)pos * pc.strideP + l, vv[u]);
-                        }
-                    }
-                } else {
-                    if (lead) {
-                        fence_proxy_async();
-                        uint32_t* dst = pc.out + t * h * (long long)L;
-                        if (dense) {
-                            bulk_s2g(dst, buf, (uint32_t)h * line_bytes);
-                        } else {
-                            for (int l = 0; l < h; ++l)
-                                bulk_s2g(dst + (long long)l * L, buf + l * a.Ls, line_bytes);
-                        }
-                        bulk_commit();
-                        bulk_wait_read0();
-                    }
-                    mbar_arrive(&empty[s]);
-                }
-            }
-            if (k < 2) {
-                // publish this CTA's pass-k stores to the grid
-                __threadfence();
-                named_bar(2, kWsStore);
-                if (lead) red_release_gpu_add(&a.sync[k], 1ull);
-            }
-            stamp_if(tr, lead, 4 + 4 * k);
-        }
-        if (lead) bulk_wait0();
-    }
-    __syncthreads();
-    if (tid == 0) {
-        __threadfence();
-        const unsigned long long old = atomicAdd(&a.sync[2], 1ull);
-        if (old == (unsigned long long)G - 1) {     // last CTA out: every spin has finished
-            a.sync[0] = 0;
-            a.sync[1] = 0;
-            a.sync[2] = 0;
-            __threadfence();
-        }
-    }
-    stamp(tr, 15);
-}
-
 // ------------------------------------------------------------------ TLC row pass (tile-level colouring)
 
 __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void* src, int c0, int c1, int c2) {
@@ -1327,9 +898,6 @@ struct TlcArgs {
     unsigned long long* trace;
     int prefetch_in;           // stream the whole input into L2 up front (HBM-resident input)
     TlcDecode dec;             // entry -> destination (plan.hpp)
-    int last_lsu;              // the CTA's last tile leaves through the permuters' 128-bit stores
-    int cw;                    // words per output chunk (tile-contiguous run in global memory)
-    long long cstride;         // global word stride between a tile's consecutive chunks
 };
 
 // Shared-memory word offsets of the TLC rings: A slots, then B slots, then mbarriers.
@@ -1499,7 +1067,6 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             for (int i = 0;; ++i) {
                 const long long t = blockIdx.x + (long long)i * G;
                 if (t >= a.ntiles) break;
-                if (a.last_lsu && t + G >= a.ntiles) break;     // the permuters store the last tile
                 const int s = i % NB;
                 mbar_wait(&R.bfull[s], (uint32_t)(i / NB) & 1u);
                 tlc_store(OUT, &tmap, a.out, R.B + (size_t)s * HL, t, HL, a.chunk, a.nbox, a.box_outer,
@@ -1550,21 +1117,6 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
             tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wq[0], a.dec, lc, &R.aempty[s],
                                       i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
-            if (a.last_lsu && t + G >= a.ntiles) {
-                // last tile: the 512 permuter threads store it (16 warps issue in parallel,
-                // shorter drain before the pass boundary than one TMA unit's 64-byte rows)
-                named_bar(1, kTlcPerm);
-                const uint4* B4 = reinterpret_cast<const uint4*>(R.B + (size_t)sb * HL);
-                const int pt = tid - 64;
-#pragma unroll
-                for (int m = 0; m < EPT / 4; ++m) {
-                    const int v = m * kTlcPerm + pt;           // 16-byte vector of the tile
-                    const int w = 4 * v;
-                    const long long g = (long long)(w / a.cw) * a.cstride + t * a.cw + (w % a.cw);
-                    st_v4(a.out + g, B4[v]);
-                }
-                break;
-            }
             mbar_arrive(&R.bfull[sb]);
 #pragma unroll
             for (int k = 0; k < AHEAD; ++k)
@@ -1752,6 +1304,150 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         }
     }
     stamp(tr, 15);
+}
+
+// ------------------------------------------------------------------ cluster path (n = 2^15..2^18)
+
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_size() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r));
+    return r;
+}
+// split cluster barrier: every thread of every block of the cluster arrives (release)
+// and later waits (acquire); work between the two halves overlaps the barrier
+__device__ __forceinline__ void cluster_arrive() {
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() {
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// shared::cta address -> the same offset in block `rank` of the cluster (shared::cluster)
+__device__ __forceinline__ uint32_t map_to(uint32_t cta_addr, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(cta_addr), "r"(rank));
+    return r;
+}
+// bulk copy of `bytes` from this block's shared memory to block `dst`'s (DSMEM), completion
+// (complete_tx) on the destination block's mbarrier
+__device__ __forceinline__ void bulk_s2cluster(uint32_t dst_cl, const void* src, uint32_t bytes, uint32_t mbar_cl) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst_cl),
+        "r"(smem_u32(src)), "r"(bytes), "r"(mbar_cl)
+        : "memory");
+}
+
+// One block's tile-coloured permute B[dst] = A[src] (full entry format):
+// warp-round m of warp `warp`: lane x reads A[32*sigma + x] (bank x) and writes B[dst];
+// the 32 dst of a round lie in 32 distinct banks (the tile colouring).
+template <int EPT, int LOGS>
+__device__ __forceinline__ void block_permute(const uint32_t* __restrict__ A, uint32_t* __restrict__ B,
+                                              const uint32_t* wc, int lane) {
+    constexpr int E = 2 * LOGS - 5;
+    constexpr uint32_t EMASK = (1u << E) - 1u;
+    constexpr uint32_t TMASK = (1u << LOGS) - 1u;
+    uint32_t v[EPT], d[EPT];
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) {
+        const int bit = m * E, w = bit >> 5, off = bit & 31;
+        uint32_t e;
+        if (off + E <= 32) e = (wc[w] >> off) & EMASK;
+        else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
+        v[m] = A[((e >> LOGS) << 5) | (uint32_t)lane];
+        d[m] = e & TMASK;
+    }
+#pragma unroll
+    for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
+}
+
+struct ClusterArgs {
+    const uint32_t* in;
+    uint32_t* out;
+    const uint32_t* sched[3];
+    long long tile_words;        // schedule words of one block's share of a phase
+};
+
+// Thm 9 (L537-L539) in ONE launch for arrays that fit in one cluster's shared memory
+// (NEXT-4; the single-SM permutation of the prior work, here spread over
+// the C <= 16 SMs of a cluster). Block g: three buffers of S words (buf0, buf1, buf2)
+// and three mbarriers. Phase 1 buf0 -> buf1 (send blocks); exchange 1: send block q ->
+// block q's buf2 at [g*Bw, ...) (DSMEM bulk copies, completion counted on block q's
+// mbarrier); phase 2 buf2 -> buf0; exchange 2: buf0 -> block q's buf1 (free once every
+// block has received exchange 1: split cluster barrier); phase 3 buf1 -> buf2 -> b.
+// Every permute hop is conflict-free in both banks (tile colouring).
+template <int EPT>
+__global__ void __launch_bounds__(kTlcPerm, 1) cluster_kernel(const ClusterArgs a) {
+    constexpr int S = kTlcPerm * EPT;
+    constexpr int LOGS = cilog2(S);
+    constexpr int E = 2 * LOGS - 5;
+    constexpr int NWORDS = (EPT * E + 31) / 32;
+    extern __shared__ __align__(128) uint32_t smem[];
+    uint32_t* buf0 = smem;
+    uint32_t* buf1 = smem + S;
+    uint32_t* buf2 = smem + 2 * S;
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 3 * S);   // [0] load, [1] exchange 1, [2] exchange 2
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const uint32_t g = cluster_rank(), C = cluster_size();
+    const uint32_t Bw = (uint32_t)S / C;                          // words per exchanged block
+    if (tid == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        mbar_init(&bar[2], 1);
+        fence_mbar_init();
+        // every byte this block will receive is announced before any peer can send
+        mbar_arrive_expect_tx(&bar[0], (uint32_t)S * 4u);
+        bulk_g2s(buf0, a.in + (size_t)g * S, (uint32_t)S * 4u, &bar[0]);
+        mbar_arrive_expect_tx(&bar[1], (uint32_t)S * 4u);
+        mbar_arrive_expect_tx(&bar[2], (uint32_t)S * 4u);
+    }
+    __syncthreads();
+    cluster_arrive();                       // (A) mbarriers initialised and armed
+    const uint32_t* sp = a.sched[0] + (size_t)g * a.tile_words + warp * NWORDS * 32 + lane;
+    uint32_t wc[NWORDS];
+#pragma unroll
+    for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+    mbar_wait(&bar[0], 0);
+    block_permute<EPT, LOGS>(buf0, buf1, wc, lane);               // phase 1
+    fence_proxy_async();                    // generic writes of buf1 -> the bulk copies' reads
+    sp = a.sched[1] + (size_t)g * a.tile_words + warp * NWORDS * 32 + lane;
+#pragma unroll
+    for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+    __syncthreads();
+    cluster_wait();                         // (A): every peer's mbarriers are armed
+    if (tid == 0) {
+        const uint32_t dst0 = smem_u32(buf2 + g * Bw), mb = smem_u32(&bar[1]);
+        for (uint32_t q = 0; q < C; ++q)
+            bulk_s2cluster(map_to(dst0, q), buf1 + q * Bw, Bw * 4u, map_to(mb, q));
+    }
+    mbar_wait(&bar[1], 0);                  // exchange 1 landed in buf2
+    cluster_arrive();                       // (B) my copies into buf2 are complete
+    block_permute<EPT, LOGS>(buf2, buf0, wc, lane);               // phase 2
+    fence_proxy_async();
+    sp = a.sched[2] + (size_t)g * a.tile_words + warp * NWORDS * 32 + lane;
+#pragma unroll
+    for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+    __syncthreads();
+    cluster_wait();                         // (B): every block received exchange 1 -> every buf1 is free
+    if (tid == 0) {
+        const uint32_t dst0 = smem_u32(buf1 + g * Bw), mb = smem_u32(&bar[2]);
+        for (uint32_t q = 0; q < C; ++q)
+            bulk_s2cluster(map_to(dst0, q), buf0 + q * Bw, Bw * 4u, map_to(mb, q));
+    }
+    mbar_wait(&bar[2], 0);                  // exchange 2 landed in buf1
+    cluster_arrive();                       // (C) my copies into buf1 are complete
+    block_permute<EPT, LOGS>(buf1, buf2, wc, lane);               // phase 3
+    fence_proxy_async();
+    __syncthreads();
+    if (tid == 0) {
+        bulk_s2g(a.out + (size_t)g * S, buf2, (uint32_t)S * 4u);
+        bulk_commit();
+        bulk_wait_read0();
+    }
+    cluster_wait();                         // (C): no peer still reads my buf0 before I exit
 }
 
 // ------------------------------------------------------------------ transpose
@@ -1968,40 +1664,16 @@ size_t tma_smem(const HostPlan& P, int f) {
                        : (size_t)3 * (g.L / 2) * 4 + (size_t)4 * kStgChunkWords * 4 + (3 + 2 * 4) * 8;
     if (rp.split) return (size_t)3 * (g.L / 2) * 4 + 3 * 8;
     const size_t stage = (size_t)rp.h * rp.Ls * 4 + (rp.sg ? 0 : (size_t)rp.h * g.wpl * 4);
-    return rp.stages * stage + rp.stages * 8 * (rp.tma == 2 ? 3 : 1);
+    return rp.stages * stage + rp.stages * 8;
 }
 
 template <int EPT>
-cudaError_t prep_ws(HostPlan& P, int f) {
-    RowPass& rp = P.rp[f];
-    const size_t smem = tma_smem(P, f);
-    cudaError_t e;
-    int nb = 0;
-    if (rp.out.cross) {
-        e = set_smem(row_pass_ws_kernel<EPT, true>, smem);
-        if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_ws_kernel<EPT, true>, rp.threads, smem);
-    } else {
-        e = set_smem(row_pass_ws_kernel<EPT, false>, smem);
-        if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, row_pass_ws_kernel<EPT, false>, rp.threads, smem);
-    }
-    if (e != cudaSuccess) return e;
-    if (nb < 1) return cudaErrorInvalidConfiguration;
-    const long long cap = (long long)nb * sm_count();
-    rp.grid = rp.ctas < cap ? rp.ctas : cap;
-    return cudaSuccess;
-}
-
-template <int EPT>
-const void* split_kernel_ptr(bool dense, bool keep) {
+const void* split_kernel_ptr(bool dense) {
     if constexpr (EPT < 8) {
         return nullptr;
     } else {
-        if (dense) return keep ? (const void*)row_pass_split_kernel<EPT, true, true>
-                               : (const void*)row_pass_split_kernel<EPT, true, false>;
-        return keep ? (const void*)row_pass_split_kernel<EPT, false, true>
-                    : (const void*)row_pass_split_kernel<EPT, false, false>;
+        return dense ? (const void*)row_pass_split_kernel<EPT, true, false>
+                     : (const void*)row_pass_split_kernel<EPT, false, false>;
     }
 }
 
@@ -2012,7 +1684,7 @@ const void* tma_kernel_ptr(bool cross, bool sg, bool split = false, bool dense =
         if (split && stg) return dense ? (const void*)row_pass_split_stg_kernel<EPT, true>
                                        : (const void*)row_pass_split_stg_kernel<EPT, false>;
     }
-    if (split) return split_kernel_ptr<EPT>(dense, keep);
+    if (split) return split_kernel_ptr<EPT>(dense);
     if (sg) return cross ? (const void*)row_pass_tma_kernel<EPT, true, true>
                          : (const void*)row_pass_tma_kernel<EPT, false, true>;
     return cross ? (const void*)row_pass_tma_kernel<EPT, true> : (const void*)row_pass_tma_kernel<EPT, false>;
@@ -2023,8 +1695,8 @@ cudaError_t set_tma_smem(bool cross, size_t smem) {
     cudaError_t e = set_smem(tma_kernel_ptr<EPT>(cross, false), smem);
     if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true), smem);
     if constexpr (EPT >= 8) {
-        for (int v = 0; v < 4 && e == cudaSuccess; ++v)
-            e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, v & 1, v >> 1), smem);
+        for (int v = 0; v < 2 && e == cudaSuccess; ++v)
+            e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, v & 1), smem);
     }
     if constexpr (EPT == 32 || EPT == 64) {
         if (e == cudaSuccess) e = set_smem(tma_kernel_ptr<EPT>(cross, true, true, false, false, true), smem);
@@ -2046,26 +1718,6 @@ cudaError_t grid_tma(HostPlan& P, int f) {
     if (nb < 1) return cudaErrorInvalidConfiguration;
     const long long cap = (long long)nb * sm_count();
     rp.grid = rp.ctas < cap ? rp.ctas : cap;
-    return cudaSuccess;
-}
-
-size_t fused3_smem(const HostPlan& P) {
-    const RowPass& rp = P.rp[0];
-    const PhaseGeom& g = P.ph[0];
-    const size_t stage = (size_t)rp.h * rp.Ls * 4 + (size_t)rp.h * (g.L / 32) * g.w64 * 8;
-    return rp.stages * stage + rp.stages * 8 * 3;
-}
-
-template <int EPT>
-cudaError_t prep_fused3(HostPlan& P) {
-    const size_t smem = fused3_smem(P);
-    cudaError_t e = set_smem(fused3_ws_kernel<EPT>, smem);
-    if (e != cudaSuccess) return e;
-    int nb = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fused3_ws_kernel<EPT>, 32 + kWsPerm + kWsStore, smem);
-    if (e != cudaSuccess) return e;
-    if (nb < 1) return cudaErrorInvalidConfiguration;
-    P.fused3_grid = sm_count();      // exactly one co-resident CTA per SM (grid barrier)
     return cudaSuccess;
 }
 
@@ -2204,13 +1856,6 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
     const dim3 grid((unsigned)tp.grid), block(64 + kTlcPerm);
     const size_t smem = tlc_smem(P, f);
     ta.dec = tp.dec;
-    {
-        static const char* env = std::getenv("PERM_TLC_LAST_LSU");
-        ta.last_lsu = env ? std::atoi(env) : 0;   // measured: no faster (explore_r01o)
-    }
-    if (tp.out_kind == 0) { ta.cw = tp.HL; ta.cstride = tp.HL; }
-    else if (tp.out_kind == 1) { ta.cw = (int)(h1 * h2); ta.cstride = P.r * h2; }
-    else { ta.cw = (int)(h3 * h2); ta.cstride = P.c * h3; }
     return tlc_dispatch(tp.ept, tp.E, [&](auto ept, auto E) {
         if (tp.out_kind == 0) return launch(row_pass_tlc_kernel<ept, 0, E>, grid, block, smem, s, pdl, map, ta);
         if (tp.out_kind == 1) return launch(row_pass_tlc_kernel<ept, 1, E>, grid, block, smem, s, pdl, map, ta);
@@ -2260,8 +1905,55 @@ cudaError_t launch_tlc_fused(const HostPlan& P, const CUtensorMap* maps, const u
     });
 }
 
+const void* cluster_kernel_ptr(int ept) {
+    switch (ept) {
+        case 4: return (const void*)cluster_kernel<4>;
+        case 8: return (const void*)cluster_kernel<8>;
+        case 16: return (const void*)cluster_kernel<16>;
+        case 32: return (const void*)cluster_kernel<32>;
+    }
+    return nullptr;
+}
+size_t cluster_smem(const HostPlan& P) { return (size_t)3 * P.tp[0].HL * 4 + 3 * 8; }
+
+cudaError_t launch_cluster(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
+                           uint32_t* b, cudaStream_t s) {
+    ClusterArgs ca{};
+    ca.in = a;
+    ca.out = b;
+    for (int f = 0; f < 3; ++f) ca.sched[f] = sched[f];
+    ca.tile_words = P.tp[0].tile_words;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)P.cluster);
+    cfg.blockDim = dim3(kTlcPerm);
+    cfg.dynamicSmemBytes = cluster_smem(P);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)P.cluster;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    switch (P.tp[0].ept) {
+        case 4: return cudaLaunchKernelEx(&cfg, cluster_kernel<4>, ca);
+        case 8: return cudaLaunchKernelEx(&cfg, cluster_kernel<8>, ca);
+        case 16: return cudaLaunchKernelEx(&cfg, cluster_kernel<16>, ca);
+        case 32: return cudaLaunchKernelEx(&cfg, cluster_kernel<32>, ca);
+    }
+    return cudaErrorInvalidValue;
+}
+
 cudaError_t prepare_kernels(HostPlan& P) {
     if (P.direct) return cudaSuccess;     // one stream kernel, no attributes to set
+    if (P.passes == 2) {
+        const void* k = cluster_kernel_ptr(P.tp[0].ept);
+        if (!k) return cudaErrorInvalidValue;
+        cudaError_t e = set_smem(k, cluster_smem(P));
+        if (e == cudaSuccess && P.cluster > 8)
+            e = cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        return e;
+    }
     if (P.layout == 3) return prep_tlc(P);
     cudaError_t e = cudaSuccess;
     auto set = [&](const void* k, size_t bytes) {
@@ -2270,14 +1962,6 @@ cudaError_t prepare_kernels(HostPlan& P) {
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     };
-    if (P.fused3) {
-        switch (P.rp[0].ept) {
-            case 8: return prep_fused3<8>(P);
-            case 16: return prep_fused3<16>(P);
-            case 32: return prep_fused3<32>(P);
-            default: return cudaErrorInvalidValue;
-        }
-    }
     if (P.passes == 1) {
         const size_t b = fused_smem(P);
         switch (P.fused_ept) {
@@ -2295,17 +1979,6 @@ cudaError_t prepare_kernels(HostPlan& P) {
     for (int f = 0; f < 3; ++f) {
         const int li = ilog2i(P.rp[f].ept);
         if (li < 2 || li > 6) return cudaErrorInvalidValue;
-        if (P.rp[f].tma == 2) {
-            switch (P.rp[f].ept) {
-                case 8: e = prep_ws<8>(P, f); break;
-                case 16: e = prep_ws<16>(P, f); break;
-                case 32: e = prep_ws<32>(P, f); break;
-                case 64: e = prep_ws<64>(P, f); break;
-                default: return cudaErrorInvalidValue;
-            }
-            if (e != cudaSuccess) return e;
-            continue;
-        }
         if (P.rp[f].tma) {
             size_t& nt = need_t[P.rp[f].out.cross ? 1 : 0][li];
             nt = nt > tma_smem(P, f) ? nt : tma_smem(P, f);
@@ -2387,29 +2060,6 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
     ra.seg_len = rp.seg_len;
     ra.seg_stride = rp.seg_stride;
     const dim3 block(rp.threads);
-    if (rp.tma == 2) {
-        WsArgs wa{};
-        wa.r = ra;
-        wa.ntiles = (int)rp.ctas;
-        wa.stages = rp.stages;
-        wa.data_words = rp.h * rp.Ls;
-        wa.sched_words = (int)ra.sched_words_per_cta;
-        const dim3 grid((unsigned)rp.grid);
-        const size_t smem = tma_smem(P, f);
-        const bool cx = rp.out.cross != 0;
-#define PERM_WS_CASE(E_)                                                                       \
-    case E_:                                                                                   \
-        return cx ? launch(row_pass_ws_kernel<E_, true>, grid, block, smem, s, pdl, wa)        \
-                  : launch(row_pass_ws_kernel<E_, false>, grid, block, smem, s, pdl, wa);
-        switch (rp.ept) {
-            PERM_WS_CASE(8)
-            PERM_WS_CASE(16)
-            PERM_WS_CASE(32)
-            PERM_WS_CASE(64)
-        }
-#undef PERM_WS_CASE
-        return cudaErrorInvalidValue;
-    }
     if (rp.tma) {
         TmaArgs ta{};
         ta.r = ra;
@@ -2430,12 +2080,10 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
             return cudaErrorInvalidValue;
         }
         if (rp.split) {
-            const bool dn = g.dense != 0, kp = rp.split_keep != 0;
+            const bool dn = g.dense != 0;
 #define PERM_SPLIT_CASE(E_)                                                                               \
     case E_:                                                                                              \
-        if (dn) return kp ? launch(row_pass_split_kernel<E_, true, true>, grid, block, smem, s, pdl, ta)    \
-                          : launch(row_pass_split_kernel<E_, true, false>, grid, block, smem, s, pdl, ta);  \
-        return kp ? launch(row_pass_split_kernel<E_, false, true>, grid, block, smem, s, pdl, ta)           \
+        return dn ? launch(row_pass_split_kernel<E_, true, false>, grid, block, smem, s, pdl, ta)           \
                   : launch(row_pass_split_kernel<E_, false, false>, grid, block, smem, s, pdl, ta);
             switch (rp.ept) {
                 PERM_SPLIT_CASE(8)
@@ -2474,55 +2122,11 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
     return cudaErrorInvalidValue;
 }
 
-cudaError_t launch_fused3(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
-                          uint32_t* x1, uint32_t* x2, uint32_t* b, unsigned long long* sync,
-                          cudaStream_t s, unsigned long long* trace) {
-    Fused3Args fa{};
-    const uint32_t* ins[3] = {a, x1, x2};
-    uint32_t* outs[3] = {x1, x2, b};
-    for (int f = 0; f < 3; ++f) {
-        const RowPass& rp = P.rp[f];
-        fa.p[f].in = ins[f];
-        fa.p[f].out = outs[f];
-        fa.p[f].sched = sched[f];
-        fa.p[f].ntiles = (int)rp.ctas;
-        fa.p[f].cross = rp.out.cross;
-        fa.p[f].strideP = rp.out.strideP;
-    }
-    const RowPass& r0 = P.rp[0];
-    const PhaseGeom& g = P.ph[0];
-    fa.logL = g.logL;
-    fa.logh = ilog2i(r0.h);
-    fa.Ls = r0.Ls;
-    fa.E = g.E;
-    fa.epw = g.epw;
-    fa.w64 = g.w64;
-    fa.stages = r0.stages;
-    fa.data_words = r0.h * r0.Ls;
-    fa.sched_words = (int)((long long)r0.h * (g.L / 32) * g.w64 * 2);
-    fa.sync = sync;
-    fa.trace = trace;
-    const dim3 grid((unsigned)P.fused3_grid), block(32 + kWsPerm + kWsStore);
-    const size_t smem = fused3_smem(P);
-    switch (r0.ept) {
-        case 8: return launch(fused3_ws_kernel<8>, grid, block, smem, s, false, fa);
-        case 16: return launch(fused3_ws_kernel<16>, grid, block, smem, s, false, fa);
-        case 32: return launch(fused3_ws_kernel<32>, grid, block, smem, s, false, fa);
-    }
-    return cudaErrorInvalidValue;
-}
-
-// 1 when the environment variable is set to something other than "0" (read once)
-static bool getenv_flag(const char* name) {
-    const char* e = std::getenv(name);
-    return e != nullptr && e[0] != '\0' && !(e[0] == '0' && e[1] == '\0');
-}
 
 cudaError_t launch_transpose(const uint32_t* in, uint32_t* out, int64_t rows, int64_t cols,
                              cudaStream_t s, bool pdl) {
     const dim3 grid((unsigned)(cols / 32), (unsigned)(rows / 32)), block(32, 8);
-    static const bool t32 = getenv_flag("PERM_TRANSPOSE32");   // A/B: the 32 x 32 kernel
-    if (rows >= 64 && cols >= 64 && !t32)
+    if (rows >= 64 && cols >= 64)
         return launch(transpose64_kernel, dim3((unsigned)(cols / 64), (unsigned)(rows / 64)), dim3(256), 0,
                       s, pdl, in, out, ilog2i(rows), ilog2i(cols));
     return launch(transpose_kernel, grid, block, 0, s, pdl, in, out, ilog2i(rows), ilog2i(cols));

@@ -17,17 +17,16 @@ cudaError_t prepare_kernels(HostPlan& P);   // also sets persistent grid sizes
 cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
                          uint32_t* b, cudaStream_t s);
 
+// Cluster path (n = 2^15..2^18): one launch of one cluster of P.cluster blocks; all three
+// phases in distributed shared memory, the column phase's transposes as block exchanges.
+cudaError_t launch_cluster(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
+                           uint32_t* b, cudaStream_t s);
+
 // One row pass (pass index f in 0..2) of the 3- or 5-pass pipeline.
 // `trace`: optional device buffer of 16 %globaltimer stamps per CTA (nullptr = off).
 cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, const uint32_t* in,
                             uint32_t* out, cudaStream_t s, bool pdl,
                             unsigned long long* trace = nullptr);
-
-// The three row passes of the LINES layout in one persistent launch (square
-// views). `sync`: 3 device u64 counters, zero-initialised once (self-resetting).
-cudaError_t launch_fused3(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
-                          uint32_t* x1, uint32_t* x2, uint32_t* b, unsigned long long* sync,
-                          cudaStream_t s, unsigned long long* trace = nullptr);
 
 // TLC layout: tensor maps of the intermediates (maps[0]: X1 for pass 1's 3-D
 // stores, maps[1]: X2 for pass 2's 4-D stores) and one pass launch.

@@ -75,7 +75,7 @@ struct RowPass {
     int32_t stages = 0;       // TMA ring depth
     int32_t sg = 0;           // 1 (tma == 1): schedule read from global (L2-prefetched), slots hold data only
     int32_t split = 0;        // 1 (tma == 1, sg, h == 1): ring of three half-line slots (L = 32768)
-    int32_t split_keep = 1;   // split: 1 = destinations kept in registers (512 threads), 0 = re-decoded
+    int32_t split_keep = 0;   // split: destinations re-decoded in the write hop (the only variant kept)
     int32_t split_stg = 0;    // split: 1 = W64 schedule streamed through smem chunks by a producer warp
     int64_t grid = 0;         // persistent CTAs (set at upload from the occupancy query)
     int32_t h = 0;            // lines per CTA (tile)
@@ -143,8 +143,9 @@ struct HostPlan {
     int64_t user_n = 0;        // elements of the caller
     int32_t k = 0;             // log2 n
     int64_t r = 0, c = 0;      // view
-    int32_t passes = 0;        // 1, 3, 5
-    int32_t layout = 0;        // 3-pass intermediates: 1 tiled, 2 lines (perm_layout)
+    int32_t passes = 0;        // 1, 3, 5; 2 = cluster path (one launch, DSMEM exchanges)
+    int32_t cluster = 0;       // cluster path: thread blocks in the cluster (C)
+    int32_t layout = 0;        // 3-pass intermediates: 1 tiled, 2 lines, 3 TLC; 4 = cluster path
     int32_t fused3 = 0;        // LINES layout, square view: all three passes in one launch
     TlcPass tp[3];             // layout TLC (3): the three passes
     // row-sharded plans: this rank owns rows [rank*r_l, +r_l) of a and b,

@@ -302,7 +302,6 @@ struct EulerColourer {
         }
         for (int64_t i = 0; i < E; ++i) { ord[i] = (uint32_t)i; pu[i] = U[i]; pv[i] = V[i]; }
         const int levels = ilog2(d);
-        static const bool seq_top = std::getenv("PERM_PLANNER_SEQ_TOP") != nullptr;
         static const bool verbose = std::getenv("PERM_PLANNER_VERBOSE") != nullptr;
         for (int lvl = 0; lvl < levels; ++lvl) {
             const int64_t G = int64_t(1) << lvl, S = E / G;
@@ -310,7 +309,7 @@ struct EulerColourer {
             // big groups: the chunked-pairing split (all threads inside one group). The choice
             // depends on S only, never on the thread count: every machine and every rank of a
             // sharded plan produces the same colouring.
-            if (!seq_top && parallel && S >= (int64_t(1) << 20)) {
+            if (parallel && S >= (int64_t(1) << 20)) {
                 for (int64_t g = 0; g < G; ++g) split_group_par(g * S, S, nodes);
             } else if (parallel && G > 1) {
 #pragma omp parallel
@@ -457,6 +456,80 @@ IoMode cross(int64_t blockP, int64_t strideP, int64_t cta_stride) {
 
 // ------------------------------------------------------------------ TLC layout
 
+// Colour every tile's bank graph (edge (src mod 32, dst mod 32) per element; the graph
+// is (HL/32)-regular because A and B are dense) and pack the entries in the TLC
+// bitstream format (plan.hpp TlcPass): colour = warp-round q, lane = source bank.
+// enum_tile(T, src, dst, tval) lists tile T's elements. W must be zeroed, sized
+// ntiles * tile_words. `bad` is set when an entry does not decode to its dst.
+template <class Enum>
+int colour_and_pack(const TlcPass& tp, bool gpu, Enum&& enum_tile, U32Buf& Wbuf, int& bad,
+                    std::string& err) {
+    const int64_t HL = tp.HL;
+    const int E = tp.E, ept = tp.ept, nwords = tp.nwords;
+    const TlcDecode dec = tp.dec;
+    Wbuf.assign((size_t)(tp.ntiles * tp.tile_words), 0u);
+    uint32_t* W = Wbuf.data();
+    std::vector<uint16_t> gcol;
+    if (gpu) {
+        // every tile's bank graph at once on the device (vertex (tile, offset mod 32))
+        const int64_t N = tp.ntiles * HL;
+        U16Buf ks((size_t)N), kd((size_t)N);
+#pragma omp parallel
+        {
+            std::vector<uint32_t> src((size_t)HL), dst((size_t)HL), tval((size_t)HL);
+#pragma omp for schedule(static)
+            for (int64_t T = 0; T < tp.ntiles; ++T) {
+                enum_tile(T, src.data(), dst.data(), tval.data());
+                for (int64_t x = 0; x < HL; ++x) {
+                    ks[T * HL + x] = (uint16_t)src[x];
+                    kd[T * HL + x] = (uint16_t)dst[x];
+                }
+            }
+        }
+        gcol.resize((size_t)N);
+        GpuPlanStats gs;
+        const cudaError_t ce = gpu_bank_colour(ks.data(), kd.data(), N, tp.logHL, gcol.data(), &gs);
+        if (ce != cudaSuccess) {
+            err = std::string("GPU planner (TLC bank colouring): ") + cudaGetErrorString(ce);
+            return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
+        }
+    }
+#pragma omp parallel reduction(| : bad)
+    {
+        EulerColourer ec;
+        std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL),
+            tval((size_t)HL);
+#pragma omp for schedule(dynamic, 1)
+        for (int64_t T = 0; T < tp.ntiles; ++T) {
+            enum_tile(T, src.data(), dst.data(), tval.data());
+            if (!gcol.empty()) {
+                for (int64_t x = 0; x < HL; ++x) col[x] = gcol[T * HL + x];
+            } else {
+                for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
+                ec.run(kW, HL / kW, HL, U.data(), V.data(), col.data(), false);
+            }
+            uint32_t* Wt = W + T * tp.tile_words;
+            for (int64_t x = 0; x < HL; ++x) {
+                const int64_t q = col[x];                 // warp-round
+                const int64_t lane = src[x] & 31;         // lane = source bank
+                const int64_t pw = q / ept, m = q % ept;
+                const uint32_t t = tval[x];
+                if (tlc_dst(dec, t, src[x]) != dst[x]) bad = 1;   // decode self-check
+                const uint64_t entry = ((uint64_t)(src[x] >> 5) << dec.lt) | t;
+                const int64_t bit = m * E;
+                const int64_t w = bit >> 5, off = bit & 31;
+                const uint64_t sh = entry << off;
+                uint32_t* base = Wt + (pw * nwords) * 32 + lane;
+                base[w * 32] |= (uint32_t)sh;
+                if (off + E > 32) base[(w + 1) * 32] |= (uint32_t)(sh >> 32);
+            }
+        }
+    }
+    return PERM_OK;
+}
+
+
+
 // Word offsets of the element (line, position) of tile T in the A / B buffers of
 // each TLC pass (see plan.hpp and DESIGN.md §5):
 //   X1 = [K][i][k_in] (K < c/h2, i < r, k_in < h2)   X2 = [I'][K][i_in'][k_in]
@@ -542,14 +615,10 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
         rp.ept = tp.ept; rp.threads = 64 + kTlcPerm; rp.Ls = P.ph[f].L;
     }
     // TMA tensor stores need 16-byte rows: h2 * 4 >= 16 (h2 >= 4 holds)
-    const int64_t NW = kTlcPerm / 32;
     for (int f = 0; f < 3; ++f) {
         const TlcPass& tp = P.tp[f];
-        P.sched[f].assign((size_t)(tp.ntiles * tp.tile_words), 0u);
-        uint32_t* W = P.sched[f].data();
         const uint16_t* ph = phi[f].data();
-        const int64_t HL = tp.HL, h = tp.h;
-        const int E = tp.E, ept = tp.ept, nwords = tp.nwords;
+        const int64_t h = tp.h;
         const TlcDecode dec = tp.dec;
         const bool full = dec.lt == tp.logHL && dec.s2 == 0 && dec.s3 == 0 && dec.m1 == 0;
         // element x of tile T: source offset in A, destination offset in B, entry payload
@@ -581,66 +650,93 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
                         }
                 }
         };
-        std::vector<uint16_t> gcol;
-        if (opt && opt->gpu_planner > 0) {
-            // every tile's bank graph at once on the device (vertex (tile, offset mod 32))
-            const int64_t N = tp.ntiles * HL;
-            U16Buf ks((size_t)N), kd((size_t)N);
-#pragma omp parallel
-            {
-                std::vector<uint32_t> src((size_t)HL), dst((size_t)HL), tval((size_t)HL);
-#pragma omp for schedule(static)
-                for (int64_t T = 0; T < tp.ntiles; ++T) {
-                    enum_tile(T, src.data(), dst.data(), tval.data());
-                    for (int64_t x = 0; x < HL; ++x) {
-                        ks[T * HL + x] = (uint16_t)src[x];
-                        kd[T * HL + x] = (uint16_t)dst[x];
-                    }
-                }
-            }
-            gcol.resize((size_t)N);
-            GpuPlanStats gs;
-            const cudaError_t ce = gpu_bank_colour(ks.data(), kd.data(), N, tp.logHL, gcol.data(), &gs);
-            if (ce != cudaSuccess) {
-                err = std::string("GPU planner (TLC bank colouring): ") + cudaGetErrorString(ce);
-                return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
-            }
-        }
         int bad = 0;
-#pragma omp parallel reduction(| : bad)
-        {
-            EulerColourer ec;
-            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL),
-                tval((size_t)HL);
-#pragma omp for schedule(dynamic, 1)
-            for (int64_t T = 0; T < tp.ntiles; ++T) {
-                enum_tile(T, src.data(), dst.data(), tval.data());
-                if (!gcol.empty()) {
-                    for (int64_t x = 0; x < HL; ++x) col[x] = gcol[T * HL + x];
-                } else {
-                    for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
-                    ec.run(kW, HL / kW, HL, U.data(), V.data(), col.data(), false);
-                }
-                uint32_t* Wt = W + T * tp.tile_words;
-                for (int64_t x = 0; x < HL; ++x) {
-                    const int64_t q = col[x];                 // warp-round
-                    const int64_t lane = src[x] & 31;         // lane = source bank
-                    const int64_t pw = q / ept, m = q % ept;
-                    const uint32_t t = tval[x];
-                    if (tlc_dst(dec, t, src[x]) != dst[x]) bad = 1;   // decode self-check
-                    const uint64_t entry = ((uint64_t)(src[x] >> 5) << dec.lt) | t;
-                    const int64_t bit = m * E;
-                    const int64_t w = bit >> 5, off = bit & 31;
-                    const uint64_t sh = entry << off;
-                    uint32_t* base = Wt + (pw * nwords) * 32 + lane;
-                    base[w * 32] |= (uint32_t)sh;
-                    if (off + E > 32) base[(w + 1) * 32] |= (uint32_t)(sh >> 32);
-                }
-            }
-        }
+        const int st = colour_and_pack(tp, opt && opt->gpu_planner > 0, enum_tile, P.sched[f], bad, err);
+        if (st != PERM_OK) return st;
         if (bad) { err = "TLC layout: internal error (entry decode mismatch)"; return PERM_ECUDA; }
     }
-    (void)NW;
+    return PERM_OK;
+}
+
+// ------------------------------------------------------------------ cluster path
+//
+// n <= 2^18 (NEXT-4: the whole array fits on chip): ONE launch of one
+// thread-block cluster of C blocks (DESIGN.md §5 "cluster path"). Block g holds
+// S = n/C words and owns rows [g*r_l, (g+1)*r_l) in phases 1 and 3, columns
+// [g*c_l, (g+1)*c_l) in phase 2 (r_l = r/C, c_l = c/C). Each phase is one
+// tile-coloured permute in the block's shared memory from its A buffer (input
+// order) to its B buffer (output order); the column phase's two transposes
+// (Lemma 8) become two exchanges of uniform Bw = r_l*c_l-word blocks over
+// distributed shared memory -- the row-sharded multi-GPU scheme
+// with DSMEM for NVLink:
+//   phase 1: A = rows of a (i_l*c + j);  B = send blocks, (i, k) at (k/c_l)*Bw + (k%c_l)*r_l + i%r_l
+//   exchange: send block q of block g -> block q's A at [g*Bw, (g+1)*Bw)
+//   phase 2: A = [sender][k_in][i_l];    B = send blocks, (i', k) at (i'/r_l)*Bw + (i'%r_l)*c_l + k%c_l
+//   exchange
+//   phase 3: A = [sender][i'_l][k_in];   B = rows of b (i'_l*c + k')
+int build_cluster(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt, std::string& err) {
+    const int64_t n = P.n, r = P.r, c = P.c;
+    int64_t C = (opt && opt->cluster > 0) ? opt->cluster : (n >= (int64_t(1) << 16) ? 16 : 8);
+    while (C > 1 && n / C > 16384) C *= 2;
+    const int64_t S = n / C;
+    if (C < 2 || C > 16 || (C & (C - 1)) || r % C || c % C || S < 2048 || S > 16384 ||
+        (r / C) * (c / C) < 4) {
+        err = "cluster path: needs a power-of-two cluster of 2..16 blocks with 2048..16384 words "
+              "per block (n = 2^15..2^18) and r, c divisible by it";
+        return PERM_EUNSUPPORTED;
+    }
+    P.passes = 2;
+    P.layout = 4;
+    P.cluster = (int32_t)C;
+    const int64_t rl = r / C, cl = c / C, Bw = rl * cl;
+    for (int f = 0; f < 3; ++f) {
+        TlcPass& tp = P.tp[f];
+        tp.h = (int32_t)(f == 1 ? cl : rl);
+        tp.HL = (int32_t)S;
+        tp.logHL = ilog2(S);
+        tp.ept = tp.HL / kTlcPerm;
+        tp.E = 2 * tp.logHL - 5;
+        tp.dec = TlcDecode{};
+        tp.dec.lt = tp.logHL;            // full format: entry = ((src >> 5) << log S) | dst
+        tp.nwords = (tp.ept * tp.E + 31) / 32;
+        tp.ntiles = C;
+        tp.tile_words = (int64_t)(kTlcPerm / 32) * tp.nwords * 32;
+        tp.stages = 0;
+        tp.bslots = 0;
+        RowPass& rp = P.rp[f];
+        rp.phase = f; rp.h = tp.h; rp.ctas = C; rp.ept = tp.ept; rp.threads = kTlcPerm; rp.Ls = P.ph[f].L;
+    }
+    for (int f = 0; f < 3; ++f) {
+        const TlcPass& tp = P.tp[f];
+        const uint16_t* ph = phi[f].data();
+        auto enum_tile = [&](int64_t g, uint32_t* src, uint32_t* dst, uint32_t* tval) {
+            for (int64_t s = 0; s < S; ++s) {
+                int64_t d;
+                if (f == 0) {
+                    const int64_t i_l = s / c, i = g * rl + i_l;
+                    const int64_t k = ph[i * c + s % c];
+                    d = (k / cl) * Bw + (k % cl) * rl + i_l;
+                } else if (f == 1) {
+                    const int64_t sender = s / Bw, rem = s % Bw;
+                    const int64_t k_in = rem / rl, i = sender * rl + rem % rl;
+                    const int64_t ip = ph[(g * cl + k_in) * r + i];
+                    d = (ip / rl) * Bw + (ip % rl) * cl + k_in;
+                } else {
+                    const int64_t sender = s / Bw, rem = s % Bw;
+                    const int64_t ip_l = rem / cl, k = sender * cl + rem % cl;
+                    const int64_t kp = ph[(g * rl + ip_l) * c + k];
+                    d = ip_l * c + kp;
+                }
+                src[s] = (uint32_t)s;
+                dst[s] = (uint32_t)d;
+                tval[s] = (uint32_t)d;
+            }
+        };
+        int bad = 0;
+        const int st = colour_and_pack(tp, opt && opt->gpu_planner > 0, enum_tile, P.sched[f], bad, err);
+        if (st != PERM_OK) return st;
+        if (bad) { err = "cluster path: internal error (entry decode mismatch)"; return PERM_ECUDA; }
+    }
     return PERM_OK;
 }
 
@@ -848,6 +944,11 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         g.wpl = (int64_t)(g.L / kW) * (g.dense ? g.E : g.w64 * 2);
         g.words = g.lines * g.wpl;
     }
+    if (passes == 2) {
+        const int st = build_cluster(P, phi, opt, err);
+        P.ms_bank = ms_since(t0);
+        return st;
+    }
     // 5-6. bank-level colouring of every line, packed (W64); not needed by TLC plans
     auto build_line_schedules = [&]() -> int {
         for (int f = 0; f < 3; ++f) {
@@ -950,8 +1051,8 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     constexpr int64_t kSmemBudget = 220 * 1024;
     int layout = opt ? opt->layout : 0;
     if (passes == 3) {
-        if (layout == 0) layout = (k <= 24) ? 2 : 1;
-        if (layout != 1 && layout != 2) { err = "layout must be 0, 1 or 2"; return PERM_EINVAL; }
+        if (layout == 0) layout = 1;
+        if (layout != 1) { err = "layout must be 0, 1 (TILED) or 3 (TLC)"; return PERM_EINVAL; }
     } else {
         layout = 0;
     }
@@ -978,31 +1079,6 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         d.phase = 2; d.h = (int32_t)h3; d.ctas = r / h3;
         d.in = runs(h2, h3 * h2, h3 * c);
         d.out = runs(c, 0, h3 * c);
-    } else if (passes == 3) {
-        // LINES: X1 column-major (c x r), X2 row-major; each pass reads whole lines.
-        for (int f = 0; f < 3; ++f) {
-            const int64_t lines_f = P.ph[f].lines, L = P.ph[f].L;
-            const bool cross_out = f < 2;
-            // default: 8 lines (32-byte column chunks = whole L2 sectors) when two
-            // stages fit, else 4
-            const int pad8 = cross_out ? 4 : 0;
-            int64_t h = pick(f, 2 * stage_bytes(8, f, pad8) <= kSmemBudget ? 8 : 4);
-            if (cross_out && h != 4 && h != 8) { err = "LINES layout: h1, h2 must be 4 or 8"; return PERM_EINVAL; }
-            if (h < 1 || h > lines_f || (h & (h - 1))) { err = "invalid h for the LINES layout"; return PERM_EINVAL; }
-            RowPass& rp = P.rp[f];
-            rp.phase = f; rp.h = (int32_t)h; rp.ctas = lines_f / h;
-            rp.in = runs(L, 0, h * L);
-            if (f == 0) rp.out = cross(1, r, h);          // X1[k*r + i]
-            else if (f == 1) rp.out = cross(1, c, h);     // X2[i'*c + k]
-            else rp.out = runs(c, 0, h * c);              // b rows
-            // warp-specialized kernel when the tile splits into 512 permuter threads
-            const int64_t ept = h * L / 512;
-            rp.tma = (h * L % 512 == 0 && ept >= 8 && ept <= 64) ? 2 : 1;
-            const int pad = (cross_out && h == 8) ? 4 : 0;
-            int st = (opt && opt->stages > 0) ? opt->stages
-                                              : (int)std::min<int64_t>(4, kSmemBudget / stage_bytes(h, f, pad));
-            rp.stages = std::max(1, st);
-        }
     } else {
         for (int f = 0; f < 3; ++f) {
             const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
@@ -1041,41 +1117,25 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         RowPass& rp = P.rp[f];
         const PhaseGeom& g = P.ph[rp.phase];
         if ((int64_t)rp.h * (g.L + 32) > 65535) { err = "tile exceeds 16-bit shared addresses; lower h"; return PERM_EINVAL; }
-        if (rp.tma == 2) {
-            rp.ept = (int32_t)((int64_t)rp.h * g.L / 512);
-            rp.threads = 32 + 512 + (rp.out.cross ? 256 : 0);
-        } else {
-            choose_threads(rp, g.L);
-            if (rp.split) {
-                // half-line ring variants (PERM_SPLIT): s512 [default] = W64 schedule streamed
-                // through shared-memory chunks (3.14 ms per pass at 2^30); r512 = 512 threads,
-                // the write hop re-reads the schedule (merged with the read hop's loads for
-                // W64 entries: 3.20 ms); r1024 = 1024 threads; k512 / k1024 = destinations
-                // kept in registers (spill: 4.8-5.4 ms). s512 falls back to r512 where the
-                // schedule words do not hold 2 entries (w64 != 16) or the format is dense.
-                const char* sv = std::getenv("PERM_SPLIT");
-                const std::string v = sv ? sv : "s512";
-                rp.split_keep = v[0] == 'k' ? 1 : 0;
-                // s512: the W64 schedule streamed through shared-memory chunks by TMA
-                // (needs 64-bit words holding 2 entries: w64 = 16)
-                const int64_t ept512 = (int64_t)rp.h * g.L / 512;
-                if (v == "s512" && (g.dense || g.w64 == 16) && (ept512 == 32 || ept512 == 64)) {
-                    rp.split_stg = 1;
-                    rp.threads = 512;
-                    rp.ept = (int32_t)ept512;
-                    goto split_done;
-                }
-                {
-                const int64_t T = (v.find("1024") != std::string::npos) ? 1024 : 512;
-                if ((int64_t)rp.h * g.L >= 8 * T) {
-                    rp.threads = (int32_t)T;
-                    rp.ept = (int32_t)((int64_t)rp.h * g.L / T);
-                } else if (rp.ept < 8) {
-                    rp.ept = 8;
-                    rp.threads = (int32_t)std::max<int64_t>(32, (int64_t)rp.h * g.L / 8);
-                }
-                }
-            split_done:;
+        choose_threads(rp, g.L);
+        if (rp.split) {
+            // half-line ring: the schedule streamed through shared-memory chunks by TMA
+            // (row_pass_split_stg_kernel, 512 threads) wherever its 64-bit W64 words hold
+            // 2 entries or the format is dense and a thread owns 32 or 64 elements (every
+            // default plan: L = 32768); otherwise (forced at small L for tests) 512
+            // threads re-decode the schedule from global memory in the write hop
+            rp.split_keep = 0;
+            const int64_t ept512 = (int64_t)rp.h * g.L / 512;
+            if ((g.dense || g.w64 == 16) && (ept512 == 32 || ept512 == 64)) {
+                rp.split_stg = 1;
+                rp.threads = 512;
+                rp.ept = (int32_t)ept512;
+            } else if ((int64_t)rp.h * g.L >= 8 * 512) {
+                rp.threads = 512;
+                rp.ept = (int32_t)ept512;
+            } else if (rp.ept < 8) {
+                rp.ept = 8;
+                rp.threads = (int32_t)std::max<int64_t>(32, (int64_t)rp.h * g.L / 8);
             }
         }
         if (rp.tma) {
@@ -1084,14 +1144,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
             const int pad = (rp.out.cross && rp.h == 8) ? 4 : 0;
             rp.Ls = g.L + pad;
             rp.conflicts_in = 1;   // bulk copies
-            if (rp.tma == 1) {
-                rp.conflicts_out = simulate_conflicts(rp, g, false);
-            } else {
-                // storer gather: 256 threads, vector f = 4*(j + 256*it)
-                RowPass tmp = rp;
-                tmp.threads = 256;
-                rp.conflicts_out = rp.out.cross ? simulate_conflicts(tmp, g, false) : 1;
-            }
+            rp.conflicts_out = simulate_conflicts(rp, g, false);
             if ((rp.h * g.wpl) % 4) { err = "TMA tile schedule is not 16-byte sized"; return PERM_EINVAL; }
             const int64_t sb = rp.split ? (int64_t)g.L / 2 * 4
                                : rp.sg ? (int64_t)rp.h * (g.L + pad) * 4 : stage_bytes(rp.h, rp.phase, pad);
@@ -1102,23 +1155,6 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
         } else {
             if ((int64_t)rp.h * g.L * 4 > 200 * 1024) { err = "a CTA's lines exceed the shared-memory budget"; return PERM_EINVAL; }
             choose_pad(rp, g);
-        }
-    }
-    // one persistent launch for all three passes: LINES layout, square view, and
-    // the three passes share tile shape, stride and pipeline depth
-    // auto (0) keeps three launches: measured faster at 2^22 on B200 so far
-    const int fuse = opt ? opt->fuse : 0;
-    if (passes == 3 && layout == 2 && fuse > 0 && r == c) {
-        const RowPass &a0 = P.rp[0], &a1 = P.rp[1], &a2 = P.rp[2];
-        const bool same = a0.tma == 2 && a1.tma == 2 && a2.tma == 2 && a0.h == a1.h &&
-                          a1.h == a2.h && a0.stages == a1.stages && a1.stages == a2.stages &&
-                          a0.ept == a1.ept && a1.ept == a2.ept && (a0.ept == 8 || a0.ept == 16 || a0.ept == 32);
-        if (same) {
-            P.fused3 = 1;
-            for (int f = 0; f < 3; ++f) {   // one shared slot layout (the CROSS stride)
-                P.rp[f].Ls = a0.Ls;
-                P.rp[f].threads = 32 + 512 + 256;
-            }
         }
     }
     return PERM_OK;

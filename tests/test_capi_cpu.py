@@ -64,7 +64,7 @@ def export_plan(lib, p, **kw):
 def test_cpp_plan_passes_oracle_checker(lib, fam, k):
     n = 1 << k
     p = W.make_perm(fam, n, seed=42 + k)
-    info, kappa, sched = export_plan(lib, p, layout=2 if k >= 15 else 0)   # per-line schedules
+    info, kappa, sched = export_plan(lib, p, passes=5 if k >= 15 else 0)   # per-line schedules
     r, c = W.view_shape(n)
     assert (info["rows"], info["cols"]) == (r, c)
     OC.assert_plan(p, kappa, sched, r, c, 32)
@@ -94,7 +94,7 @@ def test_cpp_plan_larger(lib, k):
     r, c = W.view_shape(n)
     for fam in ("random", "bitrev"):
         p = W.make_perm(fam, n)
-        _, kappa, sched = export_plan(lib, p, layout=2)
+        _, kappa, sched = export_plan(lib, p, passes=5)
         OC.assert_plan(p, kappa, sched, r, c, 32)
 
 
@@ -102,9 +102,9 @@ def test_cpp_plan_22_random(lib):
     n = 1 << 22
     r, c = W.view_shape(n)
     p = W.random(n, 42)
-    info, kappa, sched = export_plan(lib, p, layout=2)
+    info, kappa, sched = export_plan(lib, p, passes=5)
     OC.assert_plan(p, kappa, sched, r, c, 32)
-    assert info["passes"] == 3
+    assert info["passes"] == 5
     # W64 schedule: 17-bit entries, 3 per 64-bit word, 11 words per warp-round of 32
     assert info["entry_bits"] == [17, 17, 17]
     assert info["sched_bytes"] == 3 * ((n // 32) * 11 * 8 + 16)    # + 4 pad words per phase
@@ -257,7 +257,7 @@ def test_fp64_plan_is_the_word_pair_permutation(lib, k):
     # Table II(b) (L731-L755): 8-byte elements; element i = words (2i, 2i+1) -> 2P(i)+h
     n = 1 << k
     p = W.random(n, k)
-    with lib.Plan(p, elem_bytes=8, device=False, layout=2 if k >= 14 else 0) as pl:
+    with lib.Plan(p, elem_bytes=8, device=False, passes=5 if k >= 14 else 0) as pl:
         info = pl.info()
         kappa, sched = pl.export()
     assert info["elem_bytes"] == 8 and info["n"] == n
@@ -282,7 +282,7 @@ def test_planner_is_deterministic_across_thread_counts(lib):
     code = (
         "import sys, hashlib; sys.path.insert(0, %r)\n"
         "import workloads as W, paper_conf_icpp_kasagini13_b200 as P\n"
-        "pl = P.Plan(W.random(%d, 3), device=False, layout=2)\n"
+        "pl = P.Plan(W.random(%d, 3), device=False, passes=5)\n"
         "k, s = pl.export()\n"
         "print(hashlib.sha256(k.tobytes() + b''.join(x.tobytes() for x in s)).hexdigest())\n"
     ) % (ROOT, n)

@@ -88,22 +88,6 @@ def test_tile_shapes_tiled_layout(P, h):
     assert np.array_equal(b, OA.apply_ref(p, a))
 
 
-@pytest.mark.parametrize("k", [16, 18, 21, 22])
-@pytest.mark.parametrize("h,stages", [((4, 4, 4), 2), ((8, 8, 8), 2), ((4, 8, 16), 2), ((4, 4, 4), 3),
-                                      ((8, 4, 1), 1)])
-def test_tile_shapes_lines_layout(P, k, h, stages):
-    n = 1 << k
-    p = W.random(n, k)
-    a = W.make_data(n)
-    try:
-        b, info = run(P, p, a, passes=3, h=h, layout=2, stages=stages)
-    except P.PermError as e:
-        assert e.status == -1      # shared-memory budget / shape rejected up front
-        return
-    assert info["h"] == list(h)
-    assert np.array_equal(b, OA.apply_ref(p, a))
-
-
 @pytest.mark.parametrize("fam", W.FAMILIES)
 def test_config1_4M_all_families(P, fam):
     # BASELINE configs[1]: n = 2^22 float32, the five families of the paper (L373-L389)
@@ -230,7 +214,7 @@ def test_copy_kernel(P):
     assert torch.equal(a, b)
 
 
-@pytest.mark.parametrize("layout", [2, 3])
+@pytest.mark.parametrize("layout", [3])
 @pytest.mark.parametrize("k", [16, 18, 20, 22])
 def test_fused3_first_apply_and_graph_replay(P, k, layout):
     # the single-launch 3-pass kernel: grid barriers must hold on the FIRST apply of a
@@ -240,10 +224,7 @@ def test_fused3_first_apply_and_graph_replay(P, k, layout):
     p = W.random(n, 100 + k)
     a = W.make_data(n)
     ref = OA.apply_ref(p, a)
-    if layout == 2 and k < 18:
-        pytest.skip("LINES single-launch kernel needs tiles of >= 4096 elements")
-    h = (8, 8, 8) if layout == 2 else (0, 0, 0)
-    with P.Plan(p, layout=layout, h=h, fuse=1) as plan:
+    with P.Plan(p, layout=layout, fuse=1) as plan:
         info = plan.describe()
         da = dev(a)
         db = torch.full_like(da, -1)
@@ -262,7 +243,7 @@ def test_fused3_first_apply_and_graph_replay(P, k, layout):
             assert np.array_equal(host_words(db), ref)
 
 
-@pytest.mark.parametrize("layout", [1, 2, 3])
+@pytest.mark.parametrize("layout", [1, 3])
 @pytest.mark.parametrize("k", [16, 19, 20, 22])
 def test_every_layout(P, layout, k):
     n = 1 << k
@@ -426,21 +407,6 @@ def test_half_line_ring(P, fam, k):
             assert np.array_equal(host_words(db), OA.apply_ref(p, a)), fmt
 
 
-@pytest.mark.parametrize("variant", ["r1024", "k1024", "r512", "k512"])
-@pytest.mark.parametrize("k", [22, 26])
-def test_half_line_ring_variants(P, variant, k, monkeypatch):
-    # register strategies of the half-line ring (PERM_SPLIT, read at plan build), both
-    # schedule formats
-    monkeypatch.setenv("PERM_SPLIT", variant)
-    n = 1 << k
-    p = W.random(n, 70 + k)
-    a = W.make_data(n)
-    ref = OA.apply_ref(p, a)
-    for fmt in (-1, 2):
-        b, _ = run(P, p, a, passes=5, no_tma=-2, sched_format=fmt)
-        assert np.array_equal(b, ref), (variant, fmt)
-
-
 @pytest.mark.parametrize("k", [19, 21])
 @pytest.mark.parametrize("fam", ["random", "transpose", "bitrev"])
 def test_tall_views_5pass(P, k, fam):
@@ -455,10 +421,9 @@ def test_tall_views_5pass(P, k, fam):
 
 @pytest.mark.parametrize("k,log2c", [(19, 14), (20, 15), (21, 15)])
 @pytest.mark.parametrize("fam", ["random", "bitrev"])
-def test_half_line_ring_staged_schedule(P, k, log2c, fam, monkeypatch):
-    # PERM_SPLIT=s512: the half-line ring with the W64 schedule streamed through shared
-    # memory in TMA chunks (lines of 16384 / 32768 words via wide views, L603)
-    monkeypatch.setenv("PERM_SPLIT", "s512")
+def test_half_line_ring_staged_schedule(P, k, log2c, fam):
+    # the half-line ring with the schedule streamed through shared memory in TMA chunks
+    # (lines of 16384 / 32768 words via wide views, L603)
     n = 1 << k
     p = W.make_perm(fam, n, seed=k + log2c)
     a = W.make_data(n)
@@ -474,3 +439,34 @@ def test_half_line_ring_staged_schedule(P, k, log2c, fam, monkeypatch):
             plan.apply(da, db)
             torch.cuda.synchronize()
             assert np.array_equal(host_words(db), ref), fmt
+
+
+@pytest.mark.parametrize("fam", W.FAMILIES)
+@pytest.mark.parametrize("k,C", [(15, 8), (15, 16), (16, 8), (16, 16), (17, 16), (18, 16), (16, 2), (17, 4)])
+def test_cluster_path(P, fam, k, C):
+    # NEXT-4: one launch of one thread-block cluster; the column phase's
+    # transposes are DSMEM block exchanges; bit-exact against the definition
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=k * C)
+    a = W.make_data(n)
+    try:
+        b, info = run(P, p, a, passes=2, cluster=C)
+    except P.PermError as e:
+        # a cluster of C blocks with 3 * n/C words each must fit the GPU (C = 2: 2^16 only)
+        assert e.status in (-1, -3), e
+        return
+    assert info["passes"] == 2 and info["kernels_per_apply"] == 1
+    assert np.array_equal(b, OA.apply_ref(p, a)), (fam, k, C)
+
+
+def test_cluster_path_fp64_and_replay(P):
+    n = 1 << 16
+    p = W.random(n, 77)
+    a = W.make_data(n, elem_bytes=8)
+    with P.Plan(p, elem_bytes=8, passes=2, direct=-1) as plan:
+        da = torch.from_numpy(a.view(np.int32)).cuda()
+        db = torch.full_like(da, -1)
+        for _ in range(3):                       # repeated launches (fresh shared memory each)
+            plan.apply(da, db)
+        torch.cuda.synchronize()
+        assert np.array_equal(db.cpu().numpy().view(np.uint64), OA.apply_ref(p, a))
