@@ -17,8 +17,9 @@ e2e        = the same metric through perm_apply_host (pinned host a -> device ->
 roofline   = dominant kernel: algorithmic bytes per launch (read n*4 + write n*4 +
              schedule n*E/8) / its mean event-timed duration, vs MEASURED_PEAKS hbm_gbs
 cpu_baseline = the oracle's plain C loop (oracle/c/apply_ref.c, all host cores)
-N > 1      = independent replicas, one per GPU (the 2^22 workload does not shard;
-             "scaling": "weak"); rank 0 prints the JSON line.
+N > 1      = the row-sharded path: one 2^22 shard per GPU ("scaling": "weak"),
+             perm_apply_sharded (libperm kernels + two NCCL all-to-alls); rank 0 prints the
+             JSON line with the stage times, NVLink fraction and the bare all-to-all.
 """
 from __future__ import annotations
 
@@ -58,6 +59,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--sharded", action="store_true",
+                    help="run the row-sharded path even at N = 1 (a one-rank NCCL communicator)")
     ap.add_argument("--no-c3", action="store_true",
                     help="skip the n = 2^26 random side measurement (BASELINE configs[2])")
     return ap.parse_args()
@@ -193,40 +196,44 @@ def run_reference(args):
 
 
 def run_sharded(args, rank, world, local):
-    """N > 1: the row-sharded path on n = 2^log2n * N elements (each GPU
-    holds a 2^log2n shard: weak scaling). Rows stay local for phases 1 and 3; the
-    column phase runs as two NCCL all-to-all exchanges (torch.distributed, NVLink)."""
+    """N > 1 (or --sharded): the row-sharded path on n = 2^log2n * N elements
+    (each GPU holds a 2^log2n shard: weak scaling) through libperm's C ABI
+    (perm_apply_sharded: R1 + T-pack, NCCL all-to-all, R2 + T-pack, all-to-all, R3; the
+    NCCL communicator is created from a unique id broadcast over torch.distributed).
+    Also reported: each stage's device time, the all-to-all's NVLink fraction, the bare
+    all-to-all of the same size (the exchange alone: the achievable ceiling), and t_apply
+    against T_HBM + T_NVL (no overlap) and max(T_HBM, T_NVL) (perfect overlap)."""
     import torch
     import torch.distributed as dist
     import paper_conf_icpp_kasagini13_b200 as pkg
-    from paper_conf_icpp_kasagini13_b200.sharded import ShardedApply
+    from paper_conf_icpp_kasagini13_b200.sharded import sharded_plan
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
     ntot = (1 << args.log2n) * world
     shard = ntot // world
     fams = args.families.split(",")
     flush = torch.empty(FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
-    runs, bufs, build_ms = {}, {}, {}
+    peaks = measured_peaks()
+    bufs, build_ms = {}, {}
     for f in fams:
         p = W.make_perm(f, ntot)
         a = W.make_data(ntot)
         t0 = time.perf_counter()
-        pl = pkg.Plan(p, world=world, rank=rank)
+        pl = sharded_plan(p, direct=-1)
         build_ms[f] = (time.perf_counter() - t0) * 1e3
         a_sh = torch.from_numpy(a[rank * shard:(rank + 1) * shard].view(np.int32).copy()).to(dev)
-        bufs[f] = (pl, a_sh, torch.empty_like(a_sh), torch.empty_like(a_sh), torch.empty_like(a_sh),
-                   p[rank * shard:(rank + 1) * shard], a)
-        runs[f] = ShardedApply(pl)
-    def one(f):
-        pl, a_sh, b_sh, send, recv = bufs[f][:5]
-        runs[f](a_sh, b_sh, send, recv, stream)
+        bufs[f] = (pl, a_sh, torch.empty_like(a_sh), torch.empty_like(a_sh), torch.empty_like(a_sh), p, a)
+
+    def flush_l2():
+        flush.zero_()
+        flush.sum()
+
     for _ in range(max(args.warmup, 3)):
         for f in fams:
-            one(f)
+            bufs[f][0].apply_sharded(bufs[f][1], bufs[f][2], stream)
     torch.cuda.synchronize()
-    # bit-exactness of this rank's shard for the last family (numpy b[p] = a on the host)
     f = fams[-1]
-    ref = scatter_np(W.make_perm(f, ntot), bufs[f][6])[rank * shard:(rank + 1) * shard]
+    ref = scatter_np(bufs[f][5], bufs[f][6])[rank * shard:(rank + 1) * shard]
     ok = bool(np.array_equal(bufs[f][2].cpu().numpy().view(np.uint32), ref))
     evs = {f: [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                for _ in range(args.steps)] for f in fams}
@@ -235,33 +242,82 @@ def run_sharded(args, rank, world, local):
     with ClockSampler(local) as clocks:
         for s in range(args.steps):
             for f in fams:
-                flush.zero_()
-                flush.sum()
+                flush_l2()
                 dist.barrier()
                 evs[f][s][0].record(stream)
-                one(f)
+                bufs[f][0].apply_sharded(bufs[f][1], bufs[f][2], stream)
                 evs[f][s][1].record(stream)
         torch.cuda.synchronize()
     dist.barrier()
     step_ms = [sum(evs[f][s][0].elapsed_time(evs[f][s][1]) for f in fams) for s in range(args.steps)]
-    t = torch.tensor([statistics.mean(step_ms)], device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+
+    # stage breakdown of one apply (steps and exchanges between events; same buffers)
+    f = fams[0]
+    pl, a_sh, b_sh, send, recv = bufs[f][:5]
+    stages = []
+    for _ in range(max(3, args.steps // 2)):
+        flush_l2()
+        dist.barrier()
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
+        ev[0].record(stream)
+        pl.sharded_step(0, a_sh, send, stream); ev[1].record(stream)
+        pl.sharded_exchange(send, recv, stream); ev[2].record(stream)
+        pl.sharded_step(1, recv, send, stream); ev[3].record(stream)
+        pl.sharded_exchange(send, recv, stream); ev[4].record(stream)
+        pl.sharded_step(2, recv, b_sh, stream); ev[5].record(stream)
+        torch.cuda.synchronize()
+        stages.append([ev[i].elapsed_time(ev[i + 1]) for i in range(5)])
+    st_ms = [statistics.median(x[i] for x in stages) for i in range(5)]
+    # bare all-to-all of the same size, back to back (the achievable exchange ceiling)
+    ts = []
+    for _ in range(max(5, args.steps)):
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        pl.sharded_exchange(send, recv, stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    bare_ms = statistics.median(ts)
+
+    vals = torch.tensor([statistics.mean(step_ms), bare_ms] + st_ms, device=dev)
+    dist.all_reduce(vals, op=dist.ReduceOp.MAX)
     okt = torch.tensor([1 if ok else 0], device=dev)
     dist.all_reduce(okt, op=dist.ReduceOp.MIN)
-    ms_per_step = float(t.item())
+    ms_per_step, bare_ms = float(vals[0]), float(vals[1])
+    st_ms = [float(x) for x in vals[2:]]
     value = len(fams) * 2 * ntot * 4 / (ms_per_step * 1e-3) / 1e9
     if rank == 0:
+        nvl_peak = 900.0                                    # GB/s per direction (NVLink 5 spec)
+        xbytes = (world - 1) * (shard // world) * 4         # sent (= received) per GPU per exchange
+        info = pl.info()
+        desc = pl.describe()
+        sb = sched_bytes_per_elt(info, desc)
+        local_bytes = shard * (5 * 8 + sum(sb))             # R1, T, R2, T, R3 + schedules
+        t_hbm = local_bytes / (peaks["hbm_gbs"] * 1e9) * 1e3
+        t_nvl = 2 * xbytes / (nvl_peak * 1e9) * 1e3
+        t_apply = ms_per_step / len(fams)
         cfg = workload_config(args)
         cfg["workload"] = (f"row-sharded n=2^{args.log2n}*{world} float32 (raw u32 words), one "
-                           f"2^{args.log2n} shard per GPU, families {'/'.join(fams)}, NCCL all-to-all")
+                           f"2^{args.log2n} shard per GPU, families {'/'.join(fams)}, "
+                           f"perm_apply_sharded (libperm kernels + NCCL send/recv)")
         cfg["n"] = ntot
-        cfg["parallelism"] = f"row-sharded x{world} (NCCL all_to_all_single, 2 exchanges per apply)"
+        cfg["parallelism"] = f"row-sharded x{world} (2 NCCL all-to-alls per apply)"
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": cfg, "bitexact_check_all_ranks": bool(okt.item()),
                 "plan_build_ms_rank0": build_ms,
-                "exchange_bytes_per_apply_per_gpu": 2 * (world - 1) * (ntot // (world * world)) * 4,
+                "stage_ms": dict(zip(["R1+Tpack", "all-to-all 1", "R2+Tpack", "all-to-all 2", "R3"], st_ms)),
+                "exchange_bytes_per_gpu": xbytes,
+                "nvlink_frac": [(xbytes / (st_ms[i] * 1e-3) / 1e9) / nvl_peak if world > 1 else None
+                                for i in (1, 3)],
+                "bare_alltoall_ms": bare_ms,
+                "bare_alltoall_nvlink_frac": (xbytes / (bare_ms * 1e-3) / 1e9) / nvl_peak if world > 1 else None,
+                "t_apply_ms": t_apply,
+                "ideal_ms": {"T_HBM": t_hbm, "T_NVL": t_nvl, "no_overlap": t_hbm + t_nvl,
+                             "perfect_overlap": max(t_hbm, t_nvl)},
+                "nvlink_peak_gbs": nvl_peak, "hbm_peak_gbs": peaks["hbm_gbs"],
                 "gpu_launches": args.steps * len(fams) * 5,
                 "clocks": clocks.summary()}
         print(json.dumps(line), flush=True)
@@ -374,8 +430,10 @@ def main():
 
     rank, world, local = dist_env()
     torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if world > 1 or args.sharded:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local), rank=rank, world_size=world)
         return run_sharded(args, rank, world, local)
     import paper_conf_icpp_kasagini13_b200 as pkg
 
@@ -546,8 +604,14 @@ def main():
         with open(tpath) as fh:
             tj = json.load(fh)
         traffic = tj.get(f"n{args.log2n}", {}).get(kinds[dom])
+    # second fraction: the kernel's measured DRAM bytes (ncu dram__bytes
+    # read + write per launch, profiles/ncu_traffic.json) over the same duration -- what
+    # the HBM actually moved; at 2^22 the intermediates stay in the 126 MB L2, so this is
+    # below the algorithmic fraction
+    frac_dram = (traffic / (mean_k[dom] * 1e-3) / 1e9 / peaks["hbm_gbs"]) if traffic else None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / peaks["hbm_gbs"], "traffic": traffic,
+                "frac_algorithmic": achieved / peaks["hbm_gbs"], "frac_dram": frac_dram,
                 "kernel": kinds[dom], "kernel_ms": mean_k[dom],
                 "algorithmic_bytes_per_launch": alg[dom], "peak_source": peaks["_source"],
                 "per_kernel_ms": dict(zip([f"{k}#{i}" for i, k in enumerate(kinds)], mean_k)),
@@ -621,6 +685,12 @@ def main():
             "conventional_us": {f: 1e3 * conv[f] for f in fams},
             "s_designated_us": {f: 1e3 * gather[f] for f in fams},
             "speedup_vs_conventional": {f: conv[f] * 1e3 / per_fam_us[f] for f in fams},
+            "speedup_vs_s_designated": {f: gather[f] * 1e3 / per_fam_us[f] for f in fams},
+            # whole apply against the HBM roofline of its minimum traffic (read a, write b,
+            # read the three schedules once; SURVEY §8(d) "minimum-traffic fraction")
+            "apply_min_traffic_frac": {f: (2 * n * 4 + infos[f]["sched_bytes"]) / (per_fam_us[f] * 1e-6)
+                                          / 1e9 / peaks["hbm_gbs"] for f in sched_fams
+                                       if not infos[f]["direct"]},
             "effective_gbs": {f: 2 * n * 4 / (per_fam_us[f] * 1e-6) / 1e9 for f in fams},
             "plan_build_ms": build_ms,
             "sched_bytes": info["sched_bytes"],
