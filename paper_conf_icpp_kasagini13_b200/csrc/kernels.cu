@@ -1403,6 +1403,10 @@ __global__ void __launch_bounds__(kTlcPerm, 1) cluster_kernel(const ClusterArgs 
         bulk_g2s(buf0, a.in + (size_t)g * S, (uint32_t)S * 4u, &bar[0]);
         mbar_arrive_expect_tx(&bar[1], (uint32_t)S * 4u);
         mbar_arrive_expect_tx(&bar[2], (uint32_t)S * 4u);
+        // phases 2 and 3 read their schedules after the exchanges: pull them into L2 now,
+        // in the same HBM round trip as a and phase 1's schedule
+        for (int f = 1; f < 3; ++f)
+            prefetch_l2_bulk(a.sched[f] + (size_t)g * a.tile_words, (uint32_t)(a.tile_words * 4));
     }
     __syncthreads();
     cluster_arrive();                       // (A) mbarriers initialised and armed
