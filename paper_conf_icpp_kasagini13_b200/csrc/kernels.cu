@@ -833,6 +833,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
             mbar_arrive(&empty[b]);
             if (tid == 0 && g + NB < total_chunks) {
                 mbar_wait(&empty[b], (uint32_t)((g / NB) & 1));   // all 512 consumed chunk g
+                fence_proxy_async();   // their generic reads of the buffer -> the TMA refill
                 issue_chunk(g + NB);
             }
         }
@@ -1017,6 +1018,11 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     TlcRing R(smem, HL, NA, NB);
     unsigned long long* tr = a.trace;
     stamp(tr, 0);
+    if (tr != nullptr && tid == 0) {          // trace slot 15: the SM this CTA runs on
+        unsigned smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        tr[blockIdx.x * 16 + 15] = smid;
+    }
     if (tid == 0) R.init(NA, NB);
     __syncthreads();
 
@@ -1344,9 +1350,13 @@ __device__ __forceinline__ void bulk_s2cluster(uint32_t dst_cl, const void* src,
 // One block's tile-coloured permute B[dst] = A[src] (full entry format):
 // warp-round m of warp `warp`: lane x reads A[32*sigma + x] (bank x) and writes B[dst];
 // the 32 dst of a round lie in 32 distinct banks (the tile colouring).
+// With `self` (a block index) the destinations in send block `self` go straight to `Bself`
+// (the buffer that block's exchange would have delivered them to: no copy to oneself);
+// B and Bself are 128-byte aligned, so a destination keeps its bank either way.
 template <int EPT, int LOGS>
 __device__ __forceinline__ void block_permute(const uint32_t* __restrict__ A, uint32_t* __restrict__ B,
-                                              const uint32_t* wc, int lane) {
+                                              const uint32_t* wc, int lane, uint32_t* Bself = nullptr,
+                                              uint32_t self = 0, int logBw = 0) {
     constexpr int E = 2 * LOGS - 5;
     constexpr uint32_t EMASK = (1u << E) - 1u;
     constexpr uint32_t TMASK = (1u << LOGS) - 1u;
@@ -1360,8 +1370,13 @@ __device__ __forceinline__ void block_permute(const uint32_t* __restrict__ A, ui
         v[m] = A[((e >> LOGS) << 5) | (uint32_t)lane];
         d[m] = e & TMASK;
     }
+    if (Bself) {
 #pragma unroll
-    for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
+        for (int m = 0; m < EPT; ++m) ((d[m] >> logBw) == self ? Bself : B)[d[m]] = v[m];
+    } else {
+#pragma unroll
+        for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
+    }
 }
 
 struct ClusterArgs {
@@ -1385,61 +1400,86 @@ __global__ void __launch_bounds__(kTlcPerm, 1) cluster_kernel(const ClusterArgs 
     constexpr int LOGS = cilog2(S);
     constexpr int E = 2 * LOGS - 5;
     constexpr int NWORDS = (EPT * E + 31) / 32;
+    constexpr int TW = (kTlcPerm / 32) * NWORDS * 32;              // schedule words per block and phase
+    // up to 8192 words per block the three phases' schedules ride in shared memory (one TMA
+    // round trip with a); beyond, they are read from global memory (L2-prefetched)
+    constexpr bool SMEM_SCHED = EPT <= 16;
     extern __shared__ __align__(128) uint32_t smem[];
     uint32_t* buf0 = smem;
     uint32_t* buf1 = smem + S;
     uint32_t* buf2 = smem + 2 * S;
-    uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 3 * S);   // [0] load, [1] exchange 1, [2] exchange 2
+    uint32_t* sch = smem + 3 * S;                                   // [3][TW] when SMEM_SCHED
+    // [0] a (+ phase-1 schedule), [1] exchange 1, [2] exchange 2, [3] phases 2-3 schedules
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 3 * S + (SMEM_SCHED ? 3 * TW : 0));
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const uint32_t g = cluster_rank(), C = cluster_size();
     const uint32_t Bw = (uint32_t)S / C;                          // words per exchanged block
+    const int logBw = 31 - __clz((int)Bw);
+    const uint32_t rx_bytes = ((uint32_t)S - Bw) * 4u;            // received from the C-1 peers
     if (tid == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
-        mbar_init(&bar[2], 1);
+        for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);
         fence_mbar_init();
         // every byte this block will receive is announced before any peer can send
-        mbar_arrive_expect_tx(&bar[0], (uint32_t)S * 4u);
-        bulk_g2s(buf0, a.in + (size_t)g * S, (uint32_t)S * 4u, &bar[0]);
-        mbar_arrive_expect_tx(&bar[1], (uint32_t)S * 4u);
-        mbar_arrive_expect_tx(&bar[2], (uint32_t)S * 4u);
-        // phases 2 and 3 read their schedules after the exchanges: pull them into L2 now,
-        // in the same HBM round trip as a and phase 1's schedule
-        for (int f = 1; f < 3; ++f)
-            prefetch_l2_bulk(a.sched[f] + (size_t)g * a.tile_words, (uint32_t)(a.tile_words * 4));
+        mbar_arrive_expect_tx(&bar[1], rx_bytes);
+        mbar_arrive_expect_tx(&bar[2], rx_bytes);
+        if constexpr (SMEM_SCHED) {
+            mbar_arrive_expect_tx(&bar[0], (uint32_t)(S + TW) * 4u);
+            bulk_g2s(buf0, a.in + (size_t)g * S, (uint32_t)S * 4u, &bar[0]);
+            bulk_g2s(sch, a.sched[0] + (size_t)g * TW, (uint32_t)TW * 4u, &bar[0]);
+            mbar_arrive_expect_tx(&bar[3], (uint32_t)(2 * TW) * 4u);
+            bulk_g2s(sch + TW, a.sched[1] + (size_t)g * TW, (uint32_t)TW * 4u, &bar[3]);
+            bulk_g2s(sch + 2 * TW, a.sched[2] + (size_t)g * TW, (uint32_t)TW * 4u, &bar[3]);
+        } else {
+            mbar_arrive_expect_tx(&bar[0], (uint32_t)S * 4u);
+            bulk_g2s(buf0, a.in + (size_t)g * S, (uint32_t)S * 4u, &bar[0]);
+            // phases 2 and 3 read their schedules after the exchanges: pull them into L2 now,
+            // in the same HBM round trip as a and phase 1's schedule
+            for (int f = 1; f < 3; ++f) prefetch_l2_bulk(a.sched[f] + (size_t)g * TW, (uint32_t)TW * 4u);
+        }
     }
     __syncthreads();
     cluster_arrive();                       // (A) mbarriers initialised and armed
-    const uint32_t* sp = a.sched[0] + (size_t)g * a.tile_words + warp * NWORDS * 32 + lane;
     uint32_t wc[NWORDS];
+    // lane's schedule words of phase f: coalesced (word w of lane x at (warp*NWORDS + w)*32 + x)
+    auto load_sched = [&](int f) {
+        if constexpr (SMEM_SCHED) {
+            const uint32_t* sp = sch + f * TW + warp * NWORDS * 32 + lane;
 #pragma unroll
-    for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+            for (int w = 0; w < NWORDS; ++w) wc[w] = sp[w * 32];
+        } else {
+            const uint32_t* sp = a.sched[f] + (size_t)g * TW + warp * NWORDS * 32 + lane;
+#pragma unroll
+            for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+        }
+    };
+    if constexpr (!SMEM_SCHED) load_sched(0);
     mbar_wait(&bar[0], 0);
-    block_permute<EPT, LOGS>(buf0, buf1, wc, lane);               // phase 1
+    if constexpr (SMEM_SCHED) load_sched(0);
+    block_permute<EPT, LOGS>(buf0, buf1, wc, lane, buf2, g, logBw);   // phase 1 (own block -> buf2)
     fence_proxy_async();                    // generic writes of buf1 -> the bulk copies' reads
-    sp = a.sched[1] + (size_t)g * a.tile_words + warp * NWORDS * 32 + lane;
-#pragma unroll
-    for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+    if constexpr (!SMEM_SCHED) load_sched(1);
     __syncthreads();
     cluster_wait();                         // (A): every peer's mbarriers are armed
     if (tid == 0) {
         const uint32_t dst0 = smem_u32(buf2 + g * Bw), mb = smem_u32(&bar[1]);
         for (uint32_t q = 0; q < C; ++q)
-            bulk_s2cluster(map_to(dst0, q), buf1 + q * Bw, Bw * 4u, map_to(mb, q));
+            if (q != g) bulk_s2cluster(map_to(dst0, q), buf1 + q * Bw, Bw * 4u, map_to(mb, q));
+    }
+    if constexpr (SMEM_SCHED) {
+        mbar_wait(&bar[3], 0);
+        load_sched(1);
     }
     mbar_wait(&bar[1], 0);                  // exchange 1 landed in buf2
     cluster_arrive();                       // (B) my copies into buf2 are complete
-    block_permute<EPT, LOGS>(buf2, buf0, wc, lane);               // phase 2
+    block_permute<EPT, LOGS>(buf2, buf0, wc, lane, buf1, g, logBw);   // phase 2 (own block -> buf1)
     fence_proxy_async();
-    sp = a.sched[2] + (size_t)g * a.tile_words + warp * NWORDS * 32 + lane;
-#pragma unroll
-    for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + w * 32);
+    load_sched(2);
     __syncthreads();
     cluster_wait();                         // (B): every block received exchange 1 -> every buf1 is free
     if (tid == 0) {
         const uint32_t dst0 = smem_u32(buf1 + g * Bw), mb = smem_u32(&bar[2]);
         for (uint32_t q = 0; q < C; ++q)
-            bulk_s2cluster(map_to(dst0, q), buf0 + q * Bw, Bw * 4u, map_to(mb, q));
+            if (q != g) bulk_s2cluster(map_to(dst0, q), buf0 + q * Bw, Bw * 4u, map_to(mb, q));
     }
     mbar_wait(&bar[2], 0);                  // exchange 2 landed in buf1
     cluster_arrive();                       // (C) my copies into buf1 are complete
@@ -1918,7 +1958,12 @@ const void* cluster_kernel_ptr(int ept) {
     }
     return nullptr;
 }
-size_t cluster_smem(const HostPlan& P) { return (size_t)3 * P.tp[0].HL * 4 + 3 * 8; }
+size_t cluster_smem(const HostPlan& P) {
+    // three S-word buffers, the three phases' schedules when a thread owns <= 16 elements,
+    // four mbarriers (cluster_kernel)
+    const TlcPass& tp = P.tp[0];
+    return (size_t)3 * tp.HL * 4 + (tp.ept <= 16 ? (size_t)3 * tp.tile_words * 4 : 0) + 4 * 8;
+}
 
 cudaError_t launch_cluster(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
                            uint32_t* b, cudaStream_t s) {

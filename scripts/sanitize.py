@@ -30,7 +30,7 @@ CASES = [
     ("row_pass_split_kernel (re-decoding half-line ring)", 16, dict(passes=5, no_tma=-2, sched_format=-1)),
     ("row_pass_kernel (plain) + transpose", 16, dict(passes=5, no_tma=1)),
     ("row_pass_kernel TILED layout", 16, dict(passes=3, layout=1)),
-    ("transpose_kernel 32x32 (view side 32)", 10, dict(passes=5)),
+    ("transpose_kernel 32x32 (view side 32)", 11, dict(passes=5)),
 ]
 
 fails = 0

@@ -7,6 +7,7 @@ import paper_conf_icpp_kasagini13_b200 as P
 ap = argparse.ArgumentParser()
 ap.add_argument('--log2n', type=int, default=22)
 ap.add_argument('--cfg', default='{}')
+ap.add_argument('--dump', default='', help='save the raw per-CTA stamps (npz)')
 a = ap.parse_args()
 n = 1 << a.log2n
 p = W.random(n, 42)
@@ -20,8 +21,11 @@ for _ in range(3):
     flush.zero_(); flush.sum(); plan.apply(da, db)
 torch.cuda.synchronize()
 tr = plan.trace().astype(np.int64)
+if a.dump:
+    np.savez(a.dump, trace=tr, describe=json.dumps(plan.describe()))
 d = plan.describe()
-t0 = tr[tr > 0].min()
+ts_ = tr[:, :, :15]
+t0 = ts_[ts_ > 0].min()          # slot 15 holds the SM id, not a time
 names = {0: 'start', 1: 'pdl_ok', 2: 'w0', 3: 'p0', 4: 's0', 5: 'w1', 6: 'p1', 7: 's1', 8: 'w2', 9: 'p2', 10: 's2', 14: 'end'}
 print(json.dumps(kw), 'passes', d['passes'], 'layout', d.get('layout'), 'fused3', d.get('fused3'))
 if d.get('fused3'):
