@@ -52,7 +52,7 @@ enum perm_status {
 enum perm_passes {
     PERM_PASSES_AUTO  = 0,
     PERM_PASSES_FUSED = 1,   /* n <= 2^14: all three phases inside one CTA's shared memory */
-    PERM_PASSES_CLUSTER = 2, /* n = 2^15..2^18: ONE launch; the array lives in the shared memory
+    PERM_PASSES_CLUSTER = 2, /* n = 2^15..2^18 (default 2^15..2^17): ONE launch; the array lives in the shared memory
                                 of one thread-block cluster (2..16 blocks); the column phase's
                                 two transposes become block exchanges over distributed shared
                                 memory (DSMEM bulk copies); a and b cross HBM once each */
@@ -105,8 +105,7 @@ typedef struct {
                             labelling), -1 = host threads (planner.cpp), 0 = auto (device for
                             device plans with n >= 2^20, host otherwise) */
     int32_t cluster;     /* cluster path (passes = 2): thread blocks per cluster, a power of two
-                            in 2..16; 0 = 16 for n >= 2^16, else 8 (raised until a block holds
-                            <= 16384 words) */
+                            in 2..16; 0 = 16 (raised never; a block must hold 2048..16384 words) */
 } perm_plan_options;
 
 typedef struct {

@@ -676,7 +676,7 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
 //   phase 3: A = [sender][i'_l][k_in];   B = rows of b (i'_l*c + k')
 int build_cluster(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt, std::string& err) {
     const int64_t n = P.n, r = P.r, c = P.c;
-    int64_t C = (opt && opt->cluster > 0) ? opt->cluster : (n >= (int64_t(1) << 16) ? 16 : 8);
+    int64_t C = (opt && opt->cluster > 0) ? opt->cluster : 16;
     while (C > 1 && n / C > 16384) C *= 2;
     const int64_t S = n / C;
     if (C < 2 || C > 16 || (C & (C - 1)) || r % C || c % C || S < 2048 || S > 16384 ||
@@ -923,7 +923,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     int passes = opt ? opt->passes : 0;
     // measured on B200: fused CTA to 2^14, TLC 3-pass 2^15..2^25 (LINES /
     // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^26
-    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 25 ? 3 : 5);
+    // cluster path (one launch, DSMEM exchanges) for 2^15..2^17: 8.3 / 10.0 / 12.5 us vs the
+    // three TLC launches' 13.5 / 14.0 / 14.8 us (profiles/r02_small_n.jsonl)
+    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 17 ? 2 : (k <= 25 ? 3 : 5));
     // dense schedule bitstreams only where the 5-pass row kernels read them
     const bool dense_phases = passes == 5 && !(opt && opt->sched_format < 0);
     // geometry of the three phases
