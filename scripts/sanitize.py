@@ -33,8 +33,11 @@ CASES = [
     ("transpose_kernel 32x32 (view side 32)", 11, dict(passes=5)),
 ]
 
+only = sys.argv[1] if len(sys.argv) > 1 else ""      # substring filter on the case name
 fails = 0
 for name, k, kw in CASES:
+    if only and only not in name:
+        continue
     n = 1 << k
     p = W.random(n, k)
     a = W.make_data(n)
@@ -47,6 +50,9 @@ for name, k, kw in CASES:
     fails += not ok
     print(f"{name:55s} n=2^{k}: {'ok' if ok else 'MISMATCH'}", flush=True)
 
+if only:
+    print("ALL OK" if fails == 0 else f"{fails} FAILURES", flush=True)
+    sys.exit(1 if fails else 0)
 # sharded steps (G = 2 virtual ranks on this device) and the baselines / shortcut kernels
 from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
 n, G = 1 << 16, 2
