@@ -659,6 +659,7 @@ __global__ void __launch_bounds__((EPT >= 64) ? 512 : 1024, 1) row_pass_split_ke
             }
         } else {
             bulk_g2s(dst, a.r.in + t * (long long)L + (long long)q * HALF, half_bytes, &bars[slot]);
+            if (q == 0) prefetch_l2_bulk(a.r.in + t * (long long)L + HALF, half_bytes);
         }
     };
 
@@ -756,14 +757,31 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
     const int w64 = a.r.w64;
     const int chunks_per_line = EPT / 4;         // (L/32 rounds) / 64 rounds per chunk
 
+    // half q of line i -> slot j % 3. With the first half, the line's second half is pulled
+    // into L2: its TMA load can only be issued once the previous line's first half has been
+    // stored out of its slot, and then it hits L2 instead of HBM. Sharded column phases
+    // (in_segs > 1): a line is in_segs segments of seg_len <= L/2 words, one per sender.
     auto issue_half = [&](long long j) {
         const long long i = j >> 1;
         if (i >= my_lines) return;
         const int q = (int)(j & 1), slot = (int)(j % 3);
         const long long t = blockIdx.x + i * G;
+        uint32_t* dst = smem + slot * HALF;
         mbar_arrive_expect_tx(&bars[slot], half_bytes);
         if (q == 0) prefetch_l2_bulk(a.r.sched + t * a.sched_words, (uint32_t)a.sched_words * 4u);
-        bulk_g2s(smem + slot * HALF, a.r.in + t * (long long)L + (long long)q * HALF, half_bytes, &bars[slot]);
+        if (a.r.in_segs > 1) {
+            const uint32_t sb = (uint32_t)a.r.seg_len * 4u;
+            for (int g = 0; g < a.r.in_segs; ++g) {
+                const long long off = (long long)g * a.r.seg_len;
+                const uint32_t* src = a.r.in + g * a.r.seg_stride + t * a.r.seg_len;
+                if ((off >> lh) == q) bulk_g2s(dst + (off & (HALF - 1)), src, sb, &bars[slot]);
+                else if (q == 0) prefetch_l2_bulk(src, sb);
+            }
+        } else {
+            const uint32_t* src = a.r.in + t * (long long)L;
+            bulk_g2s(dst, src + (long long)q * HALF, half_bytes, &bars[slot]);
+            if (q == 0) prefetch_l2_bulk(src + HALF, half_bytes);
+        }
     };
 
     unsigned long long* tr = a.r.trace;

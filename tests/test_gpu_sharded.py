@@ -133,3 +133,32 @@ def test_apply_sharded_errors(P):
     with P.Plan(p) as pl:                                   # unsharded plan
         with pytest.raises(P.PermError):
             pl.apply_sharded(x, y)
+
+
+@pytest.mark.parametrize("G", [2, 4])
+@pytest.mark.parametrize("sched_format", [0, -1])
+def test_virtual_ranks_half_line_ring(P, G, sched_format):
+    # the C4 kernels (lines of 32768 words: the half-line ring, staged dense schedule chunks
+    # or re-decoded W64 entries) with segmented column-phase input (one segment per sender),
+    # at small n through a wide view (L603): 128 x 32768, rows sharded G ways
+    from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
+    n = 1 << 22
+    shard = n // G
+    a = W.make_data(n)
+    for fam in ("random", "bitrev"):
+        p = W.make_perm(fam, n, seed=G)
+        plans = [P.Plan(p, world=G, rank=g, log2c=15, no_tma=-2, sched_format=sched_format) for g in range(G)]
+        try:
+            d = plans[0].describe()
+            assert any(rp["split"] == 1 and rp["L"] == 32768 for rp in d["row_passes"]), d
+            a_sh = [torch.from_numpy(a[g * shard:(g + 1) * shard].view(np.int32).copy()).cuda() for g in range(G)]
+            b_sh = [torch.full((shard,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
+            send = [torch.empty(shard, dtype=torch.int32, device="cuda") for _ in range(G)]
+            recv = [torch.empty(shard, dtype=torch.int32, device="cuda") for _ in range(G)]
+            apply_virtual(plans, a_sh, b_sh, send, recv)
+            torch.cuda.synchronize()
+            b = np.concatenate([x.cpu().numpy().view(np.uint32) for x in b_sh])
+            assert np.array_equal(b, OA.apply_ref(p, a)), (fam, G, sched_format)
+        finally:
+            for pl in plans:
+                pl.close()
