@@ -749,7 +749,9 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
     uint32_t* cbuf = smem + 3 * HALF;
     uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + NB * CWS);
     uint64_t* full = bars + 3;                   // chunk landed
-    uint64_t* empty = bars + 3 + NB;             // chunk consumed by all 512 threads
+    // chunk buffer b's consumption count (warps; monotone): the warp whose arrival completes
+    // a multiple of 16 refills the buffer itself -- no thread blocks waiting for the others
+    uint32_t* consumed = reinterpret_cast<uint32_t*>(bars + 3 + NB);
     const int G = gridDim.x;
     const uint32_t half_bytes = (uint32_t)HALF * 4u;
     const long long my_lines = a.ntiles > (int)blockIdx.x ? (a.ntiles - 1 - (int)blockIdx.x) / G + 1 : 0;
@@ -790,7 +792,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
         for (int s = 0; s < 3; ++s) mbar_init(&bars[s], 1);
         for (int b = 0; b < NB; ++b) {
             mbar_init(&full[b], 1);
-            mbar_init(&empty[b], kStgWorkers);
+            consumed[b] = 0;
         }
         fence_mbar_init();
         if (my_lines > 0) prefetch_l2_bulk(a.r.sched + (long long)blockIdx.x * a.sched_words,
@@ -848,11 +850,23 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
                 if (m & 1) ta[m >> 1] |= ad << 16;
                 else ta[m >> 1] = ad;
             }
-            mbar_arrive(&empty[b]);
-            if (tid == 0 && g + NB < total_chunks) {
-                mbar_wait(&empty[b], (uint32_t)((g / NB) & 1));   // all 512 consumed chunk g
-                fence_proxy_async();   // their generic reads of the buffer -> the TMA refill
-                issue_chunk(g + NB);
+            if (c == 0 && i > 0 && tid == 0) {
+                // line i-1's second half (slot s1 of line i-1 = the slot of line i+1's first
+                // half) was handed to its TMA store at the end of line i-1; by now it has been
+                // read out, so this wait no longer holds warp 0 back at the line boundary
+                bulk_wait_read0();
+                fence_proxy_async();
+                issue_half(2 * i + 2);
+            }
+            __syncwarp();                     // the warp's reads of chunk g precede lane 0's release
+            if (lane == 0 && g + NB < total_chunks) {
+                uint32_t old;
+                asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
+                             : "=r"(old) : "r"(smem_u32(&consumed[b])) : "memory");
+                if ((old + 1) % kW == 0) {       // the last of the 16 warps to consume chunk g
+                    fence_proxy_async();         // all warps' generic reads -> the TMA refill
+                    issue_chunk(g + NB);
+                }
             }
         }
         __syncthreads();
@@ -869,10 +883,9 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
             bulk_commit();
             bulk_wait_read1();
             fence_proxy_async();
-            issue_half(2 * i + 3);
-            bulk_wait_read0();
-            fence_proxy_async();
-            issue_half(2 * i + 4);
+            issue_half(2 * i + 3);           // second half of line i+1 -> slot s0
+            // the first half of line i+2 (-> slot s1, once the second store has read it) is
+            // issued by thread 0 after its first schedule chunk of line i+1
         }
         if (i < 4) stamp(tr, 4 + 3 * (int)i);
     }
