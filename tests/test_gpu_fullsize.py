@@ -63,3 +63,22 @@ def test_default_plan_full_size(P, k, fam):
         pytest.fail(f"2^{k} {fam}: {bad.size} mismatching words, first at {bad[:8].tolist()}")
     del b, ref
     gc.collect()
+
+
+def test_fp64_large(P):
+    # Table II(b) at scale: 2^28 8-byte elements = 2^29 words (the tall-view 5-pass plan)
+    n = 1 << 28
+    p = W.random(n, 7)
+    a = W.make_data(n, elem_bytes=8)
+    with P.Plan(p, elem_bytes=8) as plan:
+        info = plan.info()
+        assert info["passes"] == 5 and info["elem_bytes"] == 8
+        da = torch.from_numpy(a.view(np.int32)).cuda()
+        db = torch.full_like(da, -1)
+        plan.apply(da, db)
+        torch.cuda.synchronize()
+        del da
+        b = db.cpu().numpy().view(np.uint64)
+        del db
+    torch.cuda.empty_cache()
+    assert np.array_equal(b, OA.apply_ref(p, a))
