@@ -316,6 +316,20 @@ int perm_sharded_step(const perm_plan* plan, int32_t step, const void* in, void*
     const uint32_t* src = static_cast<const uint32_t*>(in);
     uint32_t* dst = static_cast<uint32_t*>(out);
     cudaError_t e;
+    if (P.layout == 3) {
+        // TLC form: one tile-coloured pass per step, writing the exchange layout directly
+        // (step 0: X1 of my rows = per-peer column blocks; step 1: X2 of my columns = per-peer
+        // row blocks; step 2: rows of b) and reading received tiles as one segment per sender
+        if (step < 0 || step > 2) return fail(PERM_EINVAL, "step must be 0, 1 or 2");
+        alignas(64) CUtensorMap maps[3];
+        if (step < 2) {
+            e = perm::make_tlc_maps(P, dst, dst, maps);
+            if (e != cudaSuccess) return cuda_fail(e, "cuTensorMapEncodeTiled (sharded)");
+        }
+        e = perm::launch_tlc_pass(P, step, maps, plan->d_phase[step], src, dst, s, false, nullptr);
+        if (e != cudaSuccess) return cuda_fail(e, "sharded step launch");
+        return PERM_OK;
+    }
     if (step == 0) {          // R1 on my rows, then T-pack: (r_l x c) -> (c x r_l), peer q = rows q*c_l..
         e = perm::launch_row_pass(P, 0, plan->d_phase[0], src, plan->d_scratch[0], s, false);
         if (e == cudaSuccess) e = perm::launch_transpose(plan->d_scratch[0], dst, P.r_l, P.c, s, true);
@@ -533,7 +547,8 @@ int perm_plan_run_pass(const perm_plan* plan, int32_t pass, const void* in, void
     if (!plan) return fail(PERM_EINVAL, "null plan");
     if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
     const HostPlan& P = plan->host;
-    if (P.layout != 3 || P.fused3 || plan->d_p) return fail(PERM_EUNSUPPORTED, "run_pass needs a 3-launch TLC plan");
+    if (P.layout != 3 || P.fused3 || plan->d_p || P.r_l)
+        return fail(PERM_EUNSUPPORTED, "run_pass needs an unsharded 3-launch TLC plan");
     if (pass < 0 || pass > 2) return fail(PERM_EINVAL, "pass must be 0, 1 or 2");
     if (!in) {
         if (pass == 0) return fail(PERM_EINVAL, "pass 0 needs an input buffer");

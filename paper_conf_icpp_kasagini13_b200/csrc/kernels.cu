@@ -929,6 +929,8 @@ struct TlcArgs {
     int nbox, box_outer, box_words;
     unsigned long long* trace;
     int prefetch_in;           // stream the whole input into L2 up front (HBM-resident input)
+    int segs;                  // > 1: tile t = segs segments of seg_len words (sharded, plan.hpp)
+    long long seg_len, seg_stride;
     TlcDecode dec;             // entry -> destination (plan.hpp)
 };
 
@@ -1083,7 +1085,13 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 if (i >= NA) mbar_wait(&R.aempty[s], (uint32_t)(i / NA - 1) & 1u);
                 fence_proxy_async();           // permuters' generic reads of the slot -> TMA write
                 mbar_arrive_expect_tx(&R.afull[s], (uint32_t)HL * 4u);
-                bulk_g2s(R.A + (size_t)s * HL, a.in + t * HL, (uint32_t)HL * 4u, &R.afull[s]);
+                if (a.segs > 1) {              // one segment per sender, in sender order
+                    for (int g = 0; g < a.segs; ++g)
+                        bulk_g2s(R.A + (size_t)s * HL + g * a.seg_len, a.in + g * a.seg_stride + t * a.seg_len,
+                                 (uint32_t)a.seg_len * 4u, &R.afull[s]);
+                } else {
+                    bulk_g2s(R.A + (size_t)s * HL, a.in + t * HL, (uint32_t)HL * 4u, &R.afull[s]);
+                }
                 if (i == 0) pdl_launch_dependents();
                 if (a.prefetch_in) {
                     prefetch_sched(i + sched_ahead);
@@ -1874,6 +1882,8 @@ cudaError_t make_tlc_maps(const HostPlan& P, uint32_t* x1, uint32_t* x2, CUtenso
     }
     const cuuint64_t r = (cuuint64_t)P.r, c = (cuuint64_t)P.c;
     const cuuint64_t h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
+    // row-sharded plans: a rank's X1 holds its r/world rows, its X2 its c/world columns
+    const cuuint64_t rX1 = P.r_l ? (cuuint64_t)P.r_l : r, cX2 = P.c_l ? (cuuint64_t)P.c_l : c;
     std::memset(maps, 0, 3 * sizeof(CUtensorMap));
     // Maps whose box rows are a tile's contiguous chunks (64 bytes at h1*h2 = 16 words; at
     // most 256 words per row): a 16-byte innermost box dimension makes the TMA unit emit
@@ -1881,7 +1891,7 @@ cudaError_t make_tlc_maps(const HostPlan& P, uint32_t* x1, uint32_t* x2, CUtenso
     //   X1 = [K][i][k_in]: K-blocks of r*h2 words; pass-1 tile t writes [t*h1*h2, +h1*h2) of each
     //   X2 = [I'][K][i_in'][k_in]: I'-blocks of c*h3 words; pass-2 tile K writes [K*h3*h2, +h3*h2)
     const cuuint64_t ch[2] = {h1 * h2, h3 * h2};
-    const cuuint64_t blk[2] = {r * h2, c * h3};
+    const cuuint64_t blk[2] = {rX1 * h2, cX2 * h3};
     const cuuint64_t nblk[2] = {c / h2, r / h3};
     void* base[2] = {x1, x2};
     for (int m = 0; m < 2; ++m) {
@@ -1913,6 +1923,9 @@ cudaError_t launch_tlc_pass(const HostPlan& P, int f, const CUtensorMap* maps, c
     ta.tile_words = tp.tile_words;
     ta.trace = trace;
     ta.prefetch_in = (f == 0) ? 1 : 0;   // pass 1 reads `a` from HBM; later passes read L2-resident X
+    ta.segs = tp.segs;
+    ta.seg_len = tp.seg_len;
+    ta.seg_stride = tp.seg_stride;
     const long long h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
     if (tp.out_kind == 1) {
         const long long outer = P.c / h2, bo = outer < 256 ? outer : 256;

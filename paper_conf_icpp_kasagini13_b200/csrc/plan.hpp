@@ -134,6 +134,10 @@ struct TlcPass {
     int32_t stages = 0;       // A slots (TMA loads in flight); B slots = bslots
     int32_t bslots = 0;       // B slots (permuted tiles waiting for / under their TMA store)
     int64_t grid = 0;         // persistent CTAs (set at upload)
+    // row-sharded TLC: a tile arrives as `segs` segments of seg_len words, one
+    // per sender, at in + s*seg_stride + t*seg_len (segs = 1: the tile is in[t*HL, +HL))
+    int32_t segs = 1;
+    int64_t seg_len = 0, seg_stride = 0;
 };
 
 struct HostPlan {

@@ -1168,12 +1168,67 @@ int build_sharded_plan(const int32_t* p, int64_t n, int32_t eb, int32_t world, i
         err = "world must be a power of two and 0 <= rank < world";
         return PERM_EINVAL;
     }
-    // the global plan with per-line schedules (5-pass geometry: whole lines)
     perm_plan_options o{};
     if (opt) o = *opt;
+    o.direct = -1;                      // the shortcut is a single-device kernel
+    // TLC form (the column phase's transposes absorbed into the tile-coloured passes, so a
+    // step is ONE kernel and the exchange buffers are written / read directly): every rank
+    // holds whole tiles of every pass. The send buffers then have exactly the single-GPU
+    // X1 / X2 layouts with r -> r/world (X1) and c -> c/world (X2), and a received tile is
+    // world segments, one per sender. Otherwise the per-line 5-pass form
+    // (R1 + transpose, R2 + transpose, R3), e.g. at 2^26..2^30 or when options ask for it.
+    const bool tlc_wanted = (o.passes == 0 || o.passes == 3) && (o.layout == 0 || o.layout == 3) &&
+                            o.no_tma == 0 && o.fuse <= 0;
+    if (tlc_wanted) {
+        const int64_t nw = (eb == 8 ? 2 : 1) * n;
+        int kk = 0;
+        while ((int64_t(1) << kk) < nw) ++kk;
+        if (kk >= 15 && kk <= 25) {
+            perm_plan_options ot = o;
+            ot.passes = 3;
+            ot.layout = 3;
+            HostPlan T;
+            std::string e2;
+            int st = build_host_plan(p, n, eb, &ot, T, e2);
+            if (st != PERM_OK) { err = e2; return st; }
+            const int64_t r = T.r, c = T.c;
+            const int64_t h1 = T.tp[0].h, h2 = T.tp[1].h, h3 = T.tp[2].h;
+            if (T.layout == 3 && r % world == 0 && c % world == 0 && (r / world) % h1 == 0 &&
+                (c / world) % h2 == 0 && (r / world) % h3 == 0 && r / world >= 32 && c / world >= 32) {
+                P = std::move(T);
+                P.world = world;
+                P.rank = rank;
+                P.direct = 0;
+                P.p_copy.clear();
+                P.r_l = r / world;
+                P.c_l = c / world;
+                const int64_t Bw = P.r_l * P.c_l;
+                const int64_t first[3] = {rank * P.r_l / h1, rank * P.c_l / h2, rank * P.r_l / h3};
+                const int64_t count[3] = {P.r_l / h1, P.c_l / h2, P.r_l / h3};
+                for (int f = 0; f < 3; ++f) {
+                    TlcPass& tp = P.tp[f];
+                    U32Buf slice(P.sched[f].begin() + first[f] * tp.tile_words,
+                                 P.sched[f].begin() + (first[f] + count[f]) * tp.tile_words);
+                    P.sched[f].swap(slice);
+                    tp.ntiles = count[f];
+                    RowPass& rp = P.rp[f];
+                    rp.ctas = count[f];
+                    if (f == 0) {
+                        tp.segs = 1;
+                    } else {
+                        tp.segs = world;
+                        tp.seg_len = f == 1 ? P.r_l * h2 : P.c_l * h3;
+                        tp.seg_stride = Bw;
+                    }
+                    P.ph[f].lines = count[f] * tp.h;
+                }
+                return PERM_OK;
+            }
+        }
+    }
+    // the global plan with per-line schedules (5-pass geometry: whole lines)
     o.passes = 5;
     o.layout = 0;
-    o.direct = -1;                      // the shortcut is a single-device kernel
     int st = build_host_plan(p, n, eb, &o, P, err);
     if (st != PERM_OK) return st;
     const int64_t r = P.r, c = P.c;

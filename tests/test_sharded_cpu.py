@@ -26,11 +26,12 @@ def _lib():
 
 
 class FakeSteps:
-    """numpy execution of perm_sharded_step (test infrastructure, not the product)."""
+    """numpy execution of perm_sharded_step for the per-line (5-pass) form
+    (test infrastructure, not the product)."""
 
     def __init__(self, p, G, g):
         P = _lib()
-        with P.Plan(p, device=False, world=G, rank=g) as pl:
+        with P.Plan(p, device=False, world=G, rank=g, passes=5) as pl:
             info = pl.info()
             _, sched = pl.export()
         self.r, self.c = info["rows"], info["cols"]
@@ -64,6 +65,94 @@ class FakeSteps:
             res = self._permute(X, 2)                                      # R3 -> b rows
         out.numpy().view(np.uint32)[:] = np.ascontiguousarray(res).reshape(-1)
         return out
+
+
+class FakeTlcSteps:
+    """numpy execution of perm_sharded_step for the TLC form: the rank's
+    exported tile entries (src << 16 | dst) applied tile by tile; tiles of passes 2 and 3
+    gathered as one segment per sender; outputs scattered as chunks into the per-peer X1 /
+    X2 layouts (single-GPU layouts with r -> r/G, c -> c/G). Test infrastructure."""
+
+    def __init__(self, p, G, g):
+        P = _lib()
+        with P.Plan(p, device=False, world=G, rank=g) as pl:
+            info = pl.info()
+            d = pl.describe()
+            _, sched = pl.export()
+        assert d["layout"] == 3 and info["passes"] == 3
+        self.r, self.c = info["rows"], info["cols"]
+        self.G = G
+        self.h = [t["h"] for t in d["tlc"]]
+        self.sched = [np.asarray(x, dtype=np.int64).reshape(-1) for x in sched]
+
+    def _tiles(self, f, tiles, HL):
+        e = self.sched[f].reshape(len(tiles), HL)
+        src, dst = e >> 16, e & 0xFFFF
+        out = []
+        for T, A in enumerate(tiles):
+            B = np.empty_like(A)
+            B[dst[T]] = A[src[T]]
+            out.append(B)
+        return out
+
+    def sharded_step(self, step, inp, out, stream=None):
+        x = inp.numpy().view(np.uint32)
+        y = out.numpy().view(np.uint32)
+        G, r, c = self.G, self.r, self.c
+        rl, cl = r // G, c // G
+        h1, h2, h3 = self.h
+        Bw = rl * cl
+        if step == 0:
+            HL = h1 * c
+            tiles = [x[T * HL:(T + 1) * HL] for T in range(rl // h1)]
+            cw, cs = h1 * h2, rl * h2
+            for T, B in enumerate(self._tiles(0, tiles, HL)):
+                for m in range(c // h2):
+                    y[m * cs + T * cw:m * cs + (T + 1) * cw] = B[m * cw:(m + 1) * cw]
+        elif step == 1:
+            sl, HL = rl * h2, r * h2
+            tiles = [np.concatenate([x[q * Bw + K * sl:q * Bw + (K + 1) * sl] for q in range(G)])
+                     for K in range(cl // h2)]
+            cw, cs = h3 * h2, cl * h3
+            for K, B in enumerate(self._tiles(1, tiles, HL)):
+                for m in range(r // h3):
+                    y[m * cs + K * cw:m * cs + (K + 1) * cw] = B[m * cw:(m + 1) * cw]
+        else:
+            sl, HL = cl * h3, h3 * c
+            tiles = [np.concatenate([x[q * Bw + I * sl:q * Bw + (I + 1) * sl] for q in range(G)])
+                     for I in range(rl // h3)]
+            for I, B in enumerate(self._tiles(2, tiles, HL)):
+                y[I * HL:(I + 1) * HL] = B
+        return out
+
+
+@pytest.mark.parametrize("G", [1, 2, 4, 8])
+@pytest.mark.parametrize("fam", ["random", "bitrev", "transpose"])
+def test_virtual_ranks_tlc_form_numpy(G, fam):
+    from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
+    n = 1 << 16
+    p = W.make_perm(fam, n, seed=G + 1)
+    a = W.make_data(n)
+    shard = n // G
+    steps = [FakeTlcSteps(p, G, g) for g in range(G)]
+
+    class Wrap:
+        def __init__(self, s):
+            self.s = s
+
+        def info(self):
+            return {"block_elems": n // (G * G)}
+
+        def sharded_step(self, *args):
+            return self.s.sharded_step(*args)
+
+    a_sh = [torch.from_numpy(a[g * shard:(g + 1) * shard].view(np.int32).copy()) for g in range(G)]
+    b_sh = [torch.empty(shard, dtype=torch.int32) for _ in range(G)]
+    send = [torch.empty(shard, dtype=torch.int32) for _ in range(G)]
+    recv = [torch.empty(shard, dtype=torch.int32) for _ in range(G)]
+    apply_virtual([Wrap(s) for s in steps], a_sh, b_sh, send, recv)
+    b = np.concatenate([x.numpy().view(np.uint32) for x in b_sh])
+    assert np.array_equal(b, OA.apply_ref(p, a))
 
 
 @pytest.mark.parametrize("G", [1, 2, 4, 8])
@@ -103,7 +192,7 @@ def _free_port():
     return port
 
 
-def _gloo_worker(rank, world, port, k, fam, q):
+def _gloo_worker(rank, world, port, k, fam, q, tlc=False):
     import torch.distributed as dist
     from paper_conf_icpp_kasagini13_b200.sharded import ShardedApply
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -114,7 +203,7 @@ def _gloo_worker(rank, world, port, k, fam, q):
         p = W.make_perm(fam, n, seed=11)
         a = W.make_data(n)
         shard = n // world
-        steps = FakeSteps(p, world, rank)
+        steps = (FakeTlcSteps if tlc else FakeSteps)(p, world, rank)
         run = ShardedApply(steps)            # exchange = torch.distributed.all_to_all_single
         a_sh = torch.from_numpy(a[rank * shard:(rank + 1) * shard].view(np.int32).copy())
         b_sh = torch.empty(shard, dtype=torch.int32)
@@ -127,14 +216,15 @@ def _gloo_worker(rank, world, port, k, fam, q):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("tlc", [False, True])
 @pytest.mark.parametrize("fam", ["random", "bitrev"])
-def test_gloo_world2(fam):
+def test_gloo_world2(fam, tlc):
     import torch.multiprocessing as mp
     _lib()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_gloo_worker, args=(r, 2, port, 16, fam, q)) for r in range(2)]
+    procs = [ctx.Process(target=_gloo_worker, args=(r, 2, port, 16, fam, q, tlc)) for r in range(2)]
     for pr in procs:
         pr.start()
     for pr in procs:
