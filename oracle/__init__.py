@@ -15,7 +15,9 @@ Modules (each function cites the passage it follows):
 * ``distribution`` D_w(P) (L389-L401, Lemma 4)
 * ``konig``        König edge colouring by alternating paths (Thm 6)
 * ``planner``      reference scheduled-permutation planner (L515-L539, L603-L605)
-* ``check``        plan invariants (i)-(vii) (L519, L531-L539)
+* ``check``        plan invariants (i)-(vii) (L519, L531-L539); tiled (TLC) and cluster plans
+* ``tiled``        the oracle's own TLC / cluster plan builders and executors (L531-L539 over
+                   tiles; Lemma 8's transposes as chunk scatters / block exchanges)
 * ``emulate``      paper-faithful R,T,R,T,R with a Table I round counter (L409-L533, L681)
 * ``c/apply_ref.c`` the definition as a plain C loop, for CPU timing only
 

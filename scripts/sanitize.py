@@ -58,19 +58,20 @@ from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
 n, G = 1 << 16, 2
 p = W.random(n, 5)
 a = W.make_data(n)
-plans = [P.Plan(p, world=G, rank=g) for g in range(G)]
-sh = n // G
-a_sh = [torch.from_numpy(a[g * sh:(g + 1) * sh].view(np.int32).copy()).cuda() for g in range(G)]
-b_sh = [torch.full((sh,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
-snd = [torch.empty(sh, dtype=torch.int32, device="cuda") for _ in range(G)]
-rcv = [torch.empty(sh, dtype=torch.int32, device="cuda") for _ in range(G)]
-apply_virtual(plans, a_sh, b_sh, snd, rcv)
-torch.cuda.synchronize()
-ok = np.array_equal(np.concatenate([x.cpu().numpy().view(np.uint32) for x in b_sh]), scatter_np(p, a))
-fails += not ok
-print(f"{'sharded steps (G=2 virtual ranks)':55s} n=2^16: {'ok' if ok else 'MISMATCH'}", flush=True)
-for pl in plans:
-    pl.close()
+for form, kw in (("TLC form", {}), ("per-line 5-pass form", {"passes": 5})):
+    plans = [P.Plan(p, world=G, rank=g, **kw) for g in range(G)]
+    sh = n // G
+    a_sh = [torch.from_numpy(a[g * sh:(g + 1) * sh].view(np.int32).copy()).cuda() for g in range(G)]
+    b_sh = [torch.full((sh,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
+    snd = [torch.empty(sh, dtype=torch.int32, device="cuda") for _ in range(G)]
+    rcv = [torch.empty(sh, dtype=torch.int32, device="cuda") for _ in range(G)]
+    apply_virtual(plans, a_sh, b_sh, snd, rcv)
+    torch.cuda.synchronize()
+    ok = np.array_equal(np.concatenate([x.cpu().numpy().view(np.uint32) for x in b_sh]), scatter_np(p, a))
+    fails += not ok
+    print(f"{'sharded steps, ' + form + ' (G=2 virtual ranks)':55s} n=2^16: {'ok' if ok else 'MISMATCH'}", flush=True)
+    for pl in plans:
+        pl.close()
 
 da = torch.from_numpy(a.view(np.int32)).cuda()
 db = torch.empty_like(da)
