@@ -272,7 +272,7 @@ int perm_apply_sharded(const perm_plan* plan, const void* a_shard, void* b_shard
  * For n = 2^15..2^25 words (TLC form, info.passes == 3) each step is ONE tile-coloured pass
  * that writes the send buffer in the exchange layout directly; beyond (per-line form,
  * info.passes == 5) steps 0 and 1 are a row pass plus a transpose. The buffers' contents
- * differ between the forms; the block contract below is the same. */
+ * differ between the forms; the block contract below is the same.
  * Between steps 0->1 and 1->2 the caller performs the all-to-all: with
  * B = n/world^2, for every pair (g, q): recv_q[g*B : (g+1)*B] = send_g[q*B : (q+1)*B]
  * (perm_sharded_exchange, or device copies for ranks sharing one GPU). */

@@ -925,7 +925,9 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     // TILED 3-pass layouts on request), the paper's 5-pass structure (TMA row passes) from 2^26
     // cluster path (one launch, DSMEM exchanges) for 2^15..2^17: 8.3 / 10.0 / 12.5 us vs the
     // three TLC launches' 13.5 / 14.0 / 14.8 us (profiles/r02_small_n.jsonl)
-    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 17 ? 2 : (k <= 25 ? 3 : 5));
+    // (an explicit 3-pass layout or the single-launch TLC option keeps the TLC passes)
+    const bool tlc_opts = opt && (opt->layout != 0 || opt->fuse > 0);
+    if (passes == 0) passes = (k <= 14) ? 1 : (k <= 17 && !tlc_opts ? 2 : (k <= 25 ? 3 : 5));
     // dense schedule bitstreams only where the 5-pass row kernels read them
     const bool dense_phases = passes == 5 && !(opt && opt->sched_format < 0);
     // geometry of the three phases

@@ -355,7 +355,7 @@ def test_run_pass_chain_is_apply(P, k):
     n = 1 << k
     p = W.random(n, 900 + k)
     a = W.make_data(n)
-    with P.Plan(p) as plan:
+    with P.Plan(p, passes=3) as plan:
         da = dev(a)
         db = torch.full_like(da, -1)
         plan.run_pass(0, da)
