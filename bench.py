@@ -293,7 +293,9 @@ def run_sharded(args, rank, world, local):
         info = pl.info()
         desc = pl.describe()
         sb = sched_bytes_per_elt(info, desc)
-        local_bytes = shard * (5 * 8 + sum(sb))             # R1, T, R2, T, R3 + schedules
+        # TLC form: three passes writing / reading the exchange layouts; per-line form: R1, T,
+        # R2, T, R3 (plus the schedules either way)
+        local_bytes = shard * (info["passes"] * 8 + sum(sb))
         t_hbm = local_bytes / (peaks["hbm_gbs"] * 1e9) * 1e3
         t_nvl = 2 * xbytes / (nvl_peak * 1e9) * 1e3
         t_apply = ms_per_step / len(fams)
@@ -308,7 +310,9 @@ def run_sharded(args, rank, world, local):
                 "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": cfg, "bitexact_check_all_ranks": bool(okt.item()),
                 "plan_build_ms_rank0": build_ms,
-                "stage_ms": dict(zip(["R1+Tpack", "all-to-all 1", "R2+Tpack", "all-to-all 2", "R3"], st_ms)),
+                "sharded_form": "TLC (T-pack fused into the passes)" if info["passes"] == 3 else "per-line 5-pass",
+                "stage_ms": dict(zip(["R1" if info["passes"] == 3 else "R1+Tpack", "all-to-all 1",
+                                      "R2" if info["passes"] == 3 else "R2+Tpack", "all-to-all 2", "R3"], st_ms)),
                 "exchange_bytes_per_gpu": xbytes,
                 "nvlink_frac": [(xbytes / (st_ms[i] * 1e-3) / 1e9) / nvl_peak if world > 1 else None
                                 for i in (1, 3)],
@@ -318,7 +322,7 @@ def run_sharded(args, rank, world, local):
                 "ideal_ms": {"T_HBM": t_hbm, "T_NVL": t_nvl, "no_overlap": t_hbm + t_nvl,
                              "perfect_overlap": max(t_hbm, t_nvl)},
                 "nvlink_peak_gbs": nvl_peak, "hbm_peak_gbs": peaks["hbm_gbs"],
-                "gpu_launches": args.steps * len(fams) * 5,
+                "gpu_launches": args.steps * len(fams) * info["passes"],
                 "clocks": clocks.summary()}
         print(json.dumps(line), flush=True)
     for f in fams:
