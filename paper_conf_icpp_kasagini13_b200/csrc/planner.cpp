@@ -544,10 +544,14 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
     int64_t hs[3];
     for (int f = 0; f < 3; ++f) {
         const int64_t L = P.ph[f].L, lines_f = P.ph[f].lines;
-        // default tiles: 8192 words up to 2^24 (64-byte transposed chunks), 16384 words at
-        // 2^25 (32-byte chunks: h1*h2*4 bytes with h1*L, h2*r <= 16384 words)
-        int64_t h = (opt && (&opt->h1)[f] > 0) ? (&opt->h1)[f]
-                    : (P.k <= 24 ? std::max<int64_t>(4, 8192 / L) : std::max<int64_t>(1, 16384 / L));
+        // default tiles: 8192 words up to 2^24 (pass 2 keeps h2 >= 4 for 16-byte TMA box rows,
+        // so 16384 words at 2^24), 16384 words at 2^25. The transposed chunks are h1*h2 words:
+        // 16 at 2^22, 8 (32 bytes) at 2^23 - 2^25. Smaller row tiles at 2^23 / 2^24 measured
+        // 41.0 / 90.3 us against 47.5 / 98.0 us with h1 = h3 = 4 (profiles/r02_ab_mid.jsonl).
+        int64_t h = (opt && (&opt->h1)[f] > 0)
+                        ? (&opt->h1)[f]
+                        : (P.k <= 24 ? std::max<int64_t>(f == 1 ? 4 : 2, 8192 / L)
+                                     : std::max<int64_t>(1, 16384 / L));
         h = std::min(h, lines_f);
         // h2 is the inner dimension of the TMA tensor boxes (>= 16 bytes)
         if (h < (f == 1 ? 4 : 1) || (h & (h - 1)) || lines_f % h) {
