@@ -548,10 +548,12 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
         // so 16384 words at 2^24), 16384 words at 2^25. The transposed chunks are h1*h2 words:
         // 16 at 2^22, 8 (32 bytes) at 2^23 - 2^25. Smaller row tiles at 2^23 / 2^24 measured
         // 41.0 / 90.3 us against 47.5 / 98.0 us with h1 = h3 = 4 (profiles/r02_ab_mid.jsonl).
+        // Up to 2^19, 8192-word tiles leave SMs idle (32 / 64 tiles per pass at 2^18 / 2^19 on
+        // 148 SMs): 4096-word tiles, 14.7 -> 13.3 us and 15.5 -> 13.4 us (profiles/r02_ab_small.jsonl).
+        const int64_t T = P.k <= 19 ? 4096 : (P.k <= 24 ? 8192 : 16384);
         int64_t h = (opt && (&opt->h1)[f] > 0)
                         ? (&opt->h1)[f]
-                        : (P.k <= 24 ? std::max<int64_t>(f == 1 ? 4 : 2, 8192 / L)
-                                     : std::max<int64_t>(1, 16384 / L));
+                        : (P.k <= 24 ? std::max<int64_t>(f == 1 ? 4 : 2, T / L) : std::max<int64_t>(1, T / L));
         h = std::min(h, lines_f);
         // h2 is the inner dimension of the TMA tensor boxes (>= 16 bytes)
         if (h < (f == 1 ? 4 : 1) || (h & (h - 1)) || lines_f % h) {
