@@ -100,6 +100,23 @@ __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+// L2 eviction-priority policies (createpolicy) and a read-only load carrying one
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint32_t ld_nc_hint(const uint32_t* p, uint64_t pol) {
+    uint32_t v;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+
 // streaming 128-bit load of data that is not written by this kernel
 __device__ __forceinline__ uint4 ld_nc_v4(const uint32_t* p) {
     uint4 r;
@@ -909,11 +926,13 @@ __device__ __forceinline__ void red_release_gpu_add(unsigned long long* p, unsig
 
 // ------------------------------------------------------------------ TLC row pass (tile-level colouring)
 
+// intermediates X1 / X2 are re-read by the next pass: stored with an evict_last L2 policy
 __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void* src, int c0, int c1, int c2) {
+    const uint64_t pol = policy_evict_last();
     asm volatile(
-        "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+        "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3, %4}], [%1], %5;" ::"l"(
             reinterpret_cast<uint64_t>(map)),
-        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2)
+        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "l"(pol)
         : "memory");
 }
 
@@ -1138,7 +1157,9 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         const bool lead = tid == 64;
         const uint32_t* sp = a.sched + (warp - 2) * NWORDS * 32 + lane;
         // schedule words live in registers, loaded AHEAD tiles ahead (L2 latency under the
-        // load of a pass is about one tile period)
+        // load of a pass is about one tile period); each is read once, so it leaves L2 first
+        // (the intermediates X1 / X2 are what the next pass reads)
+        const uint64_t pol_first = policy_evict_first();
         constexpr int AHEAD = NWORDS <= 12 ? 2 : 1;
         uint32_t wq[AHEAD + 1][NWORDS];
 #pragma unroll
@@ -1146,7 +1167,7 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             const long long tk = blockIdx.x + (long long)k * G;
             if (tk < a.ntiles) {
 #pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wq[k][w] = __ldg(sp + tk * a.tile_words + w * 32);
+                for (int w = 0; w < NWORDS; ++w) wq[k][w] = ld_nc_hint(sp + tk * a.tile_words + w * 32, pol_first);
             }
         }
         for (int i = 0;; ++i) {
@@ -1156,7 +1177,7 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             const long long tn = t + (long long)AHEAD * G;
             if (tn < a.ntiles) {
 #pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wq[AHEAD][w] = __ldg(sp + tn * a.tile_words + w * 32);
+                for (int w = 0; w < NWORDS; ++w) wq[AHEAD][w] = ld_nc_hint(sp + tn * a.tile_words + w * 32, pol_first);
             }
             mbar_wait(&R.afull[s], (uint32_t)(i / NA) & 1u);
             if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
