@@ -125,7 +125,7 @@ int upload(perm_plan* pl) {
         if (e != cudaSuccess) return cuda_fail(e, "upload p (direct)");
         std::vector<int32_t>().swap(pl->host.p_copy);
     }
-    if (P.layout == 3) {
+    if (P.layout == 3 || P.layout == 5) {
         e = perm::make_tlc_maps(P, pl->d_scratch[0], pl->d_scratch[1], pl->tlc_maps);
         if (e != cudaSuccess) return cuda_fail(e, "cuTensorMapEncodeTiled");
     }
@@ -370,7 +370,7 @@ int perm_plan_get_info(const perm_plan* plan, perm_plan_info* out) {
     out->gpu_planner = P.gpu_planner;
     for (int f = 0; f < 3; ++f) {
         out->entry_bits[f] = P.layout >= 3 ? P.tp[f].E : P.ph[f].E;
-        out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : P.rp[f].h;
+        out->h[f] = P.passes == 1 ? (int32_t)P.ph[f].lines : (P.layout == 5 ? P.tp[f].h : P.rp[f].h);
     }
     out->planner_threads = P.threads_used;
     out->build_ms_colour = P.ms_colour;
@@ -452,6 +452,22 @@ int perm_plan_export(const perm_plan* plan, uint16_t* kappa, uint32_t* s1, uint3
     if (P.direct) return fail(PERM_EUNSUPPORTED, "low-distribution shortcut plan: no schedule to export");
     if (kappa) std::memcpy(kappa, P.kappa.data(), (size_t)P.n * sizeof(uint16_t));   // words
     uint32_t* outs[3] = {s1, s2, s3};
+    if (P.layout == 5) {
+        // TLC ring: tile T's entries in the dense per-round format of a 32768-word line
+        for (int f = 0; f < 3; ++f) {
+            if (!outs[f]) continue;
+            const perm::PhaseGeom& g = P.ph[f];
+#pragma omp parallel for schedule(static)
+            for (int64_t T = 0; T < g.lines; ++T)
+                for (int64_t q = 0; q < g.L; ++q) {
+                    const uint32_t e = perm::unpack_entry(P.sched[f], g, T, q);
+                    const uint32_t src = ((e >> g.logL) << 5) | (uint32_t)(q & 31);
+                    const uint32_t dst = e & ((1u << g.logL) - 1u);
+                    outs[f][T * g.L + q] = (src << 16) | dst;
+                }
+        }
+        return PERM_OK;
+    }
     if (P.layout >= 3) {
         // TLC / cluster path: entry (tile T, round q, lane x) -> (src word offset in A << 16) | dst offset in B
         for (int f = 0; f < 3; ++f) {
@@ -617,6 +633,14 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
         mark();
         if (e == cudaSuccess) { ++k; e = perm::launch_tlc_pass(P, 1, plan->tlc_maps, plan->d_phase[1], x1, x2, s, !prof, tr(1)); mark(); }
         if (e == cudaSuccess) { ++k; e = perm::launch_tlc_pass(P, 2, plan->tlc_maps, plan->d_phase[2], x2, out, s, !prof, tr(2)); mark(); }
+    } else if (P.layout == 5) {
+        // TLC passes through the half-tile ring: a -> X1 -> X2 -> b, chunked tensor stores
+        uint32_t* x1 = plan->d_scratch[0];
+        uint32_t* x2 = plan->d_scratch[1];
+        e = perm::launch_row_pass(P, 0, plan->d_phase[0], in, x1, s, false, tr(0), &plan->tlc_maps[0]);
+        mark();
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 1, plan->d_phase[1], x1, x2, s, !prof, tr(1), &plan->tlc_maps[1]); mark(); }
+        if (e == cudaSuccess) { ++k; e = perm::launch_row_pass(P, 2, plan->d_phase[2], x2, out, s, !prof, tr(2)); mark(); }
     } else if (P.passes == 3) {
         uint32_t* x1 = plan->d_scratch[0];
         uint32_t* x2 = plan->d_scratch[1];

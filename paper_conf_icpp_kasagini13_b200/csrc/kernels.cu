@@ -117,6 +117,16 @@ __device__ __forceinline__ uint32_t ld_nc_hint(const uint32_t* p, uint64_t pol) 
     return v;
 }
 
+// intermediates X1 / X2 are re-read by the next pass: stored with an evict_last L2 policy
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void* src, int c0, int c1, int c2) {
+    const uint64_t pol = policy_evict_last();
+    asm volatile(
+        "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3, %4}], [%1], %5;" ::"l"(
+            reinterpret_cast<uint64_t>(map)),
+        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "l"(pol)
+        : "memory");
+}
+
 // streaming 128-bit load of data that is not written by this kernel
 __device__ __forceinline__ uint4 ld_nc_v4(const uint32_t* p) {
     uint4 r;
@@ -420,6 +430,10 @@ struct TmaArgs {
     int ntiles, stages;
     int data_words;            // h * Ls
     int sched_words;           // h * (L/32) * E, a multiple of 4
+    // half-line ring as a TLC pass (layout 5): each half of a permuted tile leaves as 3-D
+    // tensor stores of its chunks into X1 / X2 (out_kind 1 / 2); 0 = 1-D bulk stores of rows
+    int out_kind;
+    int chunk, box_outer, box_words, boxes_per_half;
 };
 
 // Persistent, pipelined row-wise permutation pass (Lemma 7) for contiguous input
@@ -755,7 +769,8 @@ constexpr int kStgDenseWords = 64 * 25;          // dense: 64 rounds of E <= 25 
 // stay in registers across the barrier. The permute is bound by the chunk latency (per-CTA
 // traces, profiles/r01_trace_ring_s8.log), hence the dense format's smaller, deeper ring.
 template <int EPT, bool DENSE>
-__global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(const TmaArgs a) {
+__global__ void __launch_bounds__(kStgWorkers, 1)
+    row_pass_split_stg_kernel(const __grid_constant__ CUtensorMap tmap, const TmaArgs a) {
     extern __shared__ __align__(128) uint32_t smem[];
     constexpr int NB = DENSE ? 5 : 4;            // chunk ring depth
     constexpr int CWS = DENSE ? kStgDenseWords : kStgChunkWords;   // buffer stride (words)
@@ -893,11 +908,23 @@ __global__ void __launch_bounds__(kStgWorkers, 1) row_pass_split_stg_kernel(cons
         if (i < 4) stamp(tr, 3 + 3 * (int)i);
         if (tid == 0) {
             fence_proxy_async();
-            uint32_t* dst = a.r.out + t * (long long)L;
-            bulk_s2g(dst, smem + o0, half_bytes);
-            bulk_commit();
-            bulk_s2g(dst + HALF, smem + o1, half_bytes);
-            bulk_commit();
+            if (a.out_kind == 0) {
+                uint32_t* dst = a.r.out + t * (long long)L;
+                bulk_s2g(dst, smem + o0, half_bytes);
+                bulk_commit();
+                bulk_s2g(dst + HALF, smem + o1, half_bytes);
+                bulk_commit();
+            } else {
+                // the tile's output order is its chunks (one per K- / I'-block) back to back;
+                // half q holds blocks [q * nbh, (q + 1) * nbh), nbh = boxes_per_half * box_outer
+                for (int q = 0; q < 2; ++q) {
+                    const uint32_t* src = smem + (q ? o1 : o0);
+                    for (int bx = 0; bx < a.boxes_per_half; ++bx)
+                        tma_store_3d(&tmap, src + bx * a.box_words, 0, (int)t * a.chunk,
+                                     (q * a.boxes_per_half + bx) * a.box_outer);
+                    bulk_commit();
+                }
+            }
             bulk_wait_read1();
             fence_proxy_async();
             issue_half(2 * i + 3);           // second half of line i+1 -> slot s0
@@ -926,15 +953,6 @@ __device__ __forceinline__ void red_release_gpu_add(unsigned long long* p, unsig
 
 // ------------------------------------------------------------------ TLC row pass (tile-level colouring)
 
-// intermediates X1 / X2 are re-read by the next pass: stored with an evict_last L2 policy
-__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void* src, int c0, int c1, int c2) {
-    const uint64_t pol = policy_evict_last();
-    asm volatile(
-        "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3, %4}], [%1], %5;" ::"l"(
-            reinterpret_cast<uint64_t>(map)),
-        "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "l"(pol)
-        : "memory");
-}
 
 __host__ __device__ constexpr int cilog2(int v) { return v <= 1 ? 0 : 1 + cilog2(v >> 1); }
 
@@ -2152,7 +2170,8 @@ cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], cons
 }
 
 cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, const uint32_t* in,
-                            uint32_t* out, cudaStream_t s, bool pdl, unsigned long long* trace) {
+                            uint32_t* out, cudaStream_t s, bool pdl, unsigned long long* trace,
+                            const CUtensorMap* map) {
     const RowPass& rp = P.rp[f];
     const PhaseGeom& g = P.ph[rp.phase];
     RowArgs ra{};
@@ -2187,10 +2206,25 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const bool sg = rp.sg != 0;
         if (rp.split && rp.split_stg) {
             const bool dn = g.dense != 0;
-            if (rp.ept == 32) return dn ? launch(row_pass_split_stg_kernel<32, true>, grid, block, smem, s, pdl, ta)
-                                        : launch(row_pass_split_stg_kernel<32, false>, grid, block, smem, s, pdl, ta);
-            if (rp.ept == 64) return dn ? launch(row_pass_split_stg_kernel<64, true>, grid, block, smem, s, pdl, ta)
-                                        : launch(row_pass_split_stg_kernel<64, false>, grid, block, smem, s, pdl, ta);
+            CUtensorMap m{};
+            if (map) m = *map;
+            if (P.layout == 5 && P.tp[f].out_kind != 0) {
+                // TLC ring pass: chunks of h1*h2 (X1) or h3*h2 (X2) words, one per block
+                const long long h1 = P.tp[0].h, h2 = P.tp[1].h, h3 = P.tp[2].h;
+                const int kind = P.tp[f].out_kind;
+                const long long cw = kind == 1 ? h1 * h2 : h3 * h2;
+                const long long nblk = kind == 1 ? P.c / h2 : P.r / h3;
+                const long long bo = std::min<long long>(256, nblk / 2);
+                ta.out_kind = kind;
+                ta.chunk = (int)(cw / std::min<long long>(cw, 256));
+                ta.box_outer = (int)bo;
+                ta.box_words = (int)(bo * cw);
+                ta.boxes_per_half = (int)(nblk / 2 / bo);
+            }
+            if (rp.ept == 32) return dn ? launch(row_pass_split_stg_kernel<32, true>, grid, block, smem, s, pdl, m, ta)
+                                        : launch(row_pass_split_stg_kernel<32, false>, grid, block, smem, s, pdl, m, ta);
+            if (rp.ept == 64) return dn ? launch(row_pass_split_stg_kernel<64, true>, grid, block, smem, s, pdl, m, ta)
+                                        : launch(row_pass_split_stg_kernel<64, false>, grid, block, smem, s, pdl, m, ta);
             return cudaErrorInvalidValue;
         }
         if (rp.split) {

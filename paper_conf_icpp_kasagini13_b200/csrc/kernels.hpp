@@ -24,9 +24,10 @@ cudaError_t launch_cluster(const HostPlan& P, const uint32_t* const sched[3], co
 
 // One row pass (pass index f in 0..2) of the 3- or 5-pass pipeline.
 // `trace`: optional device buffer of 16 %globaltimer stamps per CTA (nullptr = off).
+// `map`: the X1 / X2 tensor map when the pass is a TLC ring pass (layout 5) with chunked output.
 cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, const uint32_t* in,
                             uint32_t* out, cudaStream_t s, bool pdl,
-                            unsigned long long* trace = nullptr);
+                            unsigned long long* trace = nullptr, const CUtensorMap* map = nullptr);
 
 // TLC layout: tensor maps of the intermediates (maps[0]: X1 for pass 1's 3-D
 // stores, maps[1]: X2 for pass 2's 4-D stores) and one pass launch.

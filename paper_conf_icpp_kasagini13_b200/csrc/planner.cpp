@@ -664,6 +664,143 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
     return PERM_OK;
 }
 
+// ------------------------------------------------------------------ TLC through the half-line ring
+//
+// 2^26 / 2^27 (layout 5): the TLC passes (tile-level colouring, transposes absorbed into the
+// intermediates' chunk layouts) with 32768-word tiles, so that the transposed
+// chunks are 16 / 8 words; a tile of 128 KiB is permuted in place through the three 64 KiB
+// half-tile slots of row_pass_split_stg_kernel (the L = 32768 row-pass machinery), whose
+// stores write the two halves of the tile's output order as X1 / X2 tensor-store chunks.
+// Schedules: every tile's bank graph (src mod 32, dst mod 32) coloured, packed in the dense
+// per-round format of a 32768-word "line" (entry (src >> 5) << 15 | dst, E = 25 bits).
+int build_tlc_ring(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt, std::string& err) {
+    const int64_t r = P.r, c = P.c;
+    constexpr int64_t HL = 32768;
+    int64_t hs[3];
+    for (int f = 0; f < 3; ++f) {
+        const int64_t L = P.ph[f].L;
+        const int64_t h = (opt && (&opt->h1)[f] > 0) ? (&opt->h1)[f] : HL / L;
+        if (h * L != HL || (h & (h - 1)) || P.ph[f].lines % h || (f == 1 && h < 4)) {
+            err = "TLC ring layout: tiles must hold 32768 words (h * L), h2 >= 4";
+            return PERM_EINVAL;
+        }
+        hs[f] = h;
+    }
+    const int64_t h1 = hs[0], h2 = hs[1], h3 = hs[2];
+    if (h1 * h2 < 4 || h3 * h2 < 4) { err = "TLC ring layout: transposed chunks under 16 bytes"; return PERM_EINVAL; }
+    P.layout = 5;
+    P.passes = 3;
+    for (int f = 0; f < 3; ++f) {
+        TlcPass& tp = P.tp[f];
+        tp = TlcPass{};
+        tp.h = (int32_t)hs[f];
+        tp.HL = (int32_t)HL;
+        tp.logHL = 15;
+        tp.E = 25;
+        tp.ntiles = P.ph[f].lines / hs[f];
+        tp.out_kind = f == 0 ? 1 : (f == 1 ? 2 : 0);
+        tp.dec.lt = 15;
+        // the tile is the ring kernel's "line": one 32768-word line per CTA step
+        PhaseGeom& g = P.ph[f];
+        g.lines = tp.ntiles;
+        g.L = (int32_t)HL;
+        g.logL = 15;
+        g.E = 25;
+        g.epw = 64 / g.E;
+        g.w64 = (kW + g.epw - 1) / g.epw;
+        g.dense = 1;
+        g.wpl = (HL / kW) * g.E;
+        g.words = g.lines * g.wpl;
+        RowPass& rp = P.rp[f];
+        rp = RowPass{};
+        rp.phase = f; rp.h = 1; rp.ctas = tp.ntiles;
+        rp.in = IoMode{}; rp.out = IoMode{};
+        rp.in.w = (int32_t)HL; rp.out.w = (int32_t)HL;
+        rp.in.cta_stride = HL; rp.out.cta_stride = HL;
+        rp.tma = 1; rp.sg = 1; rp.split = 1; rp.split_stg = 1; rp.stages = 3;
+        rp.threads = 512; rp.ept = (int32_t)(HL / 512); rp.Ls = (int32_t)HL;
+    }
+    for (int f = 0; f < 3; ++f) {
+        const TlcPass& tp = P.tp[f];
+        const PhaseGeom& g = P.ph[f];
+        const uint16_t* ph = phi[f].data();
+        const int64_t h = tp.h;
+        // element x of tile T: source offset in the tile (input order), destination offset
+        // (output order) -- the TLC layouts of build_tlc
+        auto enum_tile = [&](int64_t T, uint32_t* src, uint32_t* dst) {
+            int64_t e = 0;
+            if (f == 0) {
+                for (int64_t i_in = 0; i_in < h; ++i_in)
+                    for (int64_t j = 0; j < c; ++j, ++e) {
+                        const int64_t kk = ph[(T * h + i_in) * c + j];
+                        src[e] = (uint32_t)(i_in * c + j);
+                        dst[e] = (uint32_t)(((kk / h2) * h1 + i_in) * h2 + kk % h2);
+                    }
+            } else if (f == 1) {
+                for (int64_t k_in = 0; k_in < h; ++k_in)
+                    for (int64_t i = 0; i < r; ++i, ++e) {
+                        const int64_t ip = ph[(T * h + k_in) * r + i];
+                        src[e] = (uint32_t)(i * h2 + k_in);
+                        dst[e] = (uint32_t)(ip * h2 + k_in);
+                    }
+            } else {
+                for (int64_t i_in = 0; i_in < h; ++i_in)
+                    for (int64_t kk = 0; kk < c; ++kk, ++e) {
+                        const int64_t kp = ph[(T * h + i_in) * c + kk];
+                        src[e] = (uint32_t)(((kk / h2) * h3 + i_in) * h2 + kk % h2);
+                        dst[e] = (uint32_t)(i_in * c + kp);
+                    }
+            }
+        };
+        std::vector<uint16_t> gcol;
+        if (opt && opt->gpu_planner > 0) {
+            const int64_t N = tp.ntiles * HL;
+            U16Buf ks((size_t)N), kd((size_t)N);
+#pragma omp parallel
+            {
+                std::vector<uint32_t> src((size_t)HL), dst((size_t)HL);
+#pragma omp for schedule(static)
+                for (int64_t T = 0; T < tp.ntiles; ++T) {
+                    enum_tile(T, src.data(), dst.data());
+                    for (int64_t x = 0; x < HL; ++x) {
+                        ks[T * HL + x] = (uint16_t)src[x];
+                        kd[T * HL + x] = (uint16_t)dst[x];
+                    }
+                }
+            }
+            gcol.resize((size_t)N);
+            GpuPlanStats gs;
+            const cudaError_t ce = gpu_bank_colour(ks.data(), kd.data(), N, 15, gcol.data(), &gs);
+            if (ce != cudaSuccess) {
+                err = std::string("GPU planner (TLC ring bank colouring): ") + cudaGetErrorString(ce);
+                return ce == cudaErrorMemoryAllocation ? PERM_ENOMEM : PERM_ECUDA;
+            }
+        }
+        P.sched[f].assign((size_t)g.words + 4, 0u);
+        uint32_t* W = P.sched[f].data();
+#pragma omp parallel
+        {
+            EulerColourer ec;
+            std::vector<uint32_t> U((size_t)HL), V((size_t)HL), col((size_t)HL), src((size_t)HL), dst((size_t)HL);
+#pragma omp for schedule(dynamic, 1)
+            for (int64_t T = 0; T < tp.ntiles; ++T) {
+                enum_tile(T, src.data(), dst.data());
+                if (!gcol.empty()) {
+                    for (int64_t x = 0; x < HL; ++x) col[x] = gcol[T * HL + x];
+                } else {
+                    for (int64_t x = 0; x < HL; ++x) { U[x] = src[x] & 31; V[x] = dst[x] & 31; }
+                    ec.run(kW, HL / kW, HL, U.data(), V.data(), col.data(), false);
+                }
+                for (int64_t x = 0; x < HL; ++x) {
+                    const uint64_t entry = ((uint64_t)(src[x] >> 5) << 15) | dst[x];
+                    pack_entry(W, g, T, (int64_t)col[x] * kW + (src[x] & 31), entry);
+                }
+            }
+        }
+    }
+    return PERM_OK;
+}
+
 // ------------------------------------------------------------------ cluster path
 //
 // n <= 2^18 (NEXT-4: the whole array fits on chip): ONE launch of one
@@ -934,6 +1071,7 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     // (an explicit 3-pass layout or the single-launch TLC option keeps the TLC passes)
     const bool tlc_opts = opt && (opt->layout != 0 || opt->fuse > 0);
     if (passes == 0) passes = (k <= 14) ? 1 : (k <= 17 && !tlc_opts ? 2 : (k <= 25 ? 3 : 5));
+    if (opt && opt->layout == 5 && (!opt->passes || opt->passes == 3)) passes = 3;   // TLC ring
     // dense schedule bitstreams only where the 5-pass row kernels read them
     const bool dense_phases = passes == 5 && !(opt && opt->sched_format < 0);
     // geometry of the three phases
@@ -1029,6 +1167,11 @@ int build_host_plan(const int32_t* p, int64_t n, int32_t eb, const perm_plan_opt
     }
     {
         int layout0 = opt ? opt->layout : 0;
+        if (passes == 3 && layout0 == 5) {
+            const int st = build_tlc_ring(P, phi, opt, err);
+            P.ms_bank = ms_since(t0);
+            return st;
+        }
         if (passes == 3 && (layout0 == 3 || (layout0 == 0 && k >= 15 && k <= 25))) {
             const int st = build_tlc(P, phi, opt, err);
             P.ms_bank = ms_since(t0);

@@ -470,3 +470,16 @@ def test_cluster_path_fp64_and_replay(P):
             plan.apply(da, db)
         torch.cuda.synchronize()
         assert np.array_equal(db.cpu().numpy().view(np.uint64), OA.apply_ref(p, a))
+
+
+@pytest.mark.parametrize("fam", ["random", "bitrev", "transpose", "shuffle"])
+@pytest.mark.parametrize("k", [20, 21, 22, 26])
+def test_tlc_ring(P, fam, k):
+    # layout 5: the TLC passes (transposes absorbed into X1 / X2 chunks) with 32768-word
+    # tiles permuted in place through the half-tile ring, chunked tensor stores per half
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=k + 5)
+    a = W.make_data(n)
+    b, info = run(P, p, a, layout=5)
+    assert info["passes"] == 3 and info["entry_bits"] == [25, 25, 25]
+    assert np.array_equal(b, OA.apply_ref(p, a)), (fam, k)

@@ -180,3 +180,23 @@ def test_cluster_path_rejects_unsupported_shapes(lib):
     assert e.value.status == -3
     with pytest.raises(lib.PermError):
         lib.Plan(W.random(1 << 16, 1), device=False, passes=2, cluster=3)
+
+
+@pytest.mark.parametrize("k,fam", [(20, "random"), (20, "bitrev"), (21, "transpose")])
+def test_product_tlc_ring_plan_checks_and_runs_on_the_oracle_executor(lib, k, fam):
+    # layout 5: TLC passes with 32768-word tiles run through the half-tile ring (the 2^26 /
+    # 2^27 structure), schedules in the ring's dense per-round format; exported per tile
+    n = 1 << k
+    p = W.make_perm(fam, n, seed=k)
+    with lib.Plan(p, device=False, layout=5, direct=-1) as pl:
+        info = pl.info()
+        d = pl.describe()
+        kappa, scheds = pl.export()
+    assert info["passes"] == 3 and d["layout"] == 5 and info["entry_bits"] == [25, 25, 25]
+    r, c, h = info["rows"], info["cols"], tuple(info["h"])
+    sched = [s.reshape(-1) for s in scheds]
+    assert _ok(OC.check_tlc(p, kappa.astype(np.int64), sched, r, c, h))
+    a = W.make_data(n)
+    b, st = OT.tlc_apply(a, sched, r, c, h)
+    assert np.array_equal(b, OA.apply_ref(p, a))
+    assert st["conflict_free"] == st["rounds"] == 3 * n // 32
