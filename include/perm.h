@@ -64,8 +64,12 @@ enum perm_passes {
 enum perm_layout {
     PERM_LAYOUT_AUTO  = 0,
     PERM_LAYOUT_TILED = 1,   /* reader transposes: X1, X2 stored as h1 x h2 / h3 x h2 tiles */
-    PERM_LAYOUT_LINES = 2    /* writer transposes: X1 column-major, X2 row-major; every pass
-                                reads whole lines with TMA bulk copies (persistent, pipelined) */
+    /* 2 (LINES) was removed in round 2 */
+    PERM_LAYOUT_TLC   = 3,   /* tile-level colouring: the transposes absorbed into the passes'
+                                X1 / X2 chunk layouts (default 2^18..2^25) */
+    PERM_LAYOUT_TLC_RING = 5 /* TLC with 32768-word tiles permuted in place through the
+                                half-tile ring (3 passes at 2^26 / 2^27; measured slower than
+                                the 5-pass default there, kept as an option) */
 };
 
 typedef struct {
