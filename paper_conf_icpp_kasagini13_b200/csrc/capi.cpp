@@ -287,8 +287,10 @@ int perm_apply_sharded(const perm_plan* plan, const void* a_shard, void* b_shard
     if (!P.r_l) return fail(PERM_EINVAL, "not a row-sharded plan (use perm_apply)");
     if (!plan->comm) return fail(PERM_ENCCL, "plan has no NCCL communicator (created without nccl_uid)");
     if (overlap(a_shard, b_shard, P.n / P.world * P.eb)) return fail(PERM_EINVAL, "a and b shards overlap");
-    // R1 + T-pack -> all-to-all -> R2 + T-pack -> all-to-all -> R3 (Lemma 8: the column
-    // phase's two transposes become the two uniform, P-independent exchanges)
+    // step 0 -> all-to-all -> step 1 -> all-to-all -> step 2 (Lemma 8: the column phase's two
+    // transposes become the two uniform, P-independent exchanges; in the TLC form the steps
+    // write / read the exchange layouts directly, in the per-line form steps 0 and 1 add a
+    // transpose)
     int st = perm_sharded_step(plan, 0, a_shard, plan->d_send, stream);
     if (st == PERM_OK) st = perm_sharded_exchange(plan, plan->d_send, plan->d_recv, stream);
     if (st == PERM_OK) st = perm_sharded_step(plan, 1, plan->d_recv, plan->d_send, stream);
@@ -321,7 +323,7 @@ int perm_sharded_step(const perm_plan* plan, int32_t step, const void* in, void*
         // (step 0: X1 of my rows = per-peer column blocks; step 1: X2 of my columns = per-peer
         // row blocks; step 2: rows of b) and reading received tiles as one segment per sender
         if (step < 0 || step > 2) return fail(PERM_EINVAL, "step must be 0, 1 or 2");
-        alignas(64) CUtensorMap maps[3];
+        alignas(64) CUtensorMap maps[3] = {};
         if (step < 2) {
             e = perm::make_tlc_maps(P, dst, dst, maps);
             if (e != cudaSuccess) return cuda_fail(e, "cuTensorMapEncodeTiled (sharded)");
