@@ -950,6 +950,9 @@ __device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long
 __device__ __forceinline__ void red_release_gpu_add(unsigned long long* p, unsigned long long v) {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void red_relaxed_gpu_add(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 
 // ------------------------------------------------------------------ TLC row pass (tile-level colouring)
 
@@ -1044,25 +1047,32 @@ __device__ __forceinline__ void tlc_permute(const uint32_t* __restrict__ A, uint
     const int lt = KIND == TLC_FULL ? LOGHL : dc.lt;
     const uint32_t tmask = KIND == TLC_FULL ? (uint32_t)(HL - 1) : (1u << dc.lt) - 1u;
     const int sh_line = dc.lt + dc.s4 - 5;    // TLC_X1: line index = e >> sh_line
-    uint32_t v[EPT];
-    uint32_t d[EPT];
+    // Beyond 16 elements per thread the tile is moved in groups of 16 (read 16, write 16),
+    // so that two tiles' schedule words + one group's values fit in 96 registers.
+    constexpr int GRP = EPT <= 16 ? EPT : 16;
+    uint32_t v[GRP];
+    uint32_t d[GRP];
 #pragma unroll
-    for (int m = 0; m < EPT; ++m) {
-        const int bit = m * E, w = bit >> 5, off = bit & 31;
-        uint32_t e;
-        if (off + E <= 32) e = (wc[w] >> off) & EMASK;
-        else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
-        const uint32_t t = e & tmask;
-        v[m] = A[((e >> lt) << 5) | (uint32_t)lane];
-        if constexpr (KIND == TLC_FULL) d[m] = t;
-        else if constexpr (KIND == TLC_X2) d[m] = (t << dc.s2) | lc;
-        else if constexpr (KIND == TLC_ROWS) d[m] = t | lc;
-        else d[m] = ((t >> dc.s1) << dc.s2) | ((e >> sh_line) << dc.s3) | (t & dc.m1);
+    for (int g0 = 0; g0 < EPT; g0 += GRP) {
+#pragma unroll
+        for (int j = 0; j < GRP; ++j) {
+            const int m = g0 + j;
+            const int bit = m * E, w = bit >> 5, off = bit & 31;
+            uint32_t e;
+            if (off + E <= 32) e = (wc[w] >> off) & EMASK;
+            else e = __funnelshift_r(wc[w], wc[w + 1], off) & EMASK;
+            const uint32_t t = e & tmask;
+            v[j] = A[((e >> lt) << 5) | (uint32_t)lane];
+            if constexpr (KIND == TLC_FULL) d[j] = t;
+            else if constexpr (KIND == TLC_X2) d[j] = (t << dc.s2) | lc;
+            else if constexpr (KIND == TLC_ROWS) d[j] = t | lc;
+            else d[j] = ((t >> dc.s1) << dc.s2) | ((e >> sh_line) << dc.s3) | (t & dc.m1);
+        }
+        if (g0 + GRP == EPT) mbar_arrive(aempty);     // A slot may be refilled
+        if (g0 == 0 && bempty_wait) mbar_wait(bempty_wait, bparity);
+#pragma unroll
+        for (int j = 0; j < GRP; ++j) B[d[j]] = v[j];
     }
-    mbar_arrive(aempty);                      // A slot may be refilled
-    if (bempty_wait) mbar_wait(bempty_wait, bparity);
-#pragma unroll
-    for (int m = 0; m < EPT; ++m) B[d[m]] = v[m];
     fence_proxy_async();                      // generic-proxy writes -> the TMA store's reads
 }
 
@@ -1165,7 +1175,9 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 }
                 if (i < 4) stamp_if(tr, true, 4 + 3 * i);
             }
+            stamp_if(tr, true, 12);           // last store issued
             bulk_wait0();
+            stamp_if(tr, true, 13);           // every store of this CTA complete
         }
     } else {
         // ---------------- permuters
@@ -1179,7 +1191,11 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         // (the intermediates X1 / X2 are what the next pass reads)
         const uint64_t pol_first = policy_evict_first();
         constexpr int AHEAD = NWORDS <= 12 ? 2 : 1;
-        uint32_t wq[AHEAD + 1][NWORDS];
+        constexpr int NBUF = AHEAD + 1;
+        // The buffers rotate by unrolling the tile loop NBUF times (compile-time buffer
+        // indices): copying a buffer that has loads in flight (wq[k] = wq[k + 1]) would
+        // stall every tile on the previous tile's schedule loads (an L2 round trip).
+        uint32_t wq[NBUF][NWORDS];
 #pragma unroll
         for (int k = 0; k < AHEAD; ++k) {
             const long long tk = blockIdx.x + (long long)k * G;
@@ -1188,24 +1204,30 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 for (int w = 0; w < NWORDS; ++w) wq[k][w] = ld_nc_hint(sp + tk * a.tile_words + w * 32, pol_first);
             }
         }
-        for (int i = 0;; ++i) {
-            const long long t = blockIdx.x + (long long)i * G;
-            if (t >= a.ntiles) break;
-            const int s = i % NA, sb = i % NB;
-            const long long tn = t + (long long)AHEAD * G;
-            if (tn < a.ntiles) {
+        int s = 0, sb = 0;                    // A / B slots of tile i
+        uint32_t pa = 0u, pb = 1u;            // afull parity of slot s, bempty parity of slot sb
+        for (int i0 = 0;; i0 += NBUF) {
+            bool done = false;
 #pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wq[AHEAD][w] = ld_nc_hint(sp + tn * a.tile_words + w * 32, pol_first);
+            for (int u = 0; u < NBUF; ++u) {
+                const int i = i0 + u;
+                const long long t = blockIdx.x + (long long)i * G;
+                if (t >= a.ntiles) { done = true; break; }
+                const long long tn = t + (long long)AHEAD * G;
+                if (tn < a.ntiles) {
+#pragma unroll
+                    for (int w = 0; w < NWORDS; ++w)
+                        wq[(u + AHEAD) % NBUF][w] = ld_nc_hint(sp + tn * a.tile_words + w * 32, pol_first);
+                }
+                mbar_wait(&R.afull[s], pa);
+                if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
+                tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wq[u], a.dec, lc,
+                                          &R.aempty[s], i >= NB ? &R.bempty[sb] : nullptr, pb, lane);
+                mbar_arrive(&R.bfull[sb]);
+                if (++s == NA) { s = 0; pa ^= 1u; }
+                if (++sb == NB) { sb = 0; pb ^= 1u; }
             }
-            mbar_wait(&R.afull[s], (uint32_t)(i / NA) & 1u);
-            if (i < 4) stamp_if(tr, lead, 2 + 3 * i);
-            tlc_permute<EPT, E, KIND>(R.A + (size_t)s * HL, R.B + (size_t)sb * HL, wq[0], a.dec, lc, &R.aempty[s],
-                                      i >= NB ? &R.bempty[sb] : nullptr, (uint32_t)(i / NB - 1) & 1u, lane);
-            mbar_arrive(&R.bfull[sb]);
-#pragma unroll
-            for (int k = 0; k < AHEAD; ++k)
-#pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wq[k][w] = wq[k + 1][w];
+            if (done) break;
         }
         stamp_if(tr, lead, 3);
     }
@@ -1251,9 +1273,14 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     const int NA = a.na, NB = a.nb;
     const int G = gridDim.x;
     TlcRing R(smem, HL, NA, NB);
+    uint64_t* pdone = R.bempty + NB;   // [k]: this CTA's pass-k stores are complete and published
     unsigned long long* tr = a.trace;
     stamp(tr, 0);
-    if (tid == 0) R.init(NA, NB);
+    if (tid == 0) {
+        mbar_init(&pdone[0], 1);
+        mbar_init(&pdone[1], 1);
+        R.init(NA, NB);
+    }
     __syncthreads();
     auto my_tiles = [&](int k) -> int {
         const int nt = a.p[k].ntiles - (int)blockIdx.x;
@@ -1263,21 +1290,26 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
     if (warp == 0) {
         if (lane == 0) {
             // ---------------- producer
-            // every schedule of this CTA is independent of the data: pass 0's is requested
-            // first, passes 1 and 2 right after the first ring of pass-0 loads
-            auto prefetch_sched = [&](int k) {
-                for (int i = 0; i < my_tiles(k); ++i)
+            // Schedules are independent of the data. Pass 0 (HBM input): the first two tiles'
+            // schedules go ahead, the rest interleave behind the data loads, input tiles beyond
+            // the ring are streamed into L2. Pass k + 1's schedules are requested once this
+            // CTA's last pass-k tile has landed (HBM free of this CTA's pass-k traffic), ahead of
+            // the grid barrier.
+            auto prefetch_one = [&](int k, int i) {
+                if (i < my_tiles(k))
                     prefetch_l2_bulk(a.p[k].sched + (blockIdx.x + (long long)i * G) * a.tile_words,
                                      (uint32_t)(a.tile_words * 4));
             };
-            prefetch_sched(0);
-            const int first_ring = my_tiles(0) < NA ? my_tiles(0) : NA;
-            if (first_ring == 0) { prefetch_sched(1); prefetch_sched(2); }
+            prefetch_one(0, 0);
+            prefetch_one(0, 1);
             int j = 0;
             for (int k = 0; k < 3; ++k) {
                 const TlcPassCfg& pc = a.p[k];
                 const int nt = my_tiles(k);
                 if (k > 0) {
+                    // poll the grid counter only once this CTA has arrived (polling one L2 line
+                    // from every SM during the whole pass slows the pass's own traffic)
+                    mbar_wait(&pdone[k - 1], 0);
                     while (ld_acquire_gpu(&a.sync[k - 1]) < (unsigned long long)G) __nanosleep(32);
                     fence_proxy_async_global();
                     stamp(tr, 1 + 4 * k);
@@ -1289,7 +1321,16 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                     fence_proxy_async();       // permuters' generic reads of the slot -> TMA write
                     mbar_arrive_expect_tx(&R.afull[s], (uint32_t)HL * 4u);
                     bulk_g2s(R.A + (size_t)s * HL, pc.in + t * HL, (uint32_t)HL * 4u, &R.afull[s]);
-                    if (k == 0 && i + 1 == first_ring) { prefetch_sched(1); prefetch_sched(2); }
+                    if (k == 0) {
+                        prefetch_one(0, i + 2);
+                        if (i + 1 == NA)       // pass-0 input tiles beyond the ring: into L2 now
+                            for (int q = NA; q < nt; ++q)
+                                prefetch_l2_bulk(pc.in + (blockIdx.x + (long long)q * G) * HL, (uint32_t)HL * 4u);
+                    }
+                }
+                if (k < 2) {
+                    if (nt > 0) mbar_wait(&R.afull[(j - 1) % NA], (uint32_t)((j - 1) / NA) & 1u);
+                    for (int i = 0; i < my_tiles(k + 1); ++i) prefetch_one(k + 1, i);
                 }
             }
         }
@@ -1321,13 +1362,15 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 }
                 if (k < 2) {
                     bulk_wait0();                    // this CTA's pass-k output is written
+                    if (k == 0) stamp_if(tr, true, 14);
                     if (prev >= 0) {
                         mbar_arrive(&R.bempty[prev]);
                         prev = -1;
                     }
-                    fence_proxy_async_global();
-                    __threadfence();
-                    red_release_gpu_add(&a.sync[k], 1ull);
+                    fence_proxy_async_global();      // async-proxy writes -> the generic release
+                    if (k == 0) stamp_if(tr, true, 13);
+                    red_relaxed_gpu_add(&a.sync[k], 1ull);
+                    mbar_arrive(&pdone[k]);
                     stamp_if(tr, true, 4 + 4 * k);
                 }
             }
@@ -1335,45 +1378,64 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
         }
     } else {
         // ---------------- permuters
+        // One flat sequence of this CTA's tiles over the three passes (j -> pass k, tile i):
+        // schedule words are loaded AHEAD tiles ahead, across pass boundaries (they do not
+        // depend on the data), into NBUF register buffers rotated by unrolling.
         const bool lead = tid == 64;
-        int j = 0;
-        for (int k = 0; k < 3; ++k) {
-            const TlcPassCfg& pc = a.p[k];
-            const int nt = my_tiles(k);
-            const uint32_t lc = tlc_lane_const(pc.kind == 1 ? TLC_X1 : (pc.kind == 2 ? TLC_X2 : TLC_ROWS),
-                                               pc.dec, lane);
-            const uint32_t* sp = pc.sched + (warp - 2) * NWORDS * 32 + lane;
-            uint32_t wc[NWORDS], wn[NWORDS];
-            if (nt > 0) {
+        const int nt0 = my_tiles(0), nt1 = my_tiles(1), nt2 = my_tiles(2);
+        const int J = nt0 + nt1 + nt2;
+        const uint64_t pol_first = policy_evict_first();
+        constexpr int AHEAD = NWORDS <= 12 ? 2 : 1;
+        constexpr int NBUF = AHEAD + 1;
+        auto locate = [&](int jj, int& k, int& i) {
+            k = jj < nt0 ? 0 : (jj < nt0 + nt1 ? 1 : 2);
+            i = jj - (k == 0 ? 0 : (k == 1 ? nt0 : nt0 + nt1));
+        };
+        uint32_t wq[NBUF][NWORDS];
+        auto load_words = [&](int jj, uint32_t* dstw) {
+            int k, i;
+            locate(jj, k, i);
+            const uint32_t* sp = a.p[k].sched + (blockIdx.x + (long long)i * G) * a.tile_words +
+                                 (warp - 2) * NWORDS * 32 + lane;
 #pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wc[w] = __ldg(sp + (long long)blockIdx.x * a.tile_words + w * 32);
-            }
-            for (int i = 0; i < nt; ++i, ++j) {
-                const int s = j % NA, sb = j % NB;
-                if (i + 1 < nt) {
-                    const long long tn = blockIdx.x + (long long)(i + 1) * G;
+            for (int w = 0; w < NWORDS; ++w) dstw[w] = ld_nc_hint(sp + w * 32, pol_first);
+        };
 #pragma unroll
-                    for (int w = 0; w < NWORDS; ++w) wn[w] = __ldg(sp + tn * a.tile_words + w * 32);
-                }
-                mbar_wait(&R.afull[s], (uint32_t)(j / NA) & 1u);
+        for (int q = 0; q < AHEAD; ++q)
+            if (q < J) load_words(q, wq[q]);
+        int s = 0, sb = 0;
+        uint32_t pa = 0u, pb = 1u;
+        for (int j0 = 0; j0 < J; j0 += NBUF) {
+#pragma unroll
+            for (int u = 0; u < NBUF; ++u) {
+                const int jj = j0 + u;
+                if (jj >= J) break;
+                if (jj + AHEAD < J) load_words(jj + AHEAD, wq[(u + AHEAD) % NBUF]);
+                int k, i;
+                locate(jj, k, i);
+                const TlcPassCfg& pc = a.p[k];
+                mbar_wait(&R.afull[s], pa);
                 if (i == 0) stamp_if(tr, lead, 2 + 4 * k);
                 uint32_t* const Bs = R.B + (size_t)sb * HL;
                 const uint32_t* const As = R.A + (size_t)s * HL;
-                uint64_t* const bw = j >= NB ? &R.bempty[sb] : nullptr;
-                const uint32_t bp = (uint32_t)(j / NB - 1) & 1u;
-                if (E == 2 * cilog2(HL) - 5)
-                    tlc_permute<EPT, E, TLC_FULL>(As, Bs, wc, pc.dec, 0u, &R.aempty[s], bw, bp, lane);
-                else if (pc.kind == 1)
-                    tlc_permute<EPT, E, TLC_X1>(As, Bs, wc, pc.dec, lc, &R.aempty[s], bw, bp, lane);
-                else if (pc.kind == 2)
-                    tlc_permute<EPT, E, TLC_X2>(As, Bs, wc, pc.dec, lc, &R.aempty[s], bw, bp, lane);
-                else
-                    tlc_permute<EPT, E, TLC_ROWS>(As, Bs, wc, pc.dec, lc, &R.aempty[s], bw, bp, lane);
+                uint64_t* const bw = jj >= NB ? &R.bempty[sb] : nullptr;
+                if constexpr (E == 2 * cilog2(HL) - 5) {
+                    tlc_permute<EPT, E, TLC_FULL>(As, Bs, wq[u], pc.dec, 0u, &R.aempty[s], bw, pb, lane);
+                } else {
+                    const int kind = pc.kind == 1 ? TLC_X1 : (pc.kind == 2 ? TLC_X2 : TLC_ROWS);
+                    const uint32_t lc = tlc_lane_const(kind, pc.dec, lane);
+                    if (kind == TLC_X1)
+                        tlc_permute<EPT, E, TLC_X1>(As, Bs, wq[u], pc.dec, lc, &R.aempty[s], bw, pb, lane);
+                    else if (kind == TLC_X2)
+                        tlc_permute<EPT, E, TLC_X2>(As, Bs, wq[u], pc.dec, lc, &R.aempty[s], bw, pb, lane);
+                    else
+                        tlc_permute<EPT, E, TLC_ROWS>(As, Bs, wq[u], pc.dec, lc, &R.aempty[s], bw, pb, lane);
+                }
                 mbar_arrive(&R.bfull[sb]);
-#pragma unroll
-                for (int w = 0; w < NWORDS; ++w) wc[w] = wn[w];
+                if (i == (k == 0 ? nt0 : (k == 1 ? nt1 : nt2)) - 1) stamp_if(tr, lead, 3 + 4 * k);
+                if (++s == NA) { s = 0; pa ^= 1u; }
+                if (++sb == NB) { sb = 0; pb ^= 1u; }
             }
-            stamp_if(tr, lead, 3 + 4 * k);
         }
     }
     __syncthreads();
@@ -1845,7 +1907,8 @@ cudaError_t grid_tma(HostPlan& P, int f) {
 
 size_t tlc_smem(const HostPlan& P, int f) {
     const TlcPass& tp = P.tp[f];
-    return (size_t)(tp.stages + tp.bslots) * tp.HL * 4 + (size_t)(tp.stages + tp.bslots) * 8 * 2;
+    // + 2 mbarriers of the fused kernel (pass k stored by this CTA)
+    return (size_t)(tp.stages + tp.bslots) * tp.HL * 4 + (size_t)(tp.stages + tp.bslots) * 8 * 2 + 16;
 }
 
 // Calls f(EPT, E) (std::integral_constant) for the compiled (elements per thread,

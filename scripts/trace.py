@@ -35,6 +35,7 @@ if d.get('fused3'):
     fn = {0: 'start'}
     for k in range(3):
         fn.update({1 + 4 * k: f'P{k}data', 2 + 4 * k: f'P{k}perm0', 3 + 4 * k: f'P{k}permEnd', 4 + 4 * k: f'P{k}storeEnd'})
+    fn[13] = 'P0proxyFence'; fn[14] = 'P0bulkWait0'
     fn[15] = 'end'
     for c in sorted(fn):
         v = rel[:, c][t[:, c] > 0]
@@ -42,7 +43,8 @@ if d.get('fused3'):
             print(f"  {fn[c]:>12}: min {v.min():7.2f}  med {np.median(v):7.2f}  max {v.max():7.2f}  (n={v.size})")
     sys.exit(0)
 if d.get('layout') == 3:
-    names = {0: 'start', 1: 'pdl_ok', 2: 'w0', 4: 's0', 5: 'w1', 7: 's1', 8: 'w2', 10: 's2', 3: 'permEnd', 14: 'end'}
+    names = {0: 'start', 1: 'pdl_ok', 2: 'w0', 4: 's0', 5: 'w1', 7: 's1', 8: 'w2', 10: 's2', 3: 'permEnd', 12: 'sLast',
+             13: 'drained', 14: 'end'}
 for f in range(3):
     t = tr[f]
     t = t[(t[:, 0] > 0)]
