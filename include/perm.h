@@ -97,10 +97,11 @@ typedef struct {
                             permutation, block permutations), reading n/32 block indices */
     int32_t log2c;       /* view r x c with c = 2^log2c (the view "is not
                             restricted to a square matrix"); 0 = c = 2^ceil(k/2) */
-    int32_t sched_format; /* TLC layout entry format: 0 = full (source row << log2(tile) |
+    int32_t sched_format; /* TLC layout entry format: -1 = full (source row << log2(tile) |
                              destination); 1 = compact (the line index inside the tile is implied
                              by the source offset: 19 instead of 21 bits at n = 2^22) wherever a
-                             kernel is compiled for its width (not with fuse = 1).
+                             kernel is compiled for its width (not with fuse = 1); 0 = compact
+                             from n = 2^23 on, full below (measured).
                              5-pass per-line schedules: 0 = dense bitstreams (E bits per entry)
                              for lines of 16384 words (the schedule-from-global slots), W64
                              elsewhere; 2 = dense for every line length; -1 = W64 everywhere */

@@ -581,9 +581,11 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
         // the kernels take pass 2's and pass 3's line index from the lane alone (free decode):
         // needs h2 <= 32 (pass 2) and h2 * h3 <= 32 (pass 3)
         const bool lane_line = (f != 1 || hs[1] <= kW) && (f != 2 || hs[1] * hs[2] <= kW);
-        // (measured on B200: no faster than the full format at 2^22..2^25, so opt-in)
+        // default (0): compact from n = 2^23 on (B200, cold L2: 2^23 41.7 -> 40.6 us, 2^24 85.0 ->
+        // 84.4, 2^25 185.5 -> 181.3; equal at 2^22, profiles/r02b_compact_ab.log); -1: full
         const bool fused_req = opt && opt->fuse > 0;
-        if (cmp_opt > 0 && !fused_req && tlc_compact_supported(tp.ept, Ec) && lane_line) {
+        const bool want_compact = cmp_opt > 0 || (cmp_opt == 0 && r * c >= (int64_t(1) << 23));
+        if (want_compact && !fused_req && tlc_compact_supported(tp.ept, Ec) && lane_line) {
             const int lh1 = ilog2(hs[0]), lh2 = ilog2(hs[1]), lc = ilog2(P.c);
             d.lt = logL;
             if (f == 0) {          // dst = ((k/h2)*h1 + i_in)*h2 + k%h2, i_in = src >> log c

@@ -209,7 +209,7 @@ def test_tlc_full_and_compact_formats_agree(lib, k):
     n = 1 << k
     r, c = W.view_shape(n)
     p = W.make_perm("random", n, seed=k)
-    i_full, _, kappa_f, s_full = export_tlc(lib, p, sched_format=0)
+    i_full, _, kappa_f, s_full = export_tlc(lib, p, sched_format=-1)
     i_cmp, _, kappa_c, s_cmp = export_tlc(lib, p, sched_format=1)
     assert np.array_equal(kappa_f, kappa_c)
     for a, b in zip(s_full, s_cmp):
