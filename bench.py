@@ -623,6 +623,40 @@ def main():
                                                          events_between_ms)),
                 "timing": timing_method}
 
+    # ---- where the apply's time goes: per-pass spans of one traced apply (globaltimer stamps
+    # of every CTA; pass k from its first CTA's start (k = 0) / its grid-dependency release
+    # (k > 0) to its last CTA's drained stores). At 2^22 the intermediates stay in the
+    # 126 MB L2, so passes 2 and 3 are compared with the measured L2 copy bandwidth
+    # (profiles/l2_bw.json) over the bytes they move through L2 (in + out + schedule).
+    in_apply = None
+    if info["passes"] == 3 and info["kernels_per_apply"] == 3 and not info["direct"]:
+        pl = plans[sched_fams[0]]
+        f0 = sched_fams[0]
+        pl.set_tracing(True)
+        flush_l2()
+        pl.apply(dA[f0], dB[f0], stream)
+        torch.cuda.synchronize()
+        tr = pl.trace().astype(np.int64)
+        pl.set_tracing(False)
+        l2ref = None
+        lpath = os.path.join(ROOT, "profiles", "l2_bw.json")
+        if os.path.exists(lpath):
+            with open(lpath) as fh:
+                l2ref = json.load(fh).get("copy_warm_16MiB_gbs")
+        t0 = tr[0][:, 0][tr[0][:, 0] > 0].min()
+        passes_info = {}
+        for k in range(3):
+            tk = tr[k][tr[k][:, 0] > 0]
+            begin = tk[:, 0].min() if k == 0 else tk[:, 1].min()
+            span_us = (tk[:, 13].max() - begin) / 1e3
+            byts = alg[k]
+            passes_info[kinds[k]] = {"begin_us": (begin - t0) / 1e3, "span_us": span_us, "bytes": byts,
+                                     "gbs": byts / (span_us * 1e-6) / 1e9,
+                                     "frac_hbm": byts / (span_us * 1e-6) / 1e9 / peaks["hbm_gbs"],
+                                     "frac_l2_copy": (byts / (span_us * 1e-6) / 1e9 / l2ref) if l2ref else None}
+        in_apply = {"family": f0, "kernel_span_us": (tr[2][:, 13].max() - t0) / 1e3, "passes": passes_info,
+                    "l2_copy_gbs": l2ref, "timing": "globaltimer stamps of one traced apply, cold L2"}
+
     # ---- end to end through the C ABI with host buffers
     e2e = None
     if not args.no_e2e:
@@ -700,6 +734,7 @@ def main():
             "sched_bytes": info["sched_bytes"],
             "bitexact_check": ok,
             "roofline": roofline,
+            "in_apply_passes": in_apply,
             "c3_2pow26_random": c3,
             "cpu_baseline": cpu,
             "e2e": e2e,
