@@ -38,6 +38,8 @@ namespace {
 
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
+__host__ __device__ constexpr int cilog2(int v) { return v <= 1 ? 0 : 1 + cilog2(v >> 1); }
+
 __device__ __forceinline__ void pdl_wait() {
     asm volatile("griddepcontrol.wait;" ::: "memory");
 }
@@ -775,9 +777,13 @@ __global__ void __launch_bounds__(kStgWorkers, 1)
     constexpr int NB = DENSE ? 5 : 4;            // chunk ring depth
     constexpr int CWS = DENSE ? kStgDenseWords : kStgChunkWords;   // buffer stride (words)
     const int tid = threadIdx.x;
-    const int L = 1 << a.r.logL, HALF = L >> 1, lh = a.r.logL - 1, hmask = HALF - 1;
-    const int E = a.r.E;
-    const int CW = DENSE ? 64 * E : kStgChunkWords;                 // words per chunk
+    // geometry from EPT (one line of L = 512 * EPT words per CTA; entries of the full
+    // per-line format, E = 2 log2 L - 5 bits; launch_row_pass checks the plan agrees):
+    // compile-time shifts and masks in the decode and the half-slot addressing
+    constexpr int LOGL = cilog2(kStgWorkers * EPT);
+    constexpr int L = 1 << LOGL, HALF = L >> 1, lh = LOGL - 1, hmask = HALF - 1;
+    constexpr int E = 2 * LOGL - 5;
+    constexpr int CW = DENSE ? 64 * E : kStgChunkWords;             // words per chunk
     uint32_t* cbuf = smem + 3 * HALF;
     uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + NB * CWS);
     uint64_t* full = bars + 3;                   // chunk landed
@@ -789,7 +795,7 @@ __global__ void __launch_bounds__(kStgWorkers, 1)
     const long long my_lines = a.ntiles > (int)blockIdx.x ? (a.ntiles - 1 - (int)blockIdx.x) / G + 1 : 0;
     constexpr int kW = kStgWorkers / 32;                   // warps
     const int w64 = a.r.w64;
-    const int chunks_per_line = EPT / 4;         // (L/32 rounds) / 64 rounds per chunk
+    constexpr int chunks_per_line = EPT / 4;     // (L/32 rounds) / 64 rounds per chunk
 
     // half q of line i -> slot j % 3. With the first half, the line's second half is pulled
     // into L2: its TMA load can only be issued once the previous line's first half has been
@@ -832,15 +838,14 @@ __global__ void __launch_bounds__(kStgWorkers, 1)
     }
     __syncthreads();
     const long long total_chunks = my_lines * chunks_per_line;
-    auto issue_chunk = [&](long long g) {
-        const int b = (int)(g % NB);
+    auto issue_chunk = [&](long long g, int b) {      // b = g % NB
         const long long i = g / chunks_per_line, c = g - i * chunks_per_line;
         const long long t = blockIdx.x + i * G;
         mbar_arrive_expect_tx(&full[b], (uint32_t)CW * 4u);
         bulk_g2s(cbuf + b * CWS, a.r.sched + t * a.sched_words + c * CW, (uint32_t)CW * 4u, &full[b]);
     };
     if (tid == 0)
-        for (long long g = 0; g < NB && g < total_chunks; ++g) issue_chunk(g);
+        for (long long g = 0; g < NB && g < total_chunks; ++g) issue_chunk(g, (int)g);
     pdl_wait();
     stamp(tr, 1);
     if (tid == 0) {
@@ -851,10 +856,18 @@ __global__ void __launch_bounds__(kStgWorkers, 1)
     pdl_launch_dependents();
     const int lane = tid & 31, warp = tid >> 5;
     const SchedDec dec(DENSE ? 1 : 0, E, a.r.epw, w64, lane);
-    const uint32_t tmask = (1u << a.r.logL) - 1u;
-    const int logL = a.r.logL;
+    constexpr uint32_t tmask = (1u << LOGL) - 1u;
+    constexpr uint32_t EMASK = (1u << E) - 1u;
+    constexpr int logL = LOGL;
     constexpr int MPC = 4;               // m-steps per chunk: 64 rounds = 4 x 16 warps
     constexpr int CPL = EPT / MPC;       // chunks per line
+    // dense entries: the lane's entry of round q of a chunk starts at bit lane*E of the
+    // round's E words: words dwo, dwo2 (= dwo or dwo + 1) at warp*E (+ 16*E per m-step)
+    const int lane_w0 = warp * E + dec.dwo, lane_w1 = warp * E + dec.dwo2;
+    const uint32_t lane_sh = (uint32_t)dec.dbo;
+    long long g = 0;                     // this CTA's chunk sequence number
+    int cb_i = 0;                        // g % NB
+    uint32_t cb_ph = 0;                  // (g / NB) & 1
     for (long long i = 0; i < my_lines; ++i) {
         const long long t = blockIdx.x + i * G;
         const long long j0 = 2 * i, j1 = 2 * i + 1;
@@ -866,15 +879,20 @@ __global__ void __launch_bounds__(kStgWorkers, 1)
         uint32_t v[EPT];
         uint32_t ta[EPT / 2];
 #pragma unroll
-        for (int c = 0; c < CPL; ++c) {
-            const long long g = i * CPL + c;
-            const int b = (int)(g % NB);
-            mbar_wait(&full[b], (uint32_t)((g / NB) & 1));
+        for (int c = 0; c < CPL; ++c, ++g) {
+            const int b = cb_i;
+            mbar_wait(&full[b], cb_ph);
             const uint32_t* cb = cbuf + b * CWS;
 #pragma unroll
             for (int mm = 0; mm < MPC; ++mm) {
                 const int m = c * MPC + mm;
-                const uint32_t e = dec.get<true>(cb, warp + kW * mm);
+                uint32_t e;
+                if constexpr (DENSE) {
+                    const uint32_t lo = cb[lane_w0 + mm * kW * E], hi = cb[lane_w1 + mm * kW * E];
+                    e = __funnelshift_r(lo, hi, lane_sh) & EMASK;
+                } else {
+                    e = dec.get<true>(cb, warp + kW * mm);
+                }
                 const int s = (int)((e >> logL) << 5) + lane;
                 v[m] = smem[((s >> lh) ? o1 : o0) + (s & hmask)];
                 const int tt = (int)(e & tmask);
@@ -897,9 +915,10 @@ __global__ void __launch_bounds__(kStgWorkers, 1)
                              : "=r"(old) : "r"(smem_u32(&consumed[b])) : "memory");
                 if ((old + 1) % kW == 0) {       // the last of the 16 warps to consume chunk g
                     fence_proxy_async();         // all warps' generic reads -> the TMA refill
-                    issue_chunk(g + NB);
+                    issue_chunk(g + NB, b);
                 }
             }
+            if (++cb_i == NB) { cb_i = 0; cb_ph ^= 1u; }
         }
         __syncthreads();
 #pragma unroll
@@ -957,7 +976,6 @@ __device__ __forceinline__ void red_relaxed_gpu_add(unsigned long long* p, unsig
 // ------------------------------------------------------------------ TLC row pass (tile-level colouring)
 
 
-__host__ __device__ constexpr int cilog2(int v) { return v <= 1 ? 0 : 1 + cilog2(v >> 1); }
 
 struct TlcArgs {
     const uint32_t* in;
@@ -2269,6 +2287,9 @@ cudaError_t launch_row_pass(const HostPlan& P, int f, const uint32_t* sched, con
         const bool sg = rp.sg != 0;
         if (rp.split && rp.split_stg) {
             const bool dn = g.dense != 0;
+            // the kernel derives its geometry from EPT (one line of 512 * EPT words per CTA)
+            if ((int64_t(kStgWorkers) * rp.ept != (int64_t(1) << g.logL)) || g.E != 2 * g.logL - 5)
+                return cudaErrorInvalidValue;
             CUtensorMap m{};
             if (map) m = *map;
             if (P.layout == 5 && P.tp[f].out_kind != 0) {
