@@ -1325,9 +1325,9 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 const TlcPassCfg& pc = a.p[k];
                 const int nt = my_tiles(k);
                 if (k > 0) {
-                    // poll the grid counter only once this CTA has arrived (polling one L2 line
-                    // from every SM during the whole pass slows the pass's own traffic)
-                    mbar_wait(&pdone[k - 1], 0);
+                    // poll the grid counter only once this CTA has arrived (pdone[k - 1] was
+                    // waited on at the end of pass k - 1; polling one L2 line from every SM
+                    // during the whole pass slows the pass's own traffic)
                     while (ld_acquire_gpu(&a.sync[k - 1]) < (unsigned long long)G) __nanosleep(32);
                     fence_proxy_async_global();
                     stamp(tr, 1 + 4 * k);
@@ -1347,7 +1347,9 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                     }
                 }
                 if (k < 2) {
-                    if (nt > 0) mbar_wait(&R.afull[(j - 1) % NA], (uint32_t)((j - 1) / NA) & 1u);
+                    // pass k + 1's schedules once this CTA's pass-k stores are complete: HBM is
+                    // then free of this CTA's pass-k traffic, and the prefetch overlaps the barrier
+                    mbar_wait(&pdone[k], 0);
                     for (int i = 0; i < my_tiles(k + 1); ++i) prefetch_one(k + 1, i);
                 }
             }
@@ -1428,7 +1430,6 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
             for (int u = 0; u < NBUF; ++u) {
                 const int jj = j0 + u;
                 if (jj >= J) break;
-                if (jj + AHEAD < J) load_words(jj + AHEAD, wq[(u + AHEAD) % NBUF]);
                 int k, i;
                 locate(jj, k, i);
                 const TlcPassCfg& pc = a.p[k];
@@ -1450,6 +1451,10 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                         tlc_permute<EPT, E, TLC_ROWS>(As, Bs, wq[u], pc.dec, lc, &R.aempty[s], bw, pb, lane);
                 }
                 mbar_arrive(&R.bfull[sb]);
+                // look-ahead AFTER the permute's proxy fence (MEMBAR.CTA waits for every
+                // outstanding load of the thread; across a pass boundary the next pass's words
+                // come from HBM and would stall the last tiles of the pass)
+                if (jj + AHEAD < J) load_words(jj + AHEAD, wq[(u + AHEAD) % NBUF]);
                 if (i == (k == 0 ? nt0 : (k == 1 ? nt1 : nt2)) - 1) stamp_if(tr, lead, 3 + 4 * k);
                 if (++s == NA) { s = 0; pa ^= 1u; }
                 if (++sb == NB) { sb = 0; pb ^= 1u; }
