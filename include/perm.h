@@ -196,6 +196,16 @@ int perm_apply(const perm_plan* plan, const void* a, void* b, perm_stream_t stre
  * memory gives asynchronous copies; pageable memory works but is slower. */
 int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream);
 
+/* perm_apply_host without the final synchronisation: the H2D copy, the apply and the D2H
+ * copy are only enqueued on `stream`, so applies of DIFFERENT plans on different streams
+ * overlap one plan's device->host copy with the next one's host->device copy (the copy
+ * engines of the two directions run concurrently). a_host / b_host must be pinned, must
+ * stay valid and a_host unmodified until the stream is synchronised, and b_host holds the
+ * result only after that. The plan's staging buffers are reused by every call: two calls
+ * on the SAME plan must be on the same stream. Errors as perm_apply_host; device faults
+ * surface at the caller's synchronisation. */
+int perm_apply_host_async(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream);
+
 /* Per-kernel timing: when enabled, perm_apply records a CUDA event before its
  * first kernel and after each kernel on the launch stream. perm_plan_pass_times
  * waits for the last event and writes up to max_k kernel durations (ms) of the

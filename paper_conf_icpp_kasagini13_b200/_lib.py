@@ -89,6 +89,7 @@ _plan_describe = _sig("perm_plan_describe", _i64, _vp, ctypes.c_char_p, _i64)
 _plan_export = _sig("perm_plan_export", ctypes.c_int, _vp, _vp, _vp, _vp, _vp)
 _apply = _sig("perm_apply", ctypes.c_int, _vp, _vp, _vp, _vp)
 _apply_host = _sig("perm_apply_host", ctypes.c_int, _vp, _vp, _vp, _vp)
+_apply_host_async = _sig("perm_apply_host_async", ctypes.c_int, _vp, _vp, _vp, _vp)
 _set_prof = _sig("perm_plan_set_profiling", ctypes.c_int, _vp, ctypes.c_int)
 _pass_times = _sig("perm_plan_pass_times", ctypes.c_int, _vp, ctypes.POINTER(ctypes.c_float), ctypes.c_int)
 _set_tracing = _sig("perm_plan_set_tracing", ctypes.c_int, _vp, ctypes.c_int)
@@ -277,6 +278,17 @@ class Plan:
             if nb != self.nbytes or getattr(x, "is_cuda", False):
                 raise PermError(-1, f"{what}: host buffer of {self.nbytes} bytes expected")
         _check(_apply_host(self._h, _ptr(a_host), _ptr(b_host), _stream_handle(stream)))
+        return b_host
+
+    def apply_host_async(self, a_host, b_host, stream=None):
+        """perm_apply_host_async: enqueue H2D, apply, D2H on `stream` without synchronising.
+        a_host / b_host must be pinned torch tensors (checked); b_host is valid after the
+        stream is synchronised. Calls on the same plan must share one stream."""
+        for x, what in ((a_host, "a_host"), (b_host, "b_host")):
+            if not hasattr(x, "is_pinned") or not x.is_pinned() or \
+                    x.numel() * x.element_size() != self.nbytes:
+                raise PermError(-1, f"{what}: pinned host tensor of {self.nbytes} bytes expected")
+        _check(_apply_host_async(self._h, _ptr(a_host), _ptr(b_host), _stream_handle(stream)))
         return b_host
 
     def sharded_step(self, step: int, inp, out, stream=None):

@@ -671,7 +671,8 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
     return PERM_OK;
 }
 
-int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream) {
+namespace {
+int apply_host_impl(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream, bool sync) {
     if (!plan || !a_host || !b_host) return fail(PERM_EINVAL, "null plan or buffer");
     if (!plan->on_device) return fail(PERM_ENODEVICE, "plan was created host-only");
     if (plan->host.r_l) return fail(PERM_EINVAL, "row-sharded plan: use perm_apply_sharded or perm_sharded_step");
@@ -690,9 +691,20 @@ int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stre
     if (st != PERM_OK) return st;
     e = cudaMemcpyAsync(b_host, plan->d_stage[1], bytes, cudaMemcpyDeviceToHost, s);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpyAsync D2H");
-    e = cudaStreamSynchronize(s);
-    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+    if (sync) {
+        e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+    }
     return PERM_OK;
+}
+}  // namespace
+
+int perm_apply_host(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream) {
+    return apply_host_impl(plan, a_host, b_host, stream, true);
+}
+
+int perm_apply_host_async(perm_plan* plan, const void* a_host, void* b_host, perm_stream_t stream) {
+    return apply_host_impl(plan, a_host, b_host, stream, false);
 }
 
 int perm_scatter_baseline(const int32_t* p_dev, const void* a, void* b, int64_t n,

@@ -180,6 +180,33 @@ def test_apply_host_e2e(P):
     assert np.array_equal(b, OA.apply_ref(p, a))
 
 
+def test_apply_host_async_two_streams(P):
+    # perm_apply_host_async: several plans' host round trips enqueued on two streams
+    # (copy engines of both directions overlap), results valid after the synchronisation
+    ks = [(20, "random"), (21, "bitrev"), (22, "transpose"), (22, "random")]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    plans, bufs, refs = [], [], []
+    for i, (k, fam) in enumerate(ks):
+        n = 1 << k
+        p = W.make_perm(fam, n, seed=30 + i)
+        a = W.make_data(n, seed=60 + i)
+        ha = torch.from_numpy(a.view(np.int32)).pin_memory()
+        hb = torch.empty(n, dtype=torch.int32).pin_memory()
+        plans.append(P.Plan(p))
+        bufs.append((ha, hb))
+        refs.append(OA.apply_ref(p, a))
+    for i, pl in enumerate(plans):
+        pl.apply_host_async(bufs[i][0], bufs[i][1], streams[i % 2])
+    torch.cuda.synchronize()
+    for i, pl in enumerate(plans):
+        assert np.array_equal(bufs[i][1].numpy().view(np.uint32), refs[i]), ks[i]
+        pl.close()
+    with pytest.raises(P.PermError):          # pageable memory is refused by the binding
+        with P.Plan(W.random(1 << 12, 1)) as pl:
+            x = torch.zeros(1 << 12, dtype=torch.int32)
+            pl.apply_host_async(x, x.clone())
+
+
 def test_profiling_pass_times(P):
     n = 1 << 22
     with P.Plan(W.random(n, 1)) as plan:
