@@ -1944,6 +1944,7 @@ cudaError_t tlc_dispatch(int ept, int E, F&& f) {
     if (ept == 16) {
         switch (E) {
             case 21: return f(integral_constant<int, 16>{}, integral_constant<int, 21>{});
+            case 20: return f(integral_constant<int, 16>{}, integral_constant<int, 20>{});
             case 19: return f(integral_constant<int, 16>{}, integral_constant<int, 19>{});
             case 18: return f(integral_constant<int, 16>{}, integral_constant<int, 18>{});
             case 17: return f(integral_constant<int, 16>{}, integral_constant<int, 17>{});
@@ -1952,6 +1953,7 @@ cudaError_t tlc_dispatch(int ept, int E, F&& f) {
         }
     }
     if (ept == 32 && E == 23) return f(integral_constant<int, 32>{}, integral_constant<int, 23>{});
+    if (ept == 32 && E == 22) return f(integral_constant<int, 32>{}, integral_constant<int, 22>{});
     if (ept == 32 && E == 21) return f(integral_constant<int, 32>{}, integral_constant<int, 21>{});
     return cudaErrorInvalidValue;
 }

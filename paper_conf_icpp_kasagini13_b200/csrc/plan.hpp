@@ -118,7 +118,7 @@ inline uint32_t tlc_dst(const TlcDecode& d, uint32_t t, uint32_t src) {
 }
 // (elements per permuter thread, compact entry bits) pairs with a compiled kernel
 inline bool tlc_compact_supported(int ept, int E) {
-    return (ept == 16 && E >= 15 && E <= 19) || (ept == 32 && E == 21);
+    return (ept == 16 && E >= 15 && E <= 20) || (ept == 32 && (E == 21 || E == 22));
 }
 
 struct TlcPass {

@@ -54,6 +54,32 @@ def test_virtual_ranks(P, G, k, no_tma):
                 pl.close()
 
 
+@pytest.mark.parametrize("G", [2, 8])
+def test_virtual_ranks_tlc_compact_2pow24(P, G):
+    # the row-sharded TLC form with the compact entries that are the default from 2^23 on
+    from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
+    n = 1 << 24
+    shard = n // G
+    a = W.make_data(n)
+    for fam in ("random", "bitrev"):
+        p = W.make_perm(fam, n, seed=G)
+        plans = [P.Plan(p, world=G, rank=g) for g in range(G)]
+        try:
+            info = plans[0].info()
+            assert info["passes"] == 3 and max(info["entry_bits"]) < 2 * 13 - 5 + 2, info
+            a_sh = [torch.from_numpy(a[g * shard:(g + 1) * shard].view(np.int32).copy()).cuda() for g in range(G)]
+            b_sh = [torch.full((shard,), -1, dtype=torch.int32, device="cuda") for _ in range(G)]
+            send = [torch.empty(shard, dtype=torch.int32, device="cuda") for _ in range(G)]
+            recv = [torch.empty(shard, dtype=torch.int32, device="cuda") for _ in range(G)]
+            apply_virtual(plans, a_sh, b_sh, send, recv)
+            torch.cuda.synchronize()
+            b = np.concatenate([x.cpu().numpy().view(np.uint32) for x in b_sh])
+            assert np.array_equal(b, OA.apply_ref(p, a)), (fam, G)
+        finally:
+            for pl in plans:
+                pl.close()
+
+
 def test_sharded_step_errors(P):
     n = 1 << 16
     with P.Plan(W.random(n, 1), world=2, rank=0) as pl:
