@@ -523,6 +523,7 @@ int perm_plan_set_tracing(perm_plan* plan, int enable) {
         mx = std::max<int64_t>(mx, rp.tma ? rp.grid : rp.ctas);
     }
     mx = std::max<int64_t>(mx, plan->host.fused3_grid);
+    mx = std::max<int64_t>(mx, plan->host.cluster);
     plan->trace_stride = mx;
     cudaError_t e = cudaMalloc(&plan->d_trace, (size_t)(3 * mx * 16) * sizeof(unsigned long long));
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc trace");
@@ -621,7 +622,7 @@ int perm_apply(const perm_plan* plan_c, const void* a, void* b, perm_stream_t st
         mark();
     } else if (P.passes == 2) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};
-        e = perm::launch_cluster(P, sc, in, out, s);
+        e = perm::launch_cluster(P, sc, in, out, s, tr(0));
         mark();
     } else if (P.layout == 3 && P.fused3) {
         const uint32_t* sc[3] = {plan->d_phase[0], plan->d_phase[1], plan->d_phase[2]};

@@ -1492,6 +1492,11 @@ __device__ __forceinline__ uint32_t cluster_size() {
 __device__ __forceinline__ void cluster_arrive() {
     asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
 }
+// arrive without release semantics: for barriers whose only job is to order async-proxy
+// (bulk copy) completions that every block has already observed on its own mbarrier
+__device__ __forceinline__ void cluster_arrive_relaxed() {
+    asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+}
 __device__ __forceinline__ void cluster_wait() {
     asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
@@ -1547,6 +1552,7 @@ struct ClusterArgs {
     uint32_t* out;
     const uint32_t* sched[3];
     long long tile_words;        // schedule words of one block's share of a phase
+    unsigned long long* trace;   // optional %globaltimer stamps [block][16]
 };
 
 // Thm 9 (L537-L539) in ONE launch for arrays that fit in one cluster's shared memory
@@ -1601,6 +1607,7 @@ __global__ void __launch_bounds__(kTlcPerm, 1) cluster_kernel(const ClusterArgs 
         }
     }
     __syncthreads();
+    stamp(a.trace, 0);
     cluster_arrive();                       // (A) mbarriers initialised and armed
     uint32_t wc[NWORDS];
     // lane's schedule words of phase f: coalesced (word w of lane x at (warp*NWORDS + w)*32 + x)
@@ -1617,12 +1624,15 @@ __global__ void __launch_bounds__(kTlcPerm, 1) cluster_kernel(const ClusterArgs 
     };
     if constexpr (!SMEM_SCHED) load_sched(0);
     mbar_wait(&bar[0], 0);
+    stamp(a.trace, 1);
     if constexpr (SMEM_SCHED) load_sched(0);
     block_permute<EPT, LOGS>(buf0, buf1, wc, lane, buf2, g, logBw);   // phase 1 (own block -> buf2)
     fence_proxy_async();                    // generic writes of buf1 -> the bulk copies' reads
     if constexpr (!SMEM_SCHED) load_sched(1);
     __syncthreads();
+    stamp(a.trace, 2);
     cluster_wait();                         // (A): every peer's mbarriers are armed
+    stamp(a.trace, 3);
     if (tid == 0) {
         const uint32_t dst0 = smem_u32(buf2 + g * Bw), mb = smem_u32(&bar[1]);
         for (uint32_t q = 0; q < C; ++q)
@@ -1633,28 +1643,38 @@ __global__ void __launch_bounds__(kTlcPerm, 1) cluster_kernel(const ClusterArgs 
         load_sched(1);
     }
     mbar_wait(&bar[1], 0);                  // exchange 1 landed in buf2
-    cluster_arrive();                       // (B) my copies into buf2 are complete
+    stamp(a.trace, 4);
+    // (B) exchange 1 into me is complete. Passing (B) tells a block that every exchange-1
+    // copy (hence every read out of its buf1) has completed: completions each block observed
+    // on its own mbarrier (complete_tx), so no release of generic writes is needed here
+    cluster_arrive_relaxed();
     block_permute<EPT, LOGS>(buf2, buf0, wc, lane, buf1, g, logBw);   // phase 2 (own block -> buf1)
     fence_proxy_async();
     load_sched(2);
     __syncthreads();
+    stamp(a.trace, 5);
     cluster_wait();                         // (B): every block received exchange 1 -> every buf1 is free
+    stamp(a.trace, 6);
     if (tid == 0) {
         const uint32_t dst0 = smem_u32(buf1 + g * Bw), mb = smem_u32(&bar[2]);
         for (uint32_t q = 0; q < C; ++q)
             if (q != g) bulk_s2cluster(map_to(dst0, q), buf0 + q * Bw, Bw * 4u, map_to(mb, q));
     }
     mbar_wait(&bar[2], 0);                  // exchange 2 landed in buf1
-    cluster_arrive();                       // (C) my copies into buf1 are complete
+    stamp(a.trace, 7);
+    cluster_arrive_relaxed();               // (C) exchange 2 into me is complete (lifetime only)
     block_permute<EPT, LOGS>(buf1, buf2, wc, lane);               // phase 3
     fence_proxy_async();
     __syncthreads();
     if (tid == 0) {
+        stamp(a.trace, 8);
         bulk_s2g(a.out + (size_t)g * S, buf2, (uint32_t)S * 4u);
         bulk_commit();
         bulk_wait_read0();
+        stamp(a.trace, 9);
     }
     cluster_wait();                         // (C): no peer still reads my buf0 before I exit
+    stamp(a.trace, 10);
 }
 
 // ------------------------------------------------------------------ transpose
@@ -2137,8 +2157,9 @@ size_t cluster_smem(const HostPlan& P) {
 }
 
 cudaError_t launch_cluster(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
-                           uint32_t* b, cudaStream_t s) {
+                           uint32_t* b, cudaStream_t s, unsigned long long* trace) {
     ClusterArgs ca{};
+    ca.trace = trace;
     ca.in = a;
     ca.out = b;
     for (int f = 0; f < 3; ++f) ca.sched[f] = sched[f];

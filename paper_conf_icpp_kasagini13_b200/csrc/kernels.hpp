@@ -20,7 +20,7 @@ cudaError_t launch_fused(const HostPlan& P, const uint32_t* const sched[3], cons
 // Cluster path (n = 2^15..2^18): one launch of one cluster of P.cluster blocks; all three
 // phases in distributed shared memory, the column phase's transposes as block exchanges.
 cudaError_t launch_cluster(const HostPlan& P, const uint32_t* const sched[3], const uint32_t* a,
-                           uint32_t* b, cudaStream_t s);
+                           uint32_t* b, cudaStream_t s, unsigned long long* trace = nullptr);
 
 // One row pass (pass index f in 0..2) of the 3- or 5-pass pipeline.
 // `trace`: optional device buffer of 16 %globaltimer stamps per CTA (nullptr = off).
