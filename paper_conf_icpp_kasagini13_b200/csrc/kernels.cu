@@ -64,6 +64,19 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
                  "r"(bytes)
                  : "memory");
 }
+// polling wait with a sleep between probes: for a lone thread that waits for a long time
+// (it stops competing for issue slots with the warps doing the work on its SM sub-partition)
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_sleepy(uint64_t* bar, uint32_t parity, unsigned ns) {
+    while (!mbar_test(bar, parity)) __nanosleep(ns);
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n\t.reg .pred p;\n"
@@ -1349,7 +1362,7 @@ __global__ void __launch_bounds__(64 + kTlcPerm, 1)
                 if (k < 2) {
                     // pass k + 1's schedules once this CTA's pass-k stores are complete: HBM is
                     // then free of this CTA's pass-k traffic, and the prefetch overlaps the barrier
-                    mbar_wait(&pdone[k], 0);
+                    mbar_wait_sleepy(&pdone[k], 0, 200);
                     for (int i = 0; i < my_tiles(k + 1); ++i) prefetch_one(k + 1, i);
                 }
             }
