@@ -550,7 +550,9 @@ int build_tlc(HostPlan& P, const U16Buf* phi, const perm_plan_options* opt,
         // 41.0 / 90.3 us against 47.5 / 98.0 us with h1 = h3 = 4 (profiles/r02_ab_mid.jsonl).
         // Up to 2^19, 8192-word tiles leave SMs idle (32 / 64 tiles per pass at 2^18 / 2^19 on
         // 148 SMs): 4096-word tiles, 14.7 -> 13.3 us and 15.5 -> 13.4 us (profiles/r02_ab_small.jsonl).
-        const int64_t T = P.k <= 19 ? 4096 : (P.k <= 24 ? 8192 : 16384);
+        // At 2^21 4096-word tiles (h = 2, 4, 2; 512 tiles per pass) beat 8192-word ones (h = 4,
+        // 8, 4): 19.44 -> 18.99 us (profiles/r02b_tiles_21.log); equal at 2^20.
+        const int64_t T = (P.k <= 19 || P.k == 21) ? 4096 : (P.k <= 24 ? 8192 : 16384);
         int64_t h = (opt && (&opt->h1)[f] > 0)
                         ? (&opt->h1)[f]
                         : (P.k <= 24 ? std::max<int64_t>(f == 1 ? 4 : 2, T / L) : std::max<int64_t>(1, T / L));

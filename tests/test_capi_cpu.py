@@ -209,8 +209,10 @@ def test_tlc_full_and_compact_formats_agree(lib, k):
     n = 1 << k
     r, c = W.view_shape(n)
     p = W.make_perm("random", n, seed=k)
-    i_full, _, kappa_f, s_full = export_tlc(lib, p, sched_format=-1)
-    i_cmp, _, kappa_c, s_cmp = export_tlc(lib, p, sched_format=1)
+    # 8192-word tiles (the default at 2^21 is 4096-word tiles, which have no compact kernel)
+    h = (4, 8, 4) if k == 21 else (0, 0, 0)
+    i_full, _, kappa_f, s_full = export_tlc(lib, p, sched_format=-1, h=h)
+    i_cmp, _, kappa_c, s_cmp = export_tlc(lib, p, sched_format=1, h=h)
     assert np.array_equal(kappa_f, kappa_c)
     for a, b in zip(s_full, s_cmp):
         assert np.array_equal(a, b)

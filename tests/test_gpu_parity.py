@@ -365,7 +365,7 @@ def test_tlc_rings_wrap(P, k, h, stages, fuse, log2c):
 
 
 @pytest.mark.parametrize("fmt", [-1, 0, 1])
-@pytest.mark.parametrize("k", [15, 17, 20, 22, 23, 25])
+@pytest.mark.parametrize("k", [15, 17, 20, 21, 22, 23, 25])
 def test_tlc_entry_formats(P, k, fmt):
     # full (source row << log2 tile | destination) vs compact (line index implied) entries
     n = 1 << k

@@ -29,7 +29,7 @@ def P():
 
 @pytest.mark.parametrize("no_tma", [0, 1, -1, -2])
 @pytest.mark.parametrize("G", [1, 2, 4, 8])
-@pytest.mark.parametrize("k", [16, 19, 22])
+@pytest.mark.parametrize("k", [16, 19, 21, 22])
 def test_virtual_ranks(P, G, k, no_tma):
     from paper_conf_icpp_kasagini13_b200.sharded import apply_virtual
     n = 1 << k
